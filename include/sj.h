@@ -1,0 +1,176 @@
+/*
+ * sj.h -- C ABI of the B200-native eps-grid similarity self-join (libsj.so).
+ *
+ * Method: Gallet & Gowanlock, "Load Imbalance Mitigation Optimizations for
+ * GPU-Accelerated Similarity Joins", IPDPSW 2019.  Citations are
+ * PAPER.md line numbers ("P:L") plus the section / algorithm they fall in.
+ *
+ * The operation (§II-A): for a dataset D of n points in `dim` dimensions,
+ * return every ordered pair (i, j), i != j, with dist(p_i, p_j) <= eps.  The
+ * predicate is evaluated exactly as s(i,j) <= fl(eps*eps), where
+ * s = fl(...fl(fl(t_0*t_0) + fl(t_1*t_1)) + ...), t_d = fl(p_i[d] - p_j[d]),
+ * IEEE binary64 round-to-nearest, dimension order, no FMA (DESIGN.md readings
+ * c1, c2).  Self pairs are excluded; exact duplicates i != j are pairs (c3).
+ * Both (i, j) and (j, i) are returned (mirrored emission, c4).
+ *
+ * The hot path behind these calls: eps-grid index with a radix
+ * sort of point->cell ids, per-cell workload,
+ * SortByWL, an atomic WorkQueue over D', k threads per
+ * query point with the LID-UNICOMP cell pattern (P:172-185,
+ * Alg. 3), warp-shuffle cooperation and batched result emission with a
+ * 1 % batch estimator.
+ *
+ * Threading: a handle is not thread-safe; distinct handles are independent.
+ * Every call runs on the CUDA device that was current when the handle was
+ * created.  All calls are synchronous: they return after their GPU work ended.
+ */
+#ifndef SJ_H
+#define SJ_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SJ_ABI_VERSION 1
+
+typedef struct sj_handle sj_handle;
+
+/* Return codes. */
+enum sj_status {
+    SJ_OK = 0,       /* join complete; *count pairs written by this call            */
+    SJ_MORE = 1,     /* out_pairs filled to cap; call sj_self_join again to continue */
+    SJ_EINVAL = -1,  /* bad argument (NULL, dim, n, eps, non-finite coordinate, ...) */
+    SJ_ENOMEM = -2,  /* device or pinned host allocation failed                     */
+    SJ_ECUDA = -3,   /* CUDA runtime error (no device, launch failure, ...)         */
+    SJ_EGRID = -4,   /* grid too large: some nc_d >= 2^30 or prod nc_d >= 2^64     */
+    SJ_ESTATE = -5   /* handle is in the error state after an earlier failure       */
+};
+
+/* Options for sj_set_option (set them before the sj_self_join they should affect). */
+enum sj_option {
+    SJ_OPT_K = 1,              /* threads per query point k in {1,2,4,8,16,32}; default 8 */
+    SJ_OPT_BATCH_PAIRS = 2,    /* b_s, pairs per batch buffer; default 1e8                        */
+    SJ_OPT_STREAMS = 3,        /* CUDA streams for batches, 1..8; default 3                       */
+    SJ_OPT_SAMPLE_PPM = 4,     /* estimator sample of D' in parts per million; default 10000 = 1%*/
+    SJ_OPT_GRAB = 5,           /* queue positions one warp dequeues per atomic; multiple of 32/k; 32     */
+    SJ_OPT_COUNT_CALCS = 6,    /* 1 = instrument the join with a distance-calculation counter; default 0 */
+    SJ_OPT_BLOCKS_PER_SM = 7,  /* persistent-grid CTAs per SM; 0 = occupancy maximum (default)           */
+    SJ_OPT_FAST_PATH = 8       /* 1 = device output written in place when it fits (default); 0 = always
+                                  stage per batch (the paper's scheme)                             */
+};
+
+/* Statistics of the handle (sj_get_stats).  Times are CUDA-event milliseconds. */
+typedef struct sj_stats {
+    uint64_t n;               /* points                                              */
+    uint32_t dim;             /* dimensionality                                      */
+    uint32_t key_bits;        /* significant bits of the linear cell id              */
+    uint64_t n_cells;         /* M, non-empty cells (|B|)                      */
+    uint64_t fwd_entries;     /* sum over cells of non-empty forward neighbours      */
+    uint64_t dist_calcs;      /* D_alg: distance calculations of the LID-UNICOMP
+                                 pattern, sum_A [C(m_A,2) + m_A * sum_fwd m_B]       */
+    uint64_t calcs_measured;  /* instrumented counter of the last join (0 if off)    */
+    uint64_t pairs;           /* ordered pairs of the last completed join            */
+    uint64_t est_pairs;       /* batch estimator's estimate                  */
+    uint32_t batches;         /* nbBatches of the last join                          */
+    uint32_t retries;         /* overflow re-runs of the last join                   */
+    uint32_t join_launches;   /* join kernel launches of the last join               */
+    uint32_t k;               /* threads per query point used                        */
+    uint64_t max_cell_load;   /* largest per-point workload W                */
+    double ms_build;          /* sj_create: upload .. SortByWL (device span)         */
+    double ms_estimate;       /* estimator kernel                                    */
+    double ms_join;           /* join kernels: device span first start .. last end   */
+    double ms_join_sum;       /* join kernels: sum of per-launch durations           */
+    double ms_transfer;       /* copies of staged batches to the caller's buffer     */
+    double ms_total;          /* last sj_self_join call, device span                 */
+    uint32_t fast_path;       /* 1 if the last join wrote the caller's device buffer in place */
+    uint32_t nc[8];           /* cells per dimension                                 */
+} sj_stats;
+
+/* Build the eps-grid index of `n` points of dimension `dim` (row-major AoS,
+ * points[i*dim + d]) with threshold `eps`.
+ *   points : host (pageable or pinned) or device pointer on the current device;
+ *            read only during the call -- the library copies it (caller keeps ownership).
+ *   n      : 1 <= n < 2^32.      dim : 1 <= dim <= 8 (the paper uses 2..6).
+ *   eps    : finite, > 0.
+ * Runs steps a1..a8 of DESIGN.md §1 (upload+validate, bounding box, cell
+ * linearisation, radix sort, compaction, forward neighbours, workload, SortByWL).
+ * Returns NULL on error (see sj_last_error): NaN/Inf coordinate or bad argument
+ * (SJ_EINVAL), grid overflow (SJ_EGRID), allocation (SJ_ENOMEM), CUDA (SJ_ECUDA). */
+sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps);
+
+/* Run (or continue) the self-join.
+ *   out_pairs : caller-owned uint32[2*cap], interleaved (i, j) of 0-based input ids,
+ *               host (pinned or pageable) or device memory; a device buffer must be
+ *               16-byte aligned.  Order is unspecified; each unordered neighbour pair
+ *               appears as (i, j) and (j, i); (i, i) never appears.
+ *   cap       : capacity in pairs.
+ *   count     : receives the number of pairs written by THIS call.
+ * out_pairs == NULL && cap == 0 : count-only; *count = total pairs, nothing written.
+ * Returns SJ_OK when the join is complete, SJ_MORE when cap was filled and pairs
+ * remain (call again with the same or another buffer to receive the next ones).
+ * A call after SJ_OK restarts the join; the pair SET is deterministic.
+ * Errors: SJ_EINVAL (NULL count, out_pairs NULL with cap > 0, misaligned device
+ * buffer), SJ_ECUDA, SJ_ENOMEM; after an error the handle answers SJ_ESTATE. */
+int sj_self_join(sj_handle *h, uint32_t *out_pairs, uint64_t cap, uint64_t *count);
+
+/* Free every device / pinned resource of the handle.  NULL-safe. */
+void sj_destroy(sj_handle *h);
+
+/* Text of the last error raised on the calling thread ("" if none). */
+const char *sj_last_error(void);
+
+/* Set an option (enum sj_option).  Returns SJ_OK or SJ_EINVAL (unknown option /
+ * out-of-range value).  Takes effect at the next sj_self_join that (re)starts. */
+int sj_set_option(sj_handle *h, int opt, int64_t value);
+
+/* Restrict this handle to the queue slice of `rank` out of `world` replicas
+ * (multi-GPU): D' is cut into chunks of SJ_OPT_GRAB positions and
+ * chunk c belongs to rank c mod world.  Slices of all ranks are disjoint and
+ * cover D'; each slice's pairs are disjoint (every unordered pair is evaluated
+ * by exactly one query point).  world = 1 restores the whole queue. */
+int sj_set_slice(sj_handle *h, int rank, int world);
+
+/* Copy the statistics of the handle into *s. */
+int sj_get_stats(const sj_handle *h, sj_stats *s);
+
+/* Serialise the built index (header + device arrays) into one contiguous blob
+ * for an NCCL broadcast.  dst: device or host pointer of cap bytes, or NULL to
+ * only query the size in *bytes. */
+int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes);
+
+/* Create a handle from a blob produced by sj_export_index (device or host
+ * pointer, possibly on another GPU / process).  NULL on error. */
+sj_handle *sj_create_from_index(const void *blob, uint64_t bytes);
+
+/* ABI version (SJ_ABI_VERSION). */
+int sj_abi_version(void);
+
+/* ---- host-only helpers (no GPU needed) ------------------------------------ */
+
+/* LID-UNICOMP forward offsets (Alg. 3): the neighbour offsets o in
+ * {-1,0,1}^dim whose cell has a higher row-major linear id than the origin, i.e.
+ * whose first non-zero component is +1.  Writes F*dim int8 values (F = (3^dim-1)/2)
+ * if out != NULL and cap >= F*dim.  Returns F, or SJ_EINVAL. */
+int sj_forward_offsets(int dim, int8_t *out, uint64_t cap);
+
+/* Queue positions of slice (rank, world) for n points and chunk `grab`:
+ * writes them ascending into out (if out != NULL and cap is large enough) and
+ * returns their number, or a negative sj_status. */
+int64_t sj_slice_positions(uint64_t n, uint32_t grab, int rank, int world, uint32_t *out, uint64_t cap);
+
+/* ---- diagnostics (GPU microbenchmarks for the roofline denominators) ------ */
+
+/* FP64 pipe throughput of the current device: DADD/DMUL dependent chains on all
+ * SMs; *instr_per_s receives FP64 warp-lane instructions per second.  */
+int sj_measure_fp64(double *instr_per_s, double *ms);
+
+/* Same-address global atomicAdd rate (one lane per warp), ops per second. */
+int sj_measure_atomics(double *ops_per_s, double *ms);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SJ_H */

@@ -1,0 +1,270 @@
+"""ctypes marshalling for libsj.so (include/sj.h).  No computation happens here."""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_ROOT = os.path.dirname(_HERE)
+lib_path = os.path.join(_HERE, "libsj.so")
+HEADER = os.path.join(_ROOT, "include", "sj.h")
+
+SJ_OK, SJ_MORE, SJ_EINVAL, SJ_ENOMEM, SJ_ECUDA, SJ_EGRID, SJ_ESTATE = 0, 1, -1, -2, -3, -4, -5
+(SJ_OPT_K, SJ_OPT_BATCH_PAIRS, SJ_OPT_STREAMS, SJ_OPT_SAMPLE_PPM, SJ_OPT_GRAB, SJ_OPT_COUNT_CALCS,
+ SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH) = range(1, 9)
+_NAMES = {0: "SJ_OK", 1: "SJ_MORE", -1: "SJ_EINVAL", -2: "SJ_ENOMEM", -3: "SJ_ECUDA", -4: "SJ_EGRID",
+          -5: "SJ_ESTATE"}
+
+
+class SJError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{_NAMES.get(code, code)}: {msg}")
+        self.code = code
+
+
+class SJStats(ctypes.Structure):
+    _fields_ = [
+        ("n", ctypes.c_uint64), ("dim", ctypes.c_uint32), ("key_bits", ctypes.c_uint32),
+        ("n_cells", ctypes.c_uint64), ("fwd_entries", ctypes.c_uint64), ("dist_calcs", ctypes.c_uint64),
+        ("calcs_measured", ctypes.c_uint64), ("pairs", ctypes.c_uint64), ("est_pairs", ctypes.c_uint64),
+        ("batches", ctypes.c_uint32), ("retries", ctypes.c_uint32), ("join_launches", ctypes.c_uint32),
+        ("k", ctypes.c_uint32), ("max_cell_load", ctypes.c_uint64),
+        ("ms_build", ctypes.c_double), ("ms_estimate", ctypes.c_double), ("ms_join", ctypes.c_double),
+        ("ms_join_sum", ctypes.c_double), ("ms_transfer", ctypes.c_double), ("ms_total", ctypes.c_double),
+        ("fast_path", ctypes.c_uint32), ("nc", ctypes.c_uint32 * 8),
+    ]
+
+    def as_dict(self) -> dict:
+        d = {f[0]: getattr(self, f[0]) for f in self._fields_}
+        d["nc"] = list(self.nc)[: self.dim]
+        return d
+
+
+if not os.path.exists(lib_path):
+    raise ImportError(f"{lib_path} is not built: run `python -c 'import __graft_entry__ as g; g.build()'` "
+                      "(the CUDA path has no CPU fallback)")
+
+_lib = ctypes.CDLL(lib_path)
+_vp, _u64, _i64, _int, _dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int, ctypes.c_double
+_sig = {
+    "sj_abi_version": (_int, []),
+    "sj_last_error": (ctypes.c_char_p, []),
+    "sj_create": (_vp, [_vp, _u64, _int, _dbl]),
+    "sj_self_join": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
+    "sj_destroy": (None, [_vp]),
+    "sj_set_option": (_int, [_vp, _int, _i64]),
+    "sj_set_slice": (_int, [_vp, _int, _int]),
+    "sj_get_stats": (_int, [_vp, ctypes.POINTER(SJStats)]),
+    "sj_export_index": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
+    "sj_create_from_index": (_vp, [_vp, _u64]),
+    "sj_forward_offsets": (_int, [_int, _vp, _u64]),
+    "sj_slice_positions": (_i64, [_u64, ctypes.c_uint32, _int, _int, _vp, _u64]),
+    "sj_measure_fp64": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
+    "sj_measure_atomics": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
+}
+for _n, (_r, _a) in _sig.items():
+    _f = getattr(_lib, _n)
+    _f.restype = _r
+    _f.argtypes = _a
+
+
+def header_functions() -> list:
+    """Function names declared in include/sj.h (for the symbol-export test)."""
+    txt = open(HEADER).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(sj_[a-z0-9_]+)\s*\(", txt)))
+
+
+def _ptr(x) -> int:
+    """Raw address of a numpy array, torch tensor, ctypes buffer or int (None -> 0)."""
+    if x is None:
+        return 0
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return int(x.data_ptr())
+    if hasattr(x, "ctypes"):
+        return int(x.ctypes.data)
+    return ctypes.addressof(x)
+
+
+def _err(code: int) -> SJError:
+    return SJError(code, (_lib.sj_last_error() or b"").decode())
+
+
+def _check(code: int) -> int:
+    if code < 0:
+        raise _err(code)
+    return code
+
+
+# ------------------------------------------------------------------ same-name wrappers
+
+def sj_abi_version() -> int:
+    return _lib.sj_abi_version()
+
+
+def sj_last_error() -> str:
+    return (_lib.sj_last_error() or b"").decode()
+
+
+def sj_create(points, n: int | None = None, dim: int | None = None, eps: float | None = None) -> int:
+    """sj_create(points, eps) or sj_create(ptr, n, dim, eps).  Returns the raw handle (int)."""
+    if eps is None:  # (points, eps) form
+        eps = n
+        shape = tuple(points.shape)
+        if len(shape) != 2:
+            raise ValueError("points must be (N, dim)")
+        n, dim = shape
+        if hasattr(points, "dtype") and str(points.dtype) not in ("float64", "torch.float64"):
+            raise TypeError("points must be float64")
+        if hasattr(points, "is_contiguous") and not points.is_contiguous():
+            raise ValueError("points must be contiguous")
+        if hasattr(points, "flags") and not points.flags["C_CONTIGUOUS"]:
+            raise ValueError("points must be C-contiguous")
+    h = _lib.sj_create(_ptr(points), int(n), int(dim), float(eps))
+    if not h:
+        raise SJError(SJ_EINVAL, sj_last_error())
+    return h
+
+
+def sj_create_from_index(blob, nbytes: int) -> int:
+    h = _lib.sj_create_from_index(_ptr(blob), int(nbytes))
+    if not h:
+        raise SJError(SJ_EINVAL, sj_last_error())
+    return h
+
+
+def sj_self_join(h: int, out, cap: int):
+    """Returns (status, count) with status SJ_OK or SJ_MORE; raises SJError on error."""
+    cnt = _u64(0)
+    rc = _lib.sj_self_join(h, _ptr(out), int(cap), ctypes.byref(cnt))
+    _check(rc)
+    return rc, int(cnt.value)
+
+
+def sj_destroy(h: int) -> None:
+    _lib.sj_destroy(h)
+
+
+def sj_set_option(h: int, opt: int, value: int) -> None:
+    _check(_lib.sj_set_option(h, int(opt), int(value)))
+
+
+def sj_set_slice(h: int, rank: int, world: int) -> None:
+    _check(_lib.sj_set_slice(h, int(rank), int(world)))
+
+
+def sj_get_stats(h: int) -> dict:
+    st = SJStats()
+    _check(_lib.sj_get_stats(h, ctypes.byref(st)))
+    return st.as_dict()
+
+
+def sj_export_index(h: int, dst=None, cap: int = 0) -> int:
+    nbytes = _u64(0)
+    _check(_lib.sj_export_index(h, _ptr(dst), int(cap), ctypes.byref(nbytes)))
+    return int(nbytes.value)
+
+
+def sj_forward_offsets(dim: int):
+    import numpy as np
+
+    f = _check(_lib.sj_forward_offsets(int(dim), None, 0))
+    out = np.zeros((f, dim), dtype=np.int8)
+    _check(_lib.sj_forward_offsets(int(dim), out.ctypes.data, out.size))
+    return out
+
+
+def sj_slice_positions(n: int, grab: int, rank: int, world: int):
+    import numpy as np
+
+    cnt = _check(_lib.sj_slice_positions(int(n), int(grab), int(rank), int(world), None, 0))
+    out = np.zeros(max(cnt, 1), dtype=np.uint32)
+    _check(_lib.sj_slice_positions(int(n), int(grab), int(rank), int(world), out.ctypes.data, out.size))
+    return out[:cnt]
+
+
+def sj_measure_fp64():
+    r, ms = _dbl(0), _dbl(0)
+    _check(_lib.sj_measure_fp64(ctypes.byref(r), ctypes.byref(ms)))
+    return r.value, ms.value
+
+
+def sj_measure_atomics():
+    r, ms = _dbl(0), _dbl(0)
+    _check(_lib.sj_measure_atomics(ctypes.byref(r), ctypes.byref(ms)))
+    return r.value, ms.value
+
+
+# ------------------------------------------------------------------ RAII convenience
+
+class Handle:
+    """Owning wrapper of an sj_handle*."""
+
+    def __init__(self, points=None, eps: float | None = None, *, raw: int | None = None, **options):
+        self.h = raw if raw is not None else sj_create(points, eps)
+        for k, v in options.items():
+            self.set_option(k, v)
+
+    @classmethod
+    def from_index(cls, blob, nbytes: int) -> "Handle":
+        return cls(raw=sj_create_from_index(blob, nbytes))
+
+    _OPTS = {"k": SJ_OPT_K, "batch_pairs": SJ_OPT_BATCH_PAIRS, "streams": SJ_OPT_STREAMS,
+             "sample_ppm": SJ_OPT_SAMPLE_PPM, "grab": SJ_OPT_GRAB, "count_calcs": SJ_OPT_COUNT_CALCS,
+             "blocks_per_sm": SJ_OPT_BLOCKS_PER_SM, "fast_path": SJ_OPT_FAST_PATH}
+
+    def set_option(self, name, value) -> None:
+        sj_set_option(self.h, self._OPTS[name] if isinstance(name, str) else name, int(value))
+
+    def set_slice(self, rank: int, world: int) -> None:
+        sj_set_slice(self.h, rank, world)
+
+    def self_join(self, out=None, cap: int = 0):
+        return sj_self_join(self.h, out, cap)
+
+    def count(self) -> int:
+        return sj_self_join(self.h, None, 0)[1]
+
+    def stats(self) -> dict:
+        return sj_get_stats(self.h)
+
+    def export_index(self, dst=None, cap: int = 0) -> int:
+        return sj_export_index(self.h, dst, cap)
+
+    def close(self) -> None:
+        if getattr(self, "h", None):
+            sj_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def self_join_pairs(handle: Handle, device: str = "cuda", total: int | None = None):
+    """All pairs as a torch int32 tensor (M, 2) holding the uint32 ids (count-only call
+    first to size the buffer, then one sj_self_join into it)."""
+    import torch
+
+    if total is None:
+        total = handle.count()
+    if device == "cpu":
+        out = torch.empty((max(total, 1), 2), dtype=torch.int32, pin_memory=True)
+    else:
+        out = torch.empty((max(total, 1), 2), dtype=torch.int32, device=device)
+    got, rc = 0, SJ_MORE
+    rc, got = handle.self_join(out, max(total, 1))
+    if rc != SJ_OK:
+        raise SJError(rc, "unexpected SJ_MORE with an exactly sized buffer")
+    return out[:got]

@@ -1,0 +1,664 @@
+// grid_build.cu -- the eps-grid index I built on the GPU, plus the
+// per-cell workload and SortByWL.  Steps a2..a8 of
+// DESIGN.md §1:
+//   a2 bounding box (exact min/max per dimension)
+//   a3 cell linearisation  c_d = floor(fl(fl(x_d - min_d) / w)),  w = eps(1+2^-20)
+//      (readings c5, c6); lid = sum_d c_d * stride_d, row-major, dim 0 most significant (c7)
+//   a4 hand-written radix sort of (lid, point id) on the significant bits
+//   a5 run-length compaction -> non-empty cells B + point lookup
+//   a6 LID-UNICOMP forward neighbours (Alg. 3) resolved once per cell
+//   a7 workload W(A) = ceil((m_A-1)/2) + sum_{B in fwd(A)} m_B and D_alg
+//   a8 SortByWL: cells in non-increasing W (stable, ties by lid, c10) -> D' storage order
+#include <cmath>
+#include <cstring>
+#include <vector>
+
+#include "sj_internal.cuh"
+
+namespace sj {
+
+__constant__ uint64_t c_fwd_off[SJ_MAX_FWD];   // packed int8 offsets, dim d in byte d
+__constant__ long long c_fwd_delta[SJ_MAX_FWD];  // sum_d o_d * stride_d
+
+namespace {
+
+constexpr int kThreads = 256;
+
+inline unsigned grid_for(uint64_t n, int threads = kThreads) {
+    uint64_t b = (n + threads - 1) / threads;
+    if (b == 0) b = 1;
+    return (unsigned)b;
+}
+
+__device__ __forceinline__ unsigned long long ordered_key(double x) {
+    unsigned long long b = (unsigned long long)__double_as_longlong(x);
+    return (b >> 63) ? ~b : (b | 0x8000000000000000ull);
+}
+__host__ __device__ inline double from_ordered_key(unsigned long long k) {
+    unsigned long long b = (k >> 63) ? (k & 0x7FFFFFFFFFFFFFFFull) : ~k;
+    double d;
+    memcpy(&d, &b, sizeof d);
+    return d;
+}
+
+struct BBox {
+    unsigned long long mn[SJ_MAX_DIM];
+    unsigned long long mx[SJ_MAX_DIM];
+    unsigned int nonfinite;
+};
+
+__global__ void bbox_init_kernel(BBox *bb) {
+    int t = threadIdx.x;
+    if (t < SJ_MAX_DIM) {
+        bb->mn[t] = ~0ull;
+        bb->mx[t] = 0ull;
+    }
+    if (t == 0) bb->nonfinite = 0;
+}
+
+// a2: exact per-dimension min/max (order-independent) + non-finite check (a1 validation)
+__global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint64_t n, int dim, BBox *bb) {
+    unsigned long long mn[SJ_MAX_DIM], mx[SJ_MAX_DIM];
+#pragma unroll
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        mn[d] = ~0ull;
+        mx[d] = 0ull;
+    }
+    unsigned bad = 0;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+        for (int d = 0; d < SJ_MAX_DIM; ++d) {
+            if (d < dim) {
+                double x = raw[i * dim + d];
+                if (!isfinite(x)) bad = 1;
+                unsigned long long k = ordered_key(x);
+                mn[d] = min(mn[d], k);
+                mx[d] = max(mx[d], k);
+            }
+        }
+    }
+#pragma unroll
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        if (d < dim) {
+            unsigned long long a = mn[d], b = mx[d];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                a = min(a, __shfl_xor_sync(0xffffffffu, a, o));
+                b = max(b, __shfl_xor_sync(0xffffffffu, b, o));
+            }
+            if ((threadIdx.x & 31) == 0) {
+                atomicMin(&bb->mn[d], a);
+                atomicMax(&bb->mx[d], b);
+            }
+        }
+    }
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(&bb->nonfinite, 1u);
+}
+
+struct GridGeom {
+    double mins[SJ_MAX_DIM];
+    unsigned long long nc[SJ_MAX_DIM];
+    unsigned long long stride[SJ_MAX_DIM];
+    double w;
+    int dim;
+};
+
+// a3: cell linearisation.  IEEE RN intrinsics so the result does not depend on
+// contraction flags (reading c1): c_d = floor( (x_d - min_d) / w ).
+template <class K>
+__global__ void __launch_bounds__(kThreads) cell_id_kernel(const double *raw, uint64_t n, GridGeom g, K *keys,
+                                                           uint32_t *vals) {
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    unsigned long long lid = 0;
+#pragma unroll
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        if (d < g.dim) {
+            double q = __ddiv_rn(__dsub_rn(raw[i * g.dim + d], g.mins[d]), g.w);
+            unsigned long long c = __double2ull_rd(q);
+            lid += c * g.stride[d];
+        }
+    }
+    keys[i] = (K)lid;
+    vals[i] = (uint32_t)i;
+}
+
+// a5: run-length flags over the sorted ids
+template <class K>
+__global__ void __launch_bounds__(kThreads) rle_flags_kernel(const K *ks, uint64_t n, uint32_t *flags) {
+    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    flags[p] = (p == 0 || ks[p] != ks[p - 1]) ? 1u : 0u;
+}
+
+template <class K>
+__global__ void __launch_bounds__(kThreads) rle_write_kernel(const K *ks, uint64_t n, uint32_t *excl_to_cellof,
+                                                             unsigned long long *cell_lid, uint32_t *cell_start) {
+    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    const bool flag = (p == 0 || ks[p] != ks[p - 1]);
+    const uint32_t ex = excl_to_cellof[p];
+    if (flag) {
+        cell_lid[ex] = (unsigned long long)ks[p];
+        cell_start[ex] = (uint32_t)p;
+    }
+    excl_to_cellof[p] = flag ? ex : ex - 1;  // point (sorted position) -> cell rank
+    if (p == n - 1) cell_start[ex + (flag ? 1 : 0)] = (uint32_t)n;
+}
+
+// ---------------------------------------------------------------- lid -> cell rank lookup
+struct Lookup {
+    const uint32_t *dense;           // dense table over all prod(nc) cells, or null
+    const unsigned long long *hkeys; // open-addressing hash (linear probing)
+    const uint32_t *hvals;
+    unsigned long long hmask;
+};
+
+__device__ __forceinline__ unsigned long long hash_lid(unsigned long long x) {
+    x ^= x >> 33;
+    x *= 0xff51afd7ed558ccdull;
+    x ^= x >> 33;
+    x *= 0xc4ceb9fe1a85ec53ull;
+    x ^= x >> 33;
+    return x;
+}
+
+__device__ __forceinline__ uint32_t lookup_cell(const Lookup &L, unsigned long long lid) {
+    if (L.dense) return L.dense[lid];
+    unsigned long long h = hash_lid(lid) & L.hmask;
+    for (;;) {
+        unsigned long long k = L.hkeys[h];
+        if (k == lid) return L.hvals[h];
+        if (k == ~0ull) return 0xFFFFFFFFu;
+        h = (h + 1) & L.hmask;
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) dense_fill_kernel(const unsigned long long *cell_lid, const uint64_t *d_M,
+                                                              uint32_t *dense) {
+    uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= *d_M) return;
+    dense[cell_lid[r]] = (uint32_t)r;
+}
+
+__global__ void __launch_bounds__(kThreads) hash_insert_kernel(const unsigned long long *cell_lid, const uint64_t *d_M,
+                                                               unsigned long long *hkeys, uint32_t *hvals,
+                                                               unsigned long long hmask) {
+    uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= *d_M) return;
+    unsigned long long lid = cell_lid[r];
+    unsigned long long h = hash_lid(lid) & hmask;
+    for (;;) {
+        unsigned long long prev = atomicCAS(&hkeys[h], ~0ull, lid);
+        if (prev == ~0ull || prev == lid) {
+            hvals[h] = (uint32_t)r;
+            return;
+        }
+        h = (h + 1) & hmask;
+    }
+}
+
+struct FwdGeom {
+    unsigned long long nc[SJ_MAX_DIM];
+    unsigned long long stride[SJ_MAX_DIM];
+    int dim;
+    int F;
+};
+
+struct BuildTotals {
+    unsigned long long M;
+    unsigned long long E;
+    unsigned long long dist_calcs;
+    unsigned int max_w;
+    unsigned int pad;
+};
+
+// a6 + a7: count the non-empty forward neighbours of every cell (Alg. 3: neighbour
+// cells with a higher linear id) and its workload W:
+//   W(A) = ceil((m_A - 1)/2)          (balanced circulant home-cell half scan, reading c8)
+//        + sum_{B in fwd(A)} m_B       (forward cells)
+// plus the exact distance-calculation total D_alg = sum_A C(m_A,2) + m_A sum m_B.
+template <bool FILL>
+__global__ void __launch_bounds__(kThreads) fwd_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
+                                                       const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *fcnt,
+                                                       uint32_t *wload, const uint32_t *fbegin, uint32_t *fwd_rank,
+                                                       BuildTotals *tot) {
+    const uint64_t M = *d_M;
+    const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned long long calcs = 0;
+    uint32_t w = 0;
+    if (r < M) {
+        const unsigned long long lid = cell_lid[r];
+        long long c[SJ_MAX_DIM];
+#pragma unroll
+        for (int d = 0; d < SJ_MAX_DIM; ++d)
+            if (d < g.dim) c[d] = (long long)((lid / g.stride[d]) % g.nc[d]);
+        const uint32_t m = cell_start[r + 1] - cell_start[r];
+        uint32_t cnt = 0;
+        unsigned long long summ = 0;
+        uint32_t out = FILL ? fbegin[r] : 0;
+        for (int j = 0; j < g.F; ++j) {
+            const unsigned long long off = c_fwd_off[j];
+            bool in = true;
+#pragma unroll
+            for (int d = 0; d < SJ_MAX_DIM; ++d) {
+                if (d < g.dim) {
+                    long long o = (long long)(signed char)((off >> (8 * d)) & 0xFF);
+                    long long v = c[d] + o;
+                    in = in && (v >= 0) && (v < (long long)g.nc[d]);
+                }
+            }
+            if (!in) continue;
+            const uint32_t nb = lookup_cell(L, lid + (unsigned long long)c_fwd_delta[j]);
+            if (nb == 0xFFFFFFFFu) continue;
+            if (FILL) {
+                fwd_rank[out++] = nb;
+            } else {
+                ++cnt;
+                summ += cell_start[nb + 1] - cell_start[nb];
+            }
+        }
+        if (!FILL) {
+            fcnt[r] = cnt;
+            w = (uint32_t)((m - 1 + 1) / 2 + summ);  // ceil((m-1)/2) + sum m_B
+            wload[r] = w;
+            calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
+        }
+    }
+    if (!FILL) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            calcs += __shfl_xor_sync(0xffffffffu, calcs, o);
+            w = max(w, __shfl_xor_sync(0xffffffffu, w, o));
+        }
+        if ((threadIdx.x & 31) == 0) {
+            if (calcs) atomicAdd(&tot->dist_calcs, calcs);
+            atomicMax(&tot->max_w, w);
+        }
+    }
+}
+
+// a8 (SortByWL): key = max_w - W so an ascending stable sort gives non-increasing W
+__global__ void __launch_bounds__(kThreads) wl_keys_kernel(const uint32_t *wload, uint64_t M, uint32_t max_w,
+                                                           uint32_t *keys, uint32_t *vals) {
+    uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= M) return;
+    keys[r] = max_w - wload[r];
+    vals[r] = (uint32_t)r;
+}
+
+__global__ void __launch_bounds__(kThreads) queue_m_kernel(const uint32_t *qorder, const uint32_t *cell_start,
+                                                           uint64_t M, uint32_t *mq) {
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= M) return;
+    uint32_t r = qorder[i];
+    mq[i] = cell_start[r + 1] - cell_start[r];
+}
+
+__global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t *qorder, const uint32_t *qb,
+                                                                  const uint32_t *cell_start, const uint32_t *fbegin,
+                                                                  const unsigned long long *cell_lid, uint64_t M,
+                                                                  uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
+                                                                  uint64_t *lid_q) {
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= M) return;
+    uint32_t r = qorder[i];
+    uint32_t m = cell_start[r + 1] - cell_start[r];
+    cellq[i] = make_uint4(qb[i], m, fbegin[r], fbegin[r + 1]);
+    r2q[r] = (uint32_t)i;
+    qbr[r] = qb[i];
+    lid_q[i] = cell_lid[r];
+}
+
+__global__ void __launch_bounds__(kThreads) fwd_convert_kernel(const uint32_t *fwd_rank, uint64_t E,
+                                                               const uint32_t *qbr, const uint32_t *cell_start,
+                                                               uint2 *fwd) {
+    uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= E) return;
+    uint32_t nb = fwd_rank[e];
+    fwd[e] = make_uint2(qbr[nb], cell_start[nb + 1] - cell_start[nb]);
+}
+
+// Gather points into D' storage order (padded AoS, `pad` doubles per point).
+__global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, uint64_t n, int dim, int pad,
+                                                           const uint32_t *idx_sorted, const uint32_t *cellof,
+                                                           const uint32_t *cell_start, const uint32_t *qbr,
+                                                           const uint32_t *r2q, double *pts, uint32_t *orig,
+                                                           uint32_t *pcell) {
+    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    const uint32_t r = cellof[p];
+    const uint64_t dest = (uint64_t)qbr[r] + (p - cell_start[r]);
+    const uint32_t src = idx_sorted[p];
+    for (int d = 0; d < pad; ++d) pts[dest * pad + d] = d < dim ? raw[(uint64_t)src * dim + d] : 0.0;
+    orig[dest] = src;
+    pcell[dest] = r2q[r];
+}
+
+int bits_for(unsigned long long maxval) {
+    int b = 0;
+    while (b < 64 && (maxval >> b) != 0) ++b;
+    return b;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------ host
+
+// Forward offsets of LID-UNICOMP: o in {-1,0,1}^dim whose row-major linear id
+// delta is positive <=> first non-zero component is +1 (reading c7).
+static int forward_offsets(int dim, std::vector<int8_t> &offs) {
+    offs.clear();
+    int total = 1;
+    for (int d = 0; d < dim; ++d) total *= 3;
+    for (int t = 0; t < total; ++t) {
+        int8_t o[SJ_MAX_DIM];
+        int v = t;
+        for (int d = dim - 1; d >= 0; --d) {
+            o[d] = (int8_t)(v % 3 - 1);
+            v /= 3;
+        }
+        int first = 0;
+        for (int d = 0; d < dim; ++d)
+            if (o[d] != 0) {
+                first = o[d];
+                break;
+            }
+        if (first == 1)
+            for (int d = 0; d < dim; ++d) offs.push_back(o[d]);
+    }
+    return (int)(offs.size() / (dim ? dim : 1));
+}
+
+int forward_offsets_public(int dim, int8_t *out, uint64_t cap) {
+    if (dim < 1 || dim > SJ_MAX_DIM) return SJ_EINVAL;
+    std::vector<int8_t> offs;
+    int F = forward_offsets(dim, offs);
+    if (out) {
+        if (cap < offs.size()) return SJ_EINVAL;
+        memcpy(out, offs.data(), offs.size());
+    }
+    return F;
+}
+
+void free_index(Index &ix, cudaStream_t s) {
+    dev_free(ix.pts, s);
+    dev_free(ix.orig, s);
+    dev_free(ix.pcell, s);
+    dev_free(ix.cellq, s);
+    dev_free(ix.fwd, s);
+    dev_free(ix.cell_lid, s);
+    ix.pts = nullptr;
+    ix.orig = ix.pcell = nullptr;
+    ix.cellq = nullptr;
+    ix.fwd = nullptr;
+    ix.cell_lid = nullptr;
+}
+
+namespace {
+// RAII list of temporaries freed on the stream at scope exit.
+struct Temps {
+    cudaStream_t s;
+    std::vector<void *> ptrs;
+    explicit Temps(cudaStream_t st) : s(st) {}
+    ~Temps() {
+        for (void *p : ptrs) dev_free(p, s);
+    }
+    template <class T>
+    int alloc(T **p, size_t count) {
+        int rc = dev_alloc_t(p, count, s);
+        if (rc == SJ_OK) ptrs.push_back(*p);
+        return rc;
+    }
+};
+}  // namespace
+
+template <class K>
+static int sort_points(Temps &tmp, const double *d_raw, uint64_t n, const GridGeom &geo, int bits, cudaStream_t s,
+                       K **keys_sorted, uint32_t **idx_sorted) {
+    K *ka, *kb;
+    uint32_t *va, *vb;
+    SJ_TRY(tmp.alloc(&ka, n));
+    SJ_TRY(tmp.alloc(&kb, n));
+    SJ_TRY(tmp.alloc(&va, n));
+    SJ_TRY(tmp.alloc(&vb, n));
+    cell_id_kernel<K><<<grid_for(n), kThreads, 0, s>>>(d_raw, n, geo, ka, va);
+    SJ_CUDA_TRY(cudaGetLastError());
+    if constexpr (sizeof(K) == 4)
+        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s));
+    else
+        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s));
+    return SJ_OK;
+}
+
+template <class K>
+static int rle(Temps &tmp, const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *cell_lid,
+               uint32_t *cell_start, uint64_t *d_M, cudaStream_t s) {
+    rle_flags_kernel<K><<<grid_for(n), kThreads, 0, s>>>(ks, n, cellof);
+    uint32_t *d_m32;
+    SJ_TRY(tmp.alloc(&d_m32, 1));
+    SJ_TRY(scan_exclusive_u32(cellof, cellof, n, d_m32, s));
+    rle_write_kernel<K><<<grid_for(n), kThreads, 0, s>>>(ks, n, cellof, cell_lid, cell_start);
+    // d_M (u64) <- d_m32
+    SJ_CUDA_TRY(cudaMemsetAsync(d_M, 0, sizeof(uint64_t), s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(d_M, d_m32, sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+    SJ_CUDA_TRY(cudaGetLastError());
+    return SJ_OK;
+}
+
+int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s, cudaEvent_t ev0,
+                cudaEvent_t ev1, float *ms) {
+    Temps tmp(s);
+    ix.n = n;
+    ix.dim = dim;
+    ix.pad = dim == 1 ? 1 : ((dim + 1) & ~1);
+    ix.eps = eps;
+    ix.e2 = eps * eps;                 // e2 = fl(eps*eps)
+    ix.w = eps * (1.0 + 0x1p-20);      // reading c5
+    if (ev0) SJ_CUDA_TRY(cudaEventRecord(ev0, s));
+
+    // pinned mailbox for the two host round trips
+    static_assert(sizeof(BBox) <= 256, "bbox");
+    void *mail = nullptr;
+    SJ_CUDA_TRY(cudaMallocHost(&mail, 512));
+    struct MailFree {
+        void *p;
+        ~MailFree() { cudaFreeHost(p); }
+    } mail_free{mail};
+
+    // ---- a2: bounding box + non-finite check
+    BBox *d_bb;
+    SJ_TRY(tmp.alloc(&d_bb, 1));
+    bbox_init_kernel<<<1, 32, 0, s>>>(d_bb);
+    {
+        unsigned blocks = (unsigned)std::min<uint64_t>(grid_for(n), 148ull * 8);
+        bbox_kernel<<<blocks, kThreads, 0, s>>>(d_raw, n, dim, d_bb);
+    }
+    SJ_CUDA_TRY(cudaGetLastError());
+    SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_bb, sizeof(BBox), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    BBox bb;
+    memcpy(&bb, mail, sizeof bb);
+    if (bb.nonfinite) {
+        set_error("sj_create: non-finite coordinate");
+        return SJ_EINVAL;
+    }
+    GridGeom geo{};
+    geo.dim = dim;
+    geo.w = ix.w;
+    unsigned __int128 total = 1;
+    for (int d = 0; d < dim; ++d) {
+        double mn = from_ordered_key(bb.mn[d]);
+        double mx = from_ordered_key(bb.mx[d]);
+        ix.mins[d] = mn;
+        geo.mins[d] = mn;
+        // nc_d = max c_d + 1; c_d is monotone in x_d so max c_d = c_d(max x_d)
+        double q = (mx - mn) / ix.w;
+        if (!(q < 0x1p30)) {
+            set_error("sj_create: grid too large in dimension %d (%.3g cells >= 2^30)", d, q);
+            return SJ_EGRID;
+        }
+        ix.nc[d] = (uint64_t)floor(q) + 1;
+        total *= ix.nc[d];
+        if (total >= ((unsigned __int128)1 << 64)) {
+            set_error("sj_create: grid too large (prod nc_d >= 2^64)");
+            return SJ_EGRID;
+        }
+    }
+    for (int d = dim - 1; d >= 0; --d) ix.stride[d] = (d == dim - 1) ? 1 : ix.stride[d + 1] * ix.nc[d + 1];
+    for (int d = 0; d < dim; ++d) {
+        geo.nc[d] = ix.nc[d];
+        geo.stride[d] = ix.stride[d];
+    }
+    const unsigned long long ncells_total = (unsigned long long)total;
+    ix.key_bits = bits_for(ncells_total - 1);
+
+    // ---- a3 + a4: cell ids and radix sort
+    uint32_t *idx_sorted = nullptr;
+    uint32_t *cellof;
+    unsigned long long *cell_lid;
+    uint32_t *cell_start;
+    uint64_t *d_M;
+    SJ_TRY(tmp.alloc(&cellof, n));
+    SJ_TRY(tmp.alloc(&cell_lid, n));
+    SJ_TRY(tmp.alloc(&cell_start, n + 1));
+    SJ_TRY(tmp.alloc(&d_M, 1));
+    if (ix.key_bits <= 32) {
+        uint32_t *ks;
+        SJ_TRY(sort_points<uint32_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
+        SJ_TRY(rle<uint32_t>(tmp, ks, n, cellof, cell_lid, cell_start, d_M, s));
+    } else {
+        uint64_t *ks;
+        SJ_TRY(sort_points<uint64_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
+        SJ_TRY(rle<uint64_t>(tmp, ks, n, cellof, cell_lid, cell_start, d_M, s));
+    }
+
+    // ---- lid -> rank lookup: dense table when prod(nc) is small, else a hash table
+    Lookup L{};
+    const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
+    if (dense) {
+        uint32_t *tab;
+        SJ_TRY(tmp.alloc(&tab, ncells_total));
+        SJ_CUDA_TRY(cudaMemsetAsync(tab, 0xFF, ncells_total * sizeof(uint32_t), s));
+        dense_fill_kernel<<<grid_for(n), kThreads, 0, s>>>(cell_lid, d_M, tab);
+        L.dense = tab;
+    } else {
+        unsigned long long cap = 1024;
+        while (cap < 2 * n) cap <<= 1;
+        unsigned long long *hk;
+        uint32_t *hv;
+        SJ_TRY(tmp.alloc(&hk, cap));
+        SJ_TRY(tmp.alloc(&hv, cap));
+        SJ_CUDA_TRY(cudaMemsetAsync(hk, 0xFF, cap * sizeof(unsigned long long), s));
+        hash_insert_kernel<<<grid_for(n), kThreads, 0, s>>>(cell_lid, d_M, hk, hv, cap - 1);
+        L.hkeys = hk;
+        L.hvals = hv;
+        L.hmask = cap - 1;
+    }
+    SJ_CUDA_TRY(cudaGetLastError());
+
+    // ---- a6 + a7: forward neighbour counts, workload, D_alg
+    std::vector<int8_t> offs;
+    const int F = forward_offsets(dim, offs);
+    {
+        std::vector<uint64_t> packed(F);
+        std::vector<long long> delta(F);
+        for (int j = 0; j < F; ++j) {
+            uint64_t p = 0;
+            long long dl = 0;
+            for (int d = 0; d < dim; ++d) {
+                p |= (uint64_t)(uint8_t)offs[(size_t)j * dim + d] << (8 * d);
+                dl += (long long)offs[(size_t)j * dim + d] * (long long)ix.stride[d];
+            }
+            packed[j] = p;
+            delta[j] = dl;
+        }
+        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, packed.data(), F * sizeof(uint64_t), 0,
+                                            cudaMemcpyHostToDevice, s));
+        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_delta, delta.data(), F * sizeof(long long), 0,
+                                            cudaMemcpyHostToDevice, s));
+    }
+    FwdGeom fg{};
+    fg.dim = dim;
+    fg.F = F;
+    for (int d = 0; d < dim; ++d) {
+        fg.nc[d] = ix.nc[d];
+        fg.stride[d] = ix.stride[d];
+    }
+    uint32_t *fcnt, *wload;
+    BuildTotals *d_tot;
+    SJ_TRY(tmp.alloc(&fcnt, n + 1));
+    SJ_TRY(tmp.alloc(&wload, n));
+    SJ_TRY(tmp.alloc(&d_tot, 1));
+    SJ_CUDA_TRY(cudaMemsetAsync(d_tot, 0, sizeof(BuildTotals), s));
+    fwd_kernel<false><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, fcnt, wload, nullptr,
+                                                       nullptr, d_tot);
+    SJ_CUDA_TRY(cudaGetLastError());
+    // fbegin = exclusive scan of fcnt over M (+1 entry for the end): scan n+1 entries with
+    // fcnt[r] = 0 for r >= M so fbegin[M] = E.
+    uint32_t *fbegin;
+    SJ_TRY(tmp.alloc(&fbegin, n + 1));
+    SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_M, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    uint64_t M;
+    memcpy(&M, mail, sizeof M);
+    ix.n_cells = M;
+    uint32_t *d_E32;
+    SJ_TRY(tmp.alloc(&d_E32, 1));
+    SJ_CUDA_TRY(cudaMemsetAsync(fcnt + M, 0, sizeof(uint32_t), s));
+    SJ_TRY(scan_exclusive_u32(fcnt, fbegin, M + 1, d_E32, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, fbegin + M, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    BuildTotals bt;
+    memcpy(&bt, mail, sizeof bt);
+    uint32_t E32;
+    memcpy(&E32, (char *)mail + 256, sizeof E32);
+    const uint64_t E = E32;
+    ix.fwd_entries = E;
+    ix.dist_calcs = bt.dist_calcs;
+    ix.max_w = bt.max_w;
+
+    uint32_t *fwd_rank;
+    SJ_TRY(tmp.alloc(&fwd_rank, E + 1));
+    fwd_kernel<true><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr, fbegin,
+                                                      fwd_rank, nullptr);
+    SJ_CUDA_TRY(cudaGetLastError());
+
+    // ---- a8: SortByWL over cells
+    uint32_t *wk, *wv, *wk2, *wv2, *qorder_keys, *qorder;
+    SJ_TRY(tmp.alloc(&wk, M));
+    SJ_TRY(tmp.alloc(&wv, M));
+    SJ_TRY(tmp.alloc(&wk2, M));
+    SJ_TRY(tmp.alloc(&wv2, M));
+    wl_keys_kernel<<<grid_for(M), kThreads, 0, s>>>(wload, M, ix.max_w, wk, wv);
+    SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(ix.max_w), &qorder_keys, &qorder, s));
+    uint32_t *mq, *qb;
+    SJ_TRY(tmp.alloc(&mq, M));
+    SJ_TRY(tmp.alloc(&qb, M));
+    queue_m_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, cell_start, M, mq);
+    SJ_TRY(scan_exclusive_u32(mq, qb, M, nullptr, s));
+
+    // ---- final arrays
+    SJ_TRY(dev_alloc_t(&ix.cellq, M, s));
+    SJ_TRY(dev_alloc_t(&ix.fwd, E + 1, s));
+    SJ_TRY(dev_alloc_t(&ix.cell_lid, M, s));
+    SJ_TRY(dev_alloc_t(&ix.pts, n * ix.pad, s));
+    SJ_TRY(dev_alloc_t(&ix.orig, n, s));
+    SJ_TRY(dev_alloc_t(&ix.pcell, n, s));
+    uint32_t *r2q, *qbr;
+    SJ_TRY(tmp.alloc(&r2q, M));
+    SJ_TRY(tmp.alloc(&qbr, M));
+    cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, fbegin, cell_lid, M, ix.cellq, r2q,
+                                                           qbr, ix.cell_lid);
+    if (E) fwd_convert_kernel<<<grid_for(E), kThreads, 0, s>>>(fwd_rank, E, qbr, cell_start, ix.fwd);
+    permute_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, dim, ix.pad, idx_sorted, cellof, cell_start, qbr, r2q,
+                                                    ix.pts, ix.orig, ix.pcell);
+    SJ_CUDA_TRY(cudaGetLastError());
+    if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    if (ms && ev0 && ev1) SJ_CUDA_TRY(cudaEventElapsedTime(ms, ev0, ev1));
+    return SJ_OK;
+}
+
+}  // namespace sj

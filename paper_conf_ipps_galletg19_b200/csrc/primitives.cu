@@ -1,0 +1,288 @@
+// primitives.cu -- hand-written scan and LSD radix sort for sm_100a.
+//
+// The radix sort orders point->cell ids for the eps-grid index ("GPU Grid
+// Index", north_star "a hand-written radix sort of point-to-cell IDs") and orders
+// cells by workload for SortByWL.  Per 8-bit pass:
+//   1. tile histogram (2048 keys per CTA, shared-memory counters),
+//   2. exclusive scan of the digit-major histogram [256 x tiles] -> global starts,
+//   3. stable scatter: per-warp ranks with __match_any_sync, a block-wide
+//      prefix over warps and digits, a shared-memory reorder of the tile so the
+//      global writes of one digit run are contiguous (coalesced).
+#include <cstdio>
+
+#include "sj_internal.cuh"
+
+namespace sj {
+
+namespace {
+
+constexpr int kScanThreads = 256;
+constexpr int kScanItems = 8;
+constexpr int kScanTile = kScanThreads * kScanItems;
+
+template <class T>
+__device__ __forceinline__ T warp_inclusive_scan(T x) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    return x;
+}
+
+// Block-wide exclusive scan; every thread of the block must call it.
+template <class T>
+__device__ __forceinline__ T block_exclusive_scan(T v, T *total) {
+    __shared__ T warp_sums[32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int nw = (blockDim.x + 31) >> 5;
+    T x = warp_inclusive_scan(v);
+    __syncthreads();
+    if (lane == 31) warp_sums[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+        T w = lane < nw ? warp_sums[lane] : T(0);
+        w = warp_inclusive_scan(w);
+        warp_sums[lane] = w;
+    }
+    __syncthreads();
+    T pre = wid > 0 ? warp_sums[wid - 1] : T(0);
+    if (total) *total = warp_sums[nw - 1];
+    return pre + x - v;
+}
+
+template <class T>
+__global__ void __launch_bounds__(kScanThreads) scan_reduce_kernel(const T *in, uint64_t n, T *partials) {
+    const uint64_t base = (uint64_t)blockIdx.x * kScanTile;
+    T s = 0;
+#pragma unroll
+    for (int it = 0; it < kScanItems; ++it) {
+        uint64_t i = base + (uint64_t)it * kScanThreads + threadIdx.x;
+        if (i < n) s += in[i];
+    }
+    T tot;
+    block_exclusive_scan<T>(s, &tot);
+    if (threadIdx.x == 0) partials[blockIdx.x] = tot;
+}
+
+template <class T>
+__global__ void __launch_bounds__(1024) scan_partials_kernel(T *partials, uint64_t nt, T *d_total) {
+    T carry = 0;
+    for (uint64_t b = 0; b < nt; b += blockDim.x) {
+        uint64_t i = b + threadIdx.x;
+        T v = i < nt ? partials[i] : T(0);
+        T tot;
+        T ex = block_exclusive_scan<T>(v, &tot);
+        if (i < nt) partials[i] = carry + ex;
+        carry += tot;
+    }
+    if (threadIdx.x == 0 && d_total) *d_total = carry;
+}
+
+template <class T>
+__global__ void __launch_bounds__(kScanThreads) scan_down_kernel(const T *in, T *out, uint64_t n, const T *partials) {
+    __shared__ T tile[kScanTile];
+    const uint64_t base = (uint64_t)blockIdx.x * kScanTile;
+    // coalesced load into shared memory, then blocked per-thread scan
+#pragma unroll
+    for (int it = 0; it < kScanItems; ++it) {
+        uint64_t i = base + (uint64_t)it * kScanThreads + threadIdx.x;
+        tile[it * kScanThreads + threadIdx.x] = i < n ? in[i] : T(0);
+    }
+    __syncthreads();
+    T v[kScanItems];
+    T s = 0;
+#pragma unroll
+    for (int j = 0; j < kScanItems; ++j) {
+        v[j] = tile[threadIdx.x * kScanItems + j];
+        s += v[j];
+    }
+    T ex = block_exclusive_scan<T>(s, nullptr) + partials[blockIdx.x];
+    // block_exclusive_scan ends with __syncthreads before its final read; tile reuse is safe
+#pragma unroll
+    for (int j = 0; j < kScanItems; ++j) {
+        tile[threadIdx.x * kScanItems + j] = ex;
+        ex += v[j];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int it = 0; it < kScanItems; ++it) {
+        uint64_t i = base + (uint64_t)it * kScanThreads + threadIdx.x;
+        if (i < n) out[i] = tile[it * kScanThreads + threadIdx.x];
+    }
+}
+
+template <class T>
+int scan_exclusive(const T *in, T *out, uint64_t n, T *d_total, cudaStream_t s) {
+    if (n == 0) {
+        if (d_total) SJ_CUDA_TRY(cudaMemsetAsync(d_total, 0, sizeof(T), s));
+        return SJ_OK;
+    }
+    uint64_t nt = (n + kScanTile - 1) / kScanTile;
+    T *partials = nullptr;
+    SJ_TRY(dev_alloc_t(&partials, nt, s));
+    scan_reduce_kernel<T><<<(unsigned)nt, kScanThreads, 0, s>>>(in, n, partials);
+    scan_partials_kernel<T><<<1, 1024, 0, s>>>(partials, nt, d_total);
+    scan_down_kernel<T><<<(unsigned)nt, kScanThreads, 0, s>>>(in, out, n, partials);
+    SJ_CUDA_TRY(cudaGetLastError());
+    dev_free(partials, s);
+    return SJ_OK;
+}
+
+// ------------------------------------------------------------------ radix sort
+
+constexpr int kRadixThreads = 256;
+constexpr int kRadixWarps = kRadixThreads / 32;
+constexpr int kRadixItems = 8;  // per lane
+constexpr int kRadixTile = kRadixThreads * kRadixItems;
+constexpr int kRadixBins = 256;
+
+template <class K>
+__global__ void __launch_bounds__(kRadixThreads) radix_hist_kernel(const K *keys, uint64_t n, int shift,
+                                                                   uint32_t *hist, uint32_t ntiles) {
+    __shared__ uint32_t h[kRadixBins];
+    h[threadIdx.x] = 0;
+    __syncthreads();
+    const uint64_t base = (uint64_t)blockIdx.x * kRadixTile;
+#pragma unroll
+    for (int it = 0; it < kRadixItems; ++it) {
+        uint64_t i = base + (uint64_t)it * kRadixThreads + threadIdx.x;
+        if (i < n) atomicAdd(&h[(uint32_t)(keys[i] >> shift) & 0xFFu], 1u);
+    }
+    __syncthreads();
+    hist[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
+}
+
+template <class K>
+__global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *keys_in, const uint32_t *vals_in,
+                                                                      K *keys_out, uint32_t *vals_out, uint64_t n,
+                                                                      int shift, const uint32_t *hist_scanned,
+                                                                      uint32_t ntiles) {
+    __shared__ uint32_t cnt[kRadixWarps][kRadixBins];
+    __shared__ uint32_t dstart[kRadixBins];
+    __shared__ uint32_t gstart[kRadixBins];
+    __shared__ K skeys[kRadixTile];
+    __shared__ uint32_t svals[kRadixTile];
+
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int w = 0; w < kRadixWarps; ++w) cnt[w][threadIdx.x] = 0;
+    const uint64_t base = (uint64_t)blockIdx.x * kRadixTile;
+    const uint64_t wbase = base + (uint64_t)warp * (32 * kRadixItems);
+
+    K key[kRadixItems];
+    uint32_t val[kRadixItems];
+    uint32_t dig[kRadixItems];
+    uint32_t rank[kRadixItems];
+#pragma unroll
+    for (int it = 0; it < kRadixItems; ++it) {
+        uint64_t i = wbase + (uint64_t)it * 32 + lane;
+        if (i < n) {
+            key[it] = keys_in[i];
+            val[it] = vals_in[i];
+            dig[it] = (uint32_t)(key[it] >> shift) & 0xFFu;
+        } else {
+            key[it] = 0;
+            val[it] = 0;
+            dig[it] = kRadixBins;  // sentinel: not counted
+        }
+    }
+    __syncthreads();
+    // per-warp stable ranks in (it, lane) order
+#pragma unroll
+    for (int it = 0; it < kRadixItems; ++it) {
+        const uint32_t d = dig[it];
+        const uint32_t peers = __match_any_sync(0xffffffffu, d);
+        uint32_t before = 0;
+        if (d < kRadixBins) before = cnt[warp][d];
+        rank[it] = before + __popc(peers & lt);
+        __syncwarp();
+        if (d < kRadixBins && (peers & lt) == 0) cnt[warp][d] = before + __popc(peers);
+        __syncwarp();
+    }
+    __syncthreads();
+    // prefix over warps for digit d = threadIdx.x, then over digits
+    {
+        const uint32_t d = threadIdx.x;
+        uint32_t s = 0;
+#pragma unroll
+        for (int w = 0; w < kRadixWarps; ++w) {
+            uint32_t t = cnt[w][d];
+            cnt[w][d] = s;
+            s += t;
+        }
+        uint32_t ex = block_exclusive_scan<uint32_t>(s, nullptr);
+        dstart[d] = ex;
+        gstart[d] = hist_scanned[(uint64_t)d * ntiles + blockIdx.x];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int it = 0; it < kRadixItems; ++it) {
+        const uint32_t d = dig[it];
+        if (d < kRadixBins) {
+            uint32_t lpos = dstart[d] + cnt[warp][d] + rank[it];
+            skeys[lpos] = key[it];
+            svals[lpos] = val[it];
+        }
+    }
+    __syncthreads();
+    const uint64_t rem = n - base;
+    const uint32_t tcount = rem < (uint64_t)kRadixTile ? (uint32_t)rem : (uint32_t)kRadixTile;
+    for (uint32_t i = threadIdx.x; i < tcount; i += kRadixThreads) {
+        K k = skeys[i];
+        uint32_t d = (uint32_t)(k >> shift) & 0xFFu;
+        uint64_t dest = (uint64_t)gstart[d] + (i - dstart[d]);
+        keys_out[dest] = k;
+        vals_out[dest] = svals[i];
+    }
+}
+
+template <class K>
+int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_t n, int bits, K **keys_out,
+               uint32_t **vals_out, cudaStream_t s) {
+    *keys_out = keys;
+    *vals_out = vals;
+    if (n <= 1 || bits <= 0) return SJ_OK;
+    if (n >= (1ull << 32)) {
+        set_error("radix_sort: n >= 2^32");
+        return SJ_EINVAL;
+    }
+    const uint32_t ntiles = (uint32_t)((n + kRadixTile - 1) / kRadixTile);
+    uint32_t *hist = nullptr;
+    SJ_TRY(dev_alloc_t(&hist, (uint64_t)kRadixBins * ntiles, s));
+    K *ka = keys, *kb = keys_alt;
+    uint32_t *va = vals, *vb = vals_alt;
+    for (int shift = 0; shift < bits; shift += 8) {
+        radix_hist_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, n, shift, hist, ntiles);
+        SJ_TRY(scan_exclusive<uint32_t>(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s));
+        radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, va, kb, vb, n, shift, hist, ntiles);
+        SJ_CUDA_TRY(cudaGetLastError());
+        K *tk = ka; ka = kb; kb = tk;
+        uint32_t *tv = va; va = vb; vb = tv;
+    }
+    dev_free(hist, s);
+    *keys_out = ka;
+    *vals_out = va;
+    return SJ_OK;
+}
+
+}  // namespace
+
+int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s) {
+    return scan_exclusive<uint32_t>(in, out, n, d_total, s);
+}
+int scan_exclusive_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s) {
+    return scan_exclusive<uint64_t>(in, out, n, d_total, s);
+}
+int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
+                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s) {
+    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s);
+}
+int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
+                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s) {
+    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s);
+}
+
+}  // namespace sj

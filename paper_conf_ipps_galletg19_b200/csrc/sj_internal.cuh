@@ -1,0 +1,130 @@
+// sj_internal.cuh -- internal declarations shared by the libsj.so translation units.
+// Product code (CUDA for sm_100a + C++ host runtime).  Never includes or links the
+// oracle (oracle/), see DESIGN.md §3.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/sj.h"
+
+#define SJ_MAX_DIM 8
+#define SJ_MAX_FWD 3280  // (3^8 - 1) / 2
+
+namespace sj {
+
+// --------------------------------------------------------------------------- errors
+void set_error(const char *fmt, ...);
+struct Status {
+    int code = SJ_OK;
+};
+
+#define SJ_CUDA_TRY(expr)                                                                       \
+    do {                                                                                        \
+        cudaError_t _e = (expr);                                                                \
+        if (_e != cudaSuccess) {                                                                \
+            ::sj::set_error("%s:%d %s: %s", __FILE__, __LINE__, #expr, cudaGetErrorString(_e)); \
+            return (_e == cudaErrorMemoryAllocation) ? SJ_ENOMEM : SJ_ECUDA;                    \
+        }                                                                                       \
+    } while (0)
+
+#define SJ_TRY(expr)                 \
+    do {                             \
+        int _rc = (expr);            \
+        if (_rc < 0) return _rc;     \
+    } while (0)
+
+// --------------------------------------------------------------------------- memory
+// Stream-ordered allocations from the device's default memory pool.  The pool's
+// release threshold is raised once, so repeated create/destroy cycles reuse memory
+// instead of returning it to the driver (DESIGN.md §4 "memory").
+int dev_alloc(void **p, size_t bytes, cudaStream_t s);
+void dev_free(void *p, cudaStream_t s);
+template <class T>
+inline int dev_alloc_t(T **p, size_t count, cudaStream_t s) {
+    return dev_alloc(reinterpret_cast<void **>(p), count * sizeof(T) + 16, s);
+}
+
+// --------------------------------------------------------------------------- primitives
+// Exclusive scan of u32 (out may alias in).  total (device, optional) receives the sum.
+int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s);
+// u64 variant
+int scan_exclusive_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s);
+
+// Stable LSD radix sort of (key, value) pairs on the low `bits` bits of the keys.
+// Hand-written: per 8-bit pass a tile histogram, a digit-major scan and a stable
+// scatter through shared memory (DESIGN.md §4 a4).  Buffers are ping-ponged; the
+// result pointer pair is returned through *keys_out / *vals_out (one of the inputs
+// or the alternates).
+int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
+                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s);
+int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
+                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s);
+
+// --------------------------------------------------------------------------- index
+// The index I in its B200 layout, DESIGN.md §4.  Points are stored in the
+// SortByWL queue order D' so the WorkQueue hands out contiguous storage positions.
+struct Index {
+    uint64_t n = 0;
+    int dim = 0;
+    int pad = 0;              // doubles per stored point (dim rounded up to even; 1 for dim 1)
+    double eps = 0, e2 = 0, w = 0;
+    double mins[SJ_MAX_DIM] = {0};
+    uint64_t nc[SJ_MAX_DIM] = {0};
+    uint64_t stride[SJ_MAX_DIM] = {0};
+    int key_bits = 0;
+    uint64_t n_cells = 0;     // M
+    uint64_t fwd_entries = 0; // E
+    uint64_t dist_calcs = 0;  // D_alg
+    uint32_t max_w = 0;
+
+    double *pts = nullptr;      // [n * pad]  D' order
+    uint32_t *orig = nullptr;   // [n]        D' position -> input id
+    uint32_t *pcell = nullptr;  // [n]        D' position -> queue-order cell index
+    uint4 *cellq = nullptr;     // [M]        queue-order cell: {begin in D', m, fwd_begin, fwd_end}
+    uint2 *fwd = nullptr;       // [E]        forward neighbour cell: {begin in D', m}
+    uint64_t *cell_lid = nullptr; // [M]      queue-order cell -> linear id (export / tests)
+};
+
+struct BuildTimes {
+    float ms = 0;
+};
+
+// Builds the index from device-resident raw points (n x dim AoS).  Returns sj_status.
+int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s,
+                cudaEvent_t ev0, cudaEvent_t ev1, float *ms);
+void free_index(Index &ix, cudaStream_t s);
+// LID-UNICOMP forward offsets (host): F = (3^dim - 1)/2 offsets, int8 each dim.
+int forward_offsets_public(int dim, int8_t *out, uint64_t cap);
+
+// --------------------------------------------------------------------------- join
+struct JoinArgs {
+    const double *pts;
+    const uint32_t *orig;
+    const uint32_t *pcell;
+    const uint4 *cellq;
+    const uint2 *fwd;
+    double e2;
+    unsigned long long *head;     // dequeue counter (virtual queue positions)
+    unsigned long long v_end;     // end of this batch (virtual)
+    uint32_t n;                   // points
+    uint32_t grab;                // positions per dequeue (= slice chunk)
+    uint32_t rank, world;         // queue slice
+    uint32_t *out;                // interleaved pairs, or nullptr (count-only)
+    unsigned long long *emit_ctr; // pairs emitted (may exceed out_cap -> overflow)
+    unsigned long long out_cap;   // capacity of out in pairs
+    unsigned long long *calcs;    // instrumented distance calculations, or nullptr
+};
+
+// Launch the join kernel for dim/k; emit=false counts pairs only.
+int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaStream_t s);
+// Max resident CTAs per SM of the join kernel configuration.
+int join_occupancy(int dim, int k, bool emit, int *blocks_per_sm);
+constexpr int kJoinThreads = 256;
+
+// --------------------------------------------------------------------------- misc kernels
+int launch_fill_u64(unsigned long long *p, const unsigned long long *vals_host_pinned, int count, cudaStream_t s);
+
+}  // namespace sj

@@ -1,0 +1,823 @@
+// sj_runtime.cu -- host runtime behind the C ABI of include/sj.h (L1 + L2 of
+// DESIGN.md §2): handle state, stream-ordered memory, the batch estimator and the
+// batch loop, overflow retry, SJ_MORE continuation, statistics,
+// index export/import for the NCCL broadcast, and the host-only helpers.
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <deque>
+#include <mutex>
+#include <vector>
+
+#include "sj_internal.cuh"
+
+namespace sj {
+
+// ------------------------------------------------------------------------- errors
+static thread_local char g_err[1024] = "";
+
+void set_error(const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof g_err, fmt, ap);
+    va_end(ap);
+}
+
+// ------------------------------------------------------------------------- memory
+static std::mutex g_pool_mu;
+static bool g_pool_ready[64] = {false};
+
+static void pool_setup(int dev) {
+    std::lock_guard<std::mutex> lk(g_pool_mu);
+    if (dev < 0 || dev >= 64 || g_pool_ready[dev]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    g_pool_ready[dev] = true;
+}
+
+int dev_alloc(void **p, size_t bytes, cudaStream_t s) {
+    *p = nullptr;
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMallocAsync(p, bytes, s);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        set_error("device allocation of %zu bytes failed: %s", bytes, cudaGetErrorString(e));
+        return e == cudaErrorMemoryAllocation ? SJ_ENOMEM : SJ_ECUDA;
+    }
+    return SJ_OK;
+}
+
+void dev_free(void *p, cudaStream_t s) {
+    if (p) cudaFreeAsync(p, s);
+}
+
+// ------------------------------------------------------------------------- small kernels
+__global__ void set_u64_kernel(unsigned long long *p, unsigned long long v) { *p = v; }
+
+}  // namespace sj
+
+using namespace sj;
+
+// ------------------------------------------------------------------------- handle
+namespace {
+
+constexpr int kMaxStreams = 8;
+
+struct Job {
+    uint64_t v0, v1;  // virtual queue range [v0, v1), multiples of grab
+    int slot = -1;
+    bool launched = false, complete = false;
+    uint64_t cnt = 0, consumed = 0;
+};
+
+struct Slot {
+    cudaStream_t stream = nullptr;
+    uint32_t *buf = nullptr;
+    uint64_t cap = 0;                      // pairs
+    unsigned long long *d_ctr = nullptr;   // [0]=emit, [1]=head, [2]=calcs
+    cudaEvent_t ev_start = nullptr, ev_stop = nullptr, ev_done = nullptr;
+    bool busy = false;
+};
+
+}  // namespace
+
+struct sj_handle {
+    int device = 0;
+    int state = 0;  // 0 ready, 1 continuing (staged path), -1 error
+    cudaStream_t s_main = nullptr;
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr, ev_c = nullptr, ev_d = nullptr;
+    sj::Index ix;
+    bool owns_index = true;
+    int num_sms = 148;
+
+    // options
+    int k = 8;
+    uint64_t batch_pairs = 100000000ull;
+    int streams = 3;
+    uint32_t sample_ppm = 10000;
+    uint32_t grab = 32;
+    int count_calcs = 0;
+    int blocks_per_sm = 0;
+    int fast_path = 1;
+    int rank = 0, world = 1;
+
+    unsigned long long *d_ctr = nullptr;  // [0]=emit [1]=head [2]=calcs [3..] spare
+    uint64_t *mail = nullptr;             // pinned host mailbox [64]
+    Slot slots[kMaxStreams];
+    std::deque<Job> jobs;
+
+    sj_stats st{};
+};
+
+namespace {
+
+int fail(sj_handle *h, int rc) {
+    if (h && rc < 0) h->state = -1;
+    return rc;
+}
+
+int ensure_device(const sj_handle *h) {
+    SJ_CUDA_TRY(cudaSetDevice(h->device));
+    return SJ_OK;
+}
+
+bool is_device_ptr(const void *p, int dev) {
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (at.type == cudaMemoryTypeDevice) return at.device == dev;
+    if (at.type == cudaMemoryTypeManaged) return true;
+    return false;
+}
+
+int handle_init_common(sj_handle *h) {
+    SJ_CUDA_TRY(cudaGetDevice(&h->device));
+    pool_setup(h->device);
+    SJ_CUDA_TRY(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device));
+    SJ_CUDA_TRY(cudaStreamCreateWithFlags(&h->s_main, cudaStreamNonBlocking));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_a));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_b));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_c));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_d));
+    SJ_CUDA_TRY(cudaMallocHost(&h->mail, 64 * sizeof(uint64_t)));
+    SJ_TRY(dev_alloc_t(&h->d_ctr, 8, h->s_main));
+    return SJ_OK;
+}
+
+int slot_init(sj_handle *h, int i) {
+    Slot &s = h->slots[i];
+    if (s.stream) return SJ_OK;
+    SJ_CUDA_TRY(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    SJ_CUDA_TRY(cudaEventCreate(&s.ev_start));
+    SJ_CUDA_TRY(cudaEventCreate(&s.ev_stop));
+    SJ_CUDA_TRY(cudaEventCreateWithFlags(&s.ev_done, cudaEventDisableTiming));
+    SJ_TRY(dev_alloc_t(&s.d_ctr, 4, s.stream));
+    return SJ_OK;
+}
+
+int slot_buffer(sj_handle *h, Slot &s, uint64_t pairs) {
+    if (s.cap >= pairs && s.buf) return SJ_OK;
+    dev_free(s.buf, s.stream);
+    s.buf = nullptr;
+    s.cap = 0;
+    SJ_TRY(dev_alloc(reinterpret_cast<void **>(&s.buf), pairs * 2 * sizeof(uint32_t), s.stream));
+    s.cap = pairs;
+    return SJ_OK;
+}
+
+void slots_release(sj_handle *h) {
+    for (int i = 0; i < kMaxStreams; ++i) {
+        Slot &s = h->slots[i];
+        if (!s.stream) continue;
+        cudaStreamSynchronize(s.stream);
+        dev_free(s.buf, s.stream);
+        dev_free(s.d_ctr, s.stream);
+        cudaStreamSynchronize(s.stream);
+        cudaStreamDestroy(s.stream);
+        cudaEventDestroy(s.ev_start);
+        cudaEventDestroy(s.ev_stop);
+        cudaEventDestroy(s.ev_done);
+        s = Slot();
+    }
+}
+
+// number of virtual queue positions of this handle's slice (multiple of grab)
+uint64_t slice_chunks(const sj_handle *h) {
+    const uint64_t nchunks = (h->ix.n + h->grab - 1) / h->grab;
+    if (nchunks <= (uint64_t)h->rank) return 0;
+    return (nchunks - (uint64_t)h->rank + (uint64_t)h->world - 1) / (uint64_t)h->world;
+}
+
+JoinArgs base_args(const sj_handle *h) {
+    JoinArgs a{};
+    a.pts = h->ix.pts;
+    a.orig = h->ix.orig;
+    a.pcell = h->ix.pcell;
+    a.cellq = h->ix.cellq;
+    a.fwd = h->ix.fwd;
+    a.e2 = h->ix.e2;
+    a.n = (uint32_t)h->ix.n;
+    a.grab = h->grab;
+    a.rank = (uint32_t)h->rank;
+    a.world = (uint32_t)h->world;
+    return a;
+}
+
+int join_blocks(const sj_handle *h, bool emit, int *blocks) {
+    int occ = 0;
+    SJ_TRY(join_occupancy(h->ix.dim, h->k, emit, &occ));
+    if (h->blocks_per_sm > 0 && h->blocks_per_sm < occ) occ = h->blocks_per_sm;
+    if (occ < 1) occ = 1;
+    *blocks = occ * h->num_sms;
+    return SJ_OK;
+}
+
+// Count-only join over virtual range [v0, v1) on the main stream.  Synchronous.
+int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms) {
+    cudaStream_t s = h->s_main;
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, v0);
+    JoinArgs a = base_args(h);
+    a.head = h->d_ctr + 1;
+    a.v_end = v1;
+    a.out = nullptr;
+    a.emit_ctr = h->d_ctr;
+    a.out_cap = 0;
+    a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+    int blocks;
+    SJ_TRY(join_blocks(h, false, &blocks));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
+    if (v1 > v0) SJ_TRY(launch_join(a, h->ix.dim, h->k, false, blocks, s));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    *pairs = h->mail[0];
+    if (h->count_calcs) h->st.calcs_measured = h->mail[2];
+    if (ms) SJ_CUDA_TRY(cudaEventElapsedTime(ms, h->ev_c, h->ev_d));
+    return SJ_OK;
+}
+
+// ------------------------------------------------------------------ staged batches
+int launch_job(sj_handle *h, Job &j, int slot_idx) {
+    Slot &s = h->slots[slot_idx];
+    SJ_TRY(slot_buffer(h, s, h->batch_pairs));
+    SJ_CUDA_TRY(cudaMemsetAsync(s.d_ctr, 0, 4 * sizeof(unsigned long long), s.stream));
+    set_u64_kernel<<<1, 1, 0, s.stream>>>(s.d_ctr + 1, j.v0);
+    JoinArgs a = base_args(h);
+    a.head = s.d_ctr + 1;
+    a.v_end = j.v1;
+    a.out = s.buf;
+    a.emit_ctr = s.d_ctr;
+    a.out_cap = s.cap;
+    a.calcs = h->count_calcs ? s.d_ctr + 2 : nullptr;
+    int blocks;
+    SJ_TRY(join_blocks(h, true, &blocks));
+    SJ_CUDA_TRY(cudaEventRecord(s.ev_start, s.stream));
+    SJ_TRY(launch_join(a, h->ix.dim, h->k, true, blocks, s.stream));
+    SJ_CUDA_TRY(cudaEventRecord(s.ev_stop, s.stream));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail + 8 + 4 * slot_idx, s.d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost,
+                                s.stream));
+    SJ_CUDA_TRY(cudaEventRecord(s.ev_done, s.stream));
+    j.slot = slot_idx;
+    j.launched = true;
+    s.busy = true;
+    h->st.join_launches++;
+    return SJ_OK;
+}
+
+int fill_pipeline(sj_handle *h) {
+    for (Job &j : h->jobs) {
+        if (j.launched) continue;
+        int free_slot = -1;
+        for (int i = 0; i < h->streams; ++i)
+            if (!h->slots[i].busy) {
+                free_slot = i;
+                break;
+            }
+        if (free_slot < 0) break;
+        SJ_TRY(launch_job(h, j, free_slot));
+    }
+    return SJ_OK;
+}
+
+// Drives the staged batch pipeline until the caller's buffer is full or the join ends.
+int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
+    uint64_t written = 0;
+    for (;;) {
+        SJ_TRY(fill_pipeline(h));
+        if (h->jobs.empty()) break;
+        Job &j = h->jobs.front();
+        Slot &s = h->slots[j.slot];
+        if (!j.complete) {
+            SJ_CUDA_TRY(cudaEventSynchronize(s.ev_done));
+            const uint64_t *m = h->mail + 8 + 4 * j.slot;
+            j.cnt = m[0];
+            if (h->count_calcs) h->st.calcs_measured += m[2];
+            float ms = 0;
+            SJ_CUDA_TRY(cudaEventElapsedTime(&ms, s.ev_start, s.ev_stop));
+            h->st.ms_join_sum += ms;
+            if (j.cnt > s.cap) {
+                // overflow (estimate too low): split the range, or grow the buffer if it is one chunk
+                h->st.retries++;
+                if (h->count_calcs) h->st.calcs_measured -= m[2];
+                const Job old = j;
+                const uint64_t chunks = (old.v1 - old.v0) / h->grab;
+                h->jobs.pop_front();
+                s.busy = false;
+                if (chunks <= 1) {
+                    SJ_TRY(slot_buffer(h, s, old.cnt));
+                    Job again;
+                    again.v0 = old.v0;
+                    again.v1 = old.v1;
+                    h->jobs.push_front(again);
+                    SJ_TRY(launch_job(h, h->jobs.front(), old.slot));
+                } else {
+                    const uint64_t parts = std::min<uint64_t>(chunks, old.cnt / s.cap + 2);
+                    for (uint64_t p = parts; p-- > 0;) {
+                        Job nj;
+                        nj.v0 = old.v0 + (chunks * p / parts) * h->grab;
+                        nj.v1 = old.v0 + (chunks * (p + 1) / parts) * h->grab;
+                        if (nj.v1 > nj.v0) h->jobs.push_front(nj);
+                    }
+                    h->st.batches += (uint32_t)(parts - 1);
+                }
+                continue;
+            }
+            j.complete = true;
+        }
+        const uint64_t take = std::min<uint64_t>(j.cnt - j.consumed, cap - written);
+        if (take) {
+            SJ_CUDA_TRY(cudaMemcpyAsync(out + 2 * written, s.buf + 2 * j.consumed, take * 2 * sizeof(uint32_t),
+                                        cudaMemcpyDefault, s.stream));
+            written += take;
+            j.consumed += take;
+            h->st.pairs += take;
+        }
+        if (j.consumed == j.cnt) {
+            s.busy = false;  // the next job on this slot is ordered after the copy (same stream)
+            h->jobs.pop_front();
+            continue;
+        }
+        if (written == cap) break;  // leftover pairs in j -> SJ_MORE
+    }
+    for (int i = 0; i < h->streams; ++i)
+        if (h->slots[i].stream) SJ_CUDA_TRY(cudaStreamSynchronize(h->slots[i].stream));
+    *count = written;
+    if (h->jobs.empty()) {
+        h->state = 0;
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_b, h->s_main));
+        SJ_CUDA_TRY(cudaEventSynchronize(h->ev_b));
+        float tot = 0;
+        SJ_CUDA_TRY(cudaEventElapsedTime(&tot, h->ev_a, h->ev_b));
+        h->st.ms_total = tot;
+        h->st.ms_join = h->st.ms_join_sum;
+        return SJ_OK;
+    }
+    h->state = 1;
+    return SJ_MORE;
+}
+
+int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
+    SJ_TRY(ensure_device(h));
+    // a new join: reset per-join statistics
+    h->st.pairs = 0;
+    h->st.calcs_measured = 0;
+    h->st.batches = 0;
+    h->st.retries = 0;
+    h->st.join_launches = 0;
+    h->st.ms_join = h->st.ms_join_sum = h->st.ms_estimate = h->st.ms_transfer = h->st.ms_total = 0;
+    h->st.fast_path = 0;
+    h->st.k = (uint32_t)h->k;
+    h->jobs.clear();
+    for (int i = 0; i < kMaxStreams; ++i) h->slots[i].busy = false;
+
+    const uint64_t nch = slice_chunks(h);
+    const uint64_t V = nch * h->grab;
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_a, h->s_main));
+
+    if (out == nullptr) {  // count-only (whole slice, one launch)
+        uint64_t pairs = 0;
+        float ms = 0;
+        SJ_TRY(count_range(h, 0, V, &pairs, &ms));
+        h->st.ms_join = h->st.ms_join_sum = ms;
+        h->st.join_launches = 1;
+        h->st.batches = 1;
+        h->st.pairs = pairs;
+        *count = pairs;
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_b, h->s_main));
+        SJ_CUDA_TRY(cudaEventSynchronize(h->ev_b));
+        float tot = 0;
+        SJ_CUDA_TRY(cudaEventElapsedTime(&tot, h->ev_a, h->ev_b));
+        h->st.ms_total = tot;
+        h->state = 0;
+        return SJ_OK;
+    }
+
+    // a9: batch estimator -- count-only join over the first sample_ppm of D'
+    uint64_t sch = (nch * (uint64_t)h->sample_ppm + 999999ull) / 1000000ull;
+    if (sch < 1) sch = 1;
+    if (sch > nch) sch = nch;
+    uint64_t spairs = 0;
+    float ms_est = 0;
+    if (nch) SJ_TRY(count_range(h, 0, sch * h->grab, &spairs, &ms_est));
+    h->st.ms_estimate = ms_est;
+    h->st.calcs_measured = 0;
+    const double est = nch ? (double)spairs * (double)nch / (double)sch : 0.0;
+    h->st.est_pairs = (uint64_t)est;
+    uint64_t nb = (uint64_t)std::ceil(est / (double)h->batch_pairs);
+    if (nb < 1) nb = 1;
+    if (nb > nch && nch) nb = nch;
+
+    const bool dev_out = is_device_ptr(out, h->device);
+    if (dev_out && (reinterpret_cast<uintptr_t>(out) & 15u)) {
+        set_error("sj_self_join: device out_pairs must be 16-byte aligned");
+        return SJ_EINVAL;
+    }
+    if (dev_out && h->fast_path && est <= 4.0 * (double)cap + 1e6) {
+        // Fast path: the caller's HBM buffer is the result buffer; one persistent launch
+        // over the whole slice writes it in place (no staging, no D2D copy).
+        cudaStream_t s = h->s_main;
+        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+        set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, 0ull);
+        JoinArgs a = base_args(h);
+        a.head = h->d_ctr + 1;
+        a.v_end = V;
+        a.out = out;
+        a.emit_ctr = h->d_ctr;
+        a.out_cap = cap;
+        a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+        int blocks;
+        SJ_TRY(join_blocks(h, true, &blocks));
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
+        if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, true, blocks, s));
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        SJ_CUDA_TRY(cudaStreamSynchronize(s));
+        float ms = 0;
+        SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
+        h->st.join_launches = 1;
+        h->st.batches = 1;
+        h->st.ms_join = h->st.ms_join_sum = ms;
+        const uint64_t total = h->mail[0];
+        if (total <= cap) {
+            if (h->count_calcs) h->st.calcs_measured = h->mail[2];
+            h->st.pairs = total;
+            h->st.fast_path = 1;
+            *count = total;
+            SJ_CUDA_TRY(cudaEventRecord(h->ev_b, s));
+            SJ_CUDA_TRY(cudaEventSynchronize(h->ev_b));
+            float tot = 0;
+            SJ_CUDA_TRY(cudaEventElapsedTime(&tot, h->ev_a, h->ev_b));
+            h->st.ms_total = tot;
+            h->state = 0;
+            return SJ_OK;
+        }
+        h->st.retries++;  // did not fit: fall through to the staged path
+        h->st.ms_join = h->st.ms_join_sum = 0;
+        h->st.join_launches = 0;
+    }
+
+    // Staged path: nb batches = contiguous ranges of D' (reading c14), round-robin
+    // over `streams` streams, each into its own b_s buffer, copied out in batch order.
+    for (int i = 0; i < h->streams; ++i) SJ_TRY(slot_init(h, i));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_c, h->s_main));
+    for (int i = 0; i < h->streams; ++i) SJ_CUDA_TRY(cudaStreamWaitEvent(h->slots[i].stream, h->ev_c, 0));
+    for (uint64_t b = 0; b < nb; ++b) {
+        Job j;
+        j.v0 = (nch * b / nb) * h->grab;
+        j.v1 = (nch * (b + 1) / nb) * h->grab;
+        if (j.v1 > j.v0) h->jobs.push_back(j);
+    }
+    h->st.batches = (uint32_t)h->jobs.size();
+    h->state = 1;
+    return continue_staged(h, out, cap, count);
+}
+
+}  // namespace
+
+// =========================================================================== C ABI
+extern "C" {
+
+int sj_abi_version(void) { return SJ_ABI_VERSION; }
+
+const char *sj_last_error(void) { return g_err; }
+
+static int create_common(sj_handle **out_h) {
+    sj_handle *h = new (std::nothrow) sj_handle();
+    if (!h) {
+        set_error("out of host memory");
+        return SJ_ENOMEM;
+    }
+    int rc = handle_init_common(h);
+    if (rc < 0) {
+        sj_destroy(h);
+        return rc;
+    }
+    *out_h = h;
+    return SJ_OK;
+}
+
+static void fill_static_stats(sj_handle *h) {
+    sj_stats &st = h->st;
+    st.n = h->ix.n;
+    st.dim = (uint32_t)h->ix.dim;
+    st.key_bits = (uint32_t)h->ix.key_bits;
+    st.n_cells = h->ix.n_cells;
+    st.fwd_entries = h->ix.fwd_entries;
+    st.dist_calcs = h->ix.dist_calcs;
+    st.max_cell_load = h->ix.max_w;
+    st.k = (uint32_t)h->k;
+    for (int d = 0; d < SJ_MAX_DIM; ++d) st.nc[d] = d < h->ix.dim ? (uint32_t)h->ix.nc[d] : 0;
+}
+
+sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
+    set_error("");
+    if (!points || n == 0 || n >= (1ull << 32) || dim < 1 || dim > SJ_MAX_DIM || !(eps > 0.0) || !std::isfinite(eps)) {
+        set_error("sj_create: invalid argument (points=%p n=%llu dim=%d eps=%g)", (const void *)points,
+                  (unsigned long long)n, dim, eps);
+        return nullptr;
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        set_error("sj_create: no CUDA device available (the CUDA path has no CPU fallback)");
+        return nullptr;
+    }
+    sj_handle *h = nullptr;
+    if (create_common(&h) < 0) return nullptr;
+    cudaStream_t s = h->s_main;
+    const double *d_raw = points;
+    double *d_copy = nullptr;
+    int rc = SJ_OK;
+    if (!is_device_ptr(points, h->device)) {
+        // a1: upload (the library owns its copy; caller keeps `points`)
+        rc = dev_alloc_t(&d_copy, n * (uint64_t)dim, s);
+        if (rc == SJ_OK) {
+            cudaError_t e = cudaMemcpyAsync(d_copy, points, n * (uint64_t)dim * sizeof(double), cudaMemcpyDefault, s);
+            if (e != cudaSuccess) {
+                set_error("sj_create: upload failed: %s", cudaGetErrorString(e));
+                rc = SJ_ECUDA;
+            }
+        }
+        d_raw = d_copy;
+    }
+    float ms = 0;
+    if (rc == SJ_OK) rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_a, h->ev_b, &ms);
+    dev_free(d_copy, s);
+    if (rc == SJ_OK && cudaStreamSynchronize(s) != cudaSuccess) {
+        set_error("sj_create: %s", cudaGetErrorString(cudaGetLastError()));
+        rc = SJ_ECUDA;
+    }
+    if (rc < 0) {
+        std::string keep = g_err;
+        sj_destroy(h);
+        snprintf(g_err, sizeof g_err, "%s", keep.c_str());
+        return nullptr;
+    }
+    fill_static_stats(h);
+    h->st.ms_build = ms;
+    return h;
+}
+
+int sj_self_join(sj_handle *h, uint32_t *out_pairs, uint64_t cap, uint64_t *count) {
+    if (!h || !count) {
+        set_error("sj_self_join: NULL handle or count");
+        return SJ_EINVAL;
+    }
+    *count = 0;
+    if (h->state < 0) {
+        set_error("sj_self_join: handle is in the error state");
+        return SJ_ESTATE;
+    }
+    if ((out_pairs == nullptr) != (cap == 0)) {
+        set_error("sj_self_join: out_pairs and cap must both be set, or both NULL/0 for count-only");
+        return SJ_EINVAL;
+    }
+    int rc = ensure_device(h);
+    if (rc < 0) return fail(h, rc);
+    if (h->state == 1 && out_pairs) {
+        rc = continue_staged(h, out_pairs, cap, count);
+    } else {
+        rc = start_join(h, out_pairs, cap, count);
+    }
+    return fail(h, rc);
+}
+
+void sj_destroy(sj_handle *h) {
+    if (!h) return;
+    cudaSetDevice(h->device);
+    slots_release(h);
+    if (h->s_main) {
+        cudaStreamSynchronize(h->s_main);
+        if (h->owns_index) free_index(h->ix, h->s_main);
+        dev_free(h->d_ctr, h->s_main);
+        cudaStreamSynchronize(h->s_main);
+        cudaStreamDestroy(h->s_main);
+    }
+    if (h->ev_a) cudaEventDestroy(h->ev_a);
+    if (h->ev_b) cudaEventDestroy(h->ev_b);
+    if (h->ev_c) cudaEventDestroy(h->ev_c);
+    if (h->ev_d) cudaEventDestroy(h->ev_d);
+    if (h->mail) cudaFreeHost(h->mail);
+    delete h;
+}
+
+int sj_set_option(sj_handle *h, int opt, int64_t v) {
+    if (!h) return SJ_EINVAL;
+    switch (opt) {
+        case SJ_OPT_K:
+            if (v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32) break;
+            h->k = (int)v;
+            if (h->grab % (32 / h->k)) h->grab = ((h->grab + 32 / h->k - 1) / (32 / h->k)) * (32 / h->k);
+            h->st.k = (uint32_t)v;
+            return SJ_OK;
+        case SJ_OPT_BATCH_PAIRS:
+            if (v < 64) break;
+            h->batch_pairs = (uint64_t)v;
+            return SJ_OK;
+        case SJ_OPT_STREAMS:
+            if (v < 1 || v > kMaxStreams) break;
+            h->streams = (int)v;
+            return SJ_OK;
+        case SJ_OPT_SAMPLE_PPM:
+            if (v < 1 || v > 1000000) break;
+            h->sample_ppm = (uint32_t)v;
+            return SJ_OK;
+        case SJ_OPT_GRAB:
+            if (v < 1 || v > (1 << 20) || (v % (32 / h->k)) != 0) break;
+            h->grab = (uint32_t)v;
+            return SJ_OK;
+        case SJ_OPT_COUNT_CALCS:
+            h->count_calcs = v ? 1 : 0;
+            return SJ_OK;
+        case SJ_OPT_BLOCKS_PER_SM:
+            if (v < 0 || v > 32) break;
+            h->blocks_per_sm = (int)v;
+            return SJ_OK;
+        case SJ_OPT_FAST_PATH:
+            h->fast_path = v ? 1 : 0;
+            return SJ_OK;
+    }
+    set_error("sj_set_option: invalid option %d or value %lld", opt, (long long)v);
+    return SJ_EINVAL;
+}
+
+int sj_set_slice(sj_handle *h, int rank, int world) {
+    if (!h || world < 1 || rank < 0 || rank >= world) {
+        set_error("sj_set_slice: invalid rank %d / world %d", rank, world);
+        return SJ_EINVAL;
+    }
+    h->rank = rank;
+    h->world = world;
+    h->state = h->state < 0 ? h->state : 0;
+    return SJ_OK;
+}
+
+int sj_get_stats(const sj_handle *h, sj_stats *s) {
+    if (!h || !s) return SJ_EINVAL;
+    *s = h->st;
+    return SJ_OK;
+}
+
+// ---------------------------------------------------------------- index export / import
+namespace {
+struct BlobHeader {
+    uint64_t magic;  // "SJIDX001"
+    uint64_t n;
+    int32_t dim, pad, key_bits, reserved;
+    double eps, e2, w;
+    double mins[SJ_MAX_DIM];
+    uint64_t nc[SJ_MAX_DIM];
+    uint64_t stride[SJ_MAX_DIM];
+    uint64_t n_cells, fwd_entries, dist_calcs;
+    uint32_t max_w, reserved2;
+    uint64_t off[6], bytes[6];  // pts, orig, pcell, cellq, fwd, cell_lid
+    uint64_t total;
+};
+constexpr uint64_t kMagic = 0x3130305844494a53ull;  // "SJIDX001"
+constexpr uint64_t kHdr = 1024;
+static_assert(sizeof(BlobHeader) <= kHdr, "header");
+
+BlobHeader make_header(const Index &ix) {
+    BlobHeader b{};
+    b.magic = kMagic;
+    b.n = ix.n;
+    b.dim = ix.dim;
+    b.pad = ix.pad;
+    b.key_bits = ix.key_bits;
+    b.eps = ix.eps;
+    b.e2 = ix.e2;
+    b.w = ix.w;
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        b.mins[d] = ix.mins[d];
+        b.nc[d] = ix.nc[d];
+        b.stride[d] = ix.stride[d];
+    }
+    b.n_cells = ix.n_cells;
+    b.fwd_entries = ix.fwd_entries;
+    b.dist_calcs = ix.dist_calcs;
+    b.max_w = ix.max_w;
+    const uint64_t sz[6] = {ix.n * ix.pad * sizeof(double), ix.n * sizeof(uint32_t), ix.n * sizeof(uint32_t),
+                            ix.n_cells * sizeof(uint4), ix.fwd_entries * sizeof(uint2), ix.n_cells * sizeof(uint64_t)};
+    uint64_t o = kHdr;
+    for (int i = 0; i < 6; ++i) {
+        b.off[i] = o;
+        b.bytes[i] = sz[i];
+        o += (sz[i] + 255) & ~255ull;
+    }
+    b.total = o;
+    return b;
+}
+}  // namespace
+
+int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes) {
+    if (!h || !bytes) return SJ_EINVAL;
+    BlobHeader b = make_header(h->ix);
+    *bytes = b.total;
+    if (!dst) return SJ_OK;
+    if (cap < b.total) {
+        set_error("sj_export_index: cap %llu < %llu bytes", (unsigned long long)cap, (unsigned long long)b.total);
+        return SJ_EINVAL;
+    }
+    SJ_TRY(ensure_device(h));
+    char *d = static_cast<char *>(dst);
+    const void *src[6] = {h->ix.pts, h->ix.orig, h->ix.pcell, h->ix.cellq, h->ix.fwd, h->ix.cell_lid};
+    SJ_CUDA_TRY(cudaMemcpyAsync(d, &b, sizeof b, cudaMemcpyDefault, h->s_main));
+    for (int i = 0; i < 6; ++i)
+        if (b.bytes[i]) SJ_CUDA_TRY(cudaMemcpyAsync(d + b.off[i], src[i], b.bytes[i], cudaMemcpyDefault, h->s_main));
+    SJ_CUDA_TRY(cudaStreamSynchronize(h->s_main));
+    return SJ_OK;
+}
+
+sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
+    set_error("");
+    if (!blob || bytes < kHdr) {
+        set_error("sj_create_from_index: invalid blob");
+        return nullptr;
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        set_error("sj_create_from_index: no CUDA device available");
+        return nullptr;
+    }
+    BlobHeader b;
+    if (cudaMemcpy(&b, blob, sizeof b, cudaMemcpyDefault) != cudaSuccess) {
+        set_error("sj_create_from_index: %s", cudaGetErrorString(cudaGetLastError()));
+        return nullptr;
+    }
+    if (b.magic != kMagic || b.total > bytes || b.dim < 1 || b.dim > SJ_MAX_DIM) {
+        set_error("sj_create_from_index: bad header");
+        return nullptr;
+    }
+    sj_handle *h = nullptr;
+    if (create_common(&h) < 0) return nullptr;
+    Index &ix = h->ix;
+    ix.n = b.n;
+    ix.dim = b.dim;
+    ix.pad = b.pad;
+    ix.key_bits = b.key_bits;
+    ix.eps = b.eps;
+    ix.e2 = b.e2;
+    ix.w = b.w;
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        ix.mins[d] = b.mins[d];
+        ix.nc[d] = b.nc[d];
+        ix.stride[d] = b.stride[d];
+    }
+    ix.n_cells = b.n_cells;
+    ix.fwd_entries = b.fwd_entries;
+    ix.dist_calcs = b.dist_calcs;
+    ix.max_w = b.max_w;
+    cudaStream_t s = h->s_main;
+    void **dst[6] = {(void **)&ix.pts, (void **)&ix.orig, (void **)&ix.pcell, (void **)&ix.cellq, (void **)&ix.fwd,
+                     (void **)&ix.cell_lid};
+    int rc = SJ_OK;
+    for (int i = 0; i < 6 && rc == SJ_OK; ++i) {
+        rc = dev_alloc(dst[i], b.bytes[i] + 16, s);
+        if (rc == SJ_OK && b.bytes[i] &&
+            cudaMemcpyAsync(*dst[i], static_cast<const char *>(blob) + b.off[i], b.bytes[i], cudaMemcpyDefault, s) !=
+                cudaSuccess) {
+            set_error("sj_create_from_index: copy failed");
+            rc = SJ_ECUDA;
+        }
+    }
+    if (rc == SJ_OK && cudaStreamSynchronize(s) != cudaSuccess) rc = SJ_ECUDA;
+    if (rc < 0) {
+        sj_destroy(h);
+        return nullptr;
+    }
+    fill_static_stats(h);
+    return h;
+}
+
+// ---------------------------------------------------------------- host-only helpers
+int sj_forward_offsets(int dim, int8_t *out, uint64_t cap) {
+    return sj::forward_offsets_public(dim, out, cap);
+}
+
+int64_t sj_slice_positions(uint64_t n, uint32_t grab, int rank, int world, uint32_t *out, uint64_t cap) {
+    if (grab == 0 || world < 1 || rank < 0 || rank >= world || n >= (1ull << 32)) return SJ_EINVAL;
+    const uint64_t nchunks = (n + grab - 1) / grab;
+    int64_t cnt = 0;
+    for (uint64_t c = (uint64_t)rank; c < nchunks; c += (uint64_t)world) {
+        const uint64_t b = c * grab, e = std::min<uint64_t>(n, b + grab);
+        for (uint64_t q = b; q < e; ++q) {
+            if (out) {
+                if ((uint64_t)cnt >= cap) return SJ_EINVAL;
+                out[cnt] = (uint32_t)q;
+            }
+            ++cnt;
+        }
+    }
+    return cnt;
+}
+
+}  // extern "C"
