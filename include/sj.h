@@ -147,6 +147,9 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes);
 /* ABI version (SJ_ABI_VERSION). */
 int sj_abi_version(void);
 
+/* Number of CUDA kernels libsj.so has launched in this process (diagnostics). */
+uint64_t sj_kernel_launches(void);
+
 /* ---- host-only helpers (no GPU needed) ------------------------------------ */
 
 /* LID-UNICOMP forward offsets (Alg. 3): the neighbour offsets o in

@@ -49,6 +49,7 @@ _lib = ctypes.CDLL(lib_path)
 _vp, _u64, _i64, _int, _dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int64, ctypes.c_int, ctypes.c_double
 _sig = {
     "sj_abi_version": (_int, []),
+    "sj_kernel_launches": (_u64, []),
     "sj_last_error": (ctypes.c_char_p, []),
     "sj_create": (_vp, [_vp, _u64, _int, _dbl]),
     "sj_self_join": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
@@ -103,6 +104,10 @@ def _check(code: int) -> int:
 
 def sj_abi_version() -> int:
     return _lib.sj_abi_version()
+
+
+def sj_kernel_launches() -> int:
+    return int(_lib.sj_kernel_launches())
 
 
 def sj_last_error() -> str:

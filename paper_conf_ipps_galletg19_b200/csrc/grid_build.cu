@@ -423,6 +423,7 @@ static int sort_points(Temps &tmp, const double *d_raw, uint64_t n, const GridGe
     SJ_TRY(tmp.alloc(&va, n));
     SJ_TRY(tmp.alloc(&vb, n));
     cell_id_kernel<K><<<grid_for(n), kThreads, 0, s>>>(d_raw, n, geo, ka, va);
+    note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     if constexpr (sizeof(K) == 4)
         SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s));
@@ -435,10 +436,12 @@ template <class K>
 static int rle(Temps &tmp, const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *cell_lid,
                uint32_t *cell_start, uint64_t *d_M, cudaStream_t s) {
     rle_flags_kernel<K><<<grid_for(n), kThreads, 0, s>>>(ks, n, cellof);
+    note_launch();
     uint32_t *d_m32;
     SJ_TRY(tmp.alloc(&d_m32, 1));
     SJ_TRY(scan_exclusive_u32(cellof, cellof, n, d_m32, s));
     rle_write_kernel<K><<<grid_for(n), kThreads, 0, s>>>(ks, n, cellof, cell_lid, cell_start);
+    note_launch();
     // d_M (u64) <- d_m32
     SJ_CUDA_TRY(cudaMemsetAsync(d_M, 0, sizeof(uint64_t), s));
     SJ_CUDA_TRY(cudaMemcpyAsync(d_M, d_m32, sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
@@ -457,22 +460,24 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     ix.w = eps * (1.0 + 0x1p-20);      // reading c5
     if (ev0) SJ_CUDA_TRY(cudaEventRecord(ev0, s));
 
-    // pinned mailbox for the two host round trips
+    // pinned mailbox (from the process-wide pool) for the two host round trips
     static_assert(sizeof(BBox) <= 256, "bbox");
-    void *mail = nullptr;
-    SJ_CUDA_TRY(cudaMallocHost(&mail, 512));
+    void *mail = pinned_acquire();
+    if (!mail) return SJ_ENOMEM;
     struct MailFree {
         void *p;
-        ~MailFree() { cudaFreeHost(p); }
+        ~MailFree() { pinned_release(p); }
     } mail_free{mail};
 
     // ---- a2: bounding box + non-finite check
     BBox *d_bb;
     SJ_TRY(tmp.alloc(&d_bb, 1));
     bbox_init_kernel<<<1, 32, 0, s>>>(d_bb);
+    note_launch();
     {
         unsigned blocks = (unsigned)std::min<uint64_t>(grid_for(n), 148ull * 8);
         bbox_kernel<<<blocks, kThreads, 0, s>>>(d_raw, n, dim, d_bb);
+        note_launch();
     }
     SJ_CUDA_TRY(cudaGetLastError());
     SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_bb, sizeof(BBox), cudaMemcpyDeviceToHost, s));
@@ -541,6 +546,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         SJ_TRY(tmp.alloc(&tab, ncells_total));
         SJ_CUDA_TRY(cudaMemsetAsync(tab, 0xFF, ncells_total * sizeof(uint32_t), s));
         dense_fill_kernel<<<grid_for(n), kThreads, 0, s>>>(cell_lid, d_M, tab);
+        note_launch();
         L.dense = tab;
     } else {
         unsigned long long cap = 1024;
@@ -551,6 +557,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         SJ_TRY(tmp.alloc(&hv, cap));
         SJ_CUDA_TRY(cudaMemsetAsync(hk, 0xFF, cap * sizeof(unsigned long long), s));
         hash_insert_kernel<<<grid_for(n), kThreads, 0, s>>>(cell_lid, d_M, hk, hv, cap - 1);
+        note_launch();
         L.hkeys = hk;
         L.hvals = hv;
         L.hmask = cap - 1;
@@ -593,6 +600,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_CUDA_TRY(cudaMemsetAsync(d_tot, 0, sizeof(BuildTotals), s));
     fwd_kernel<false><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, fcnt, wload, nullptr,
                                                        nullptr, d_tot);
+    note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     // fbegin = exclusive scan of fcnt over M (+1 entry for the end): scan n+1 entries with
     // fcnt[r] = 0 for r >= M so fbegin[M] = E.
@@ -623,6 +631,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&fwd_rank, E + 1));
     fwd_kernel<true><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr, fbegin,
                                                       fwd_rank, nullptr);
+    note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
     // ---- a8: SortByWL over cells
@@ -632,11 +641,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wk2, M));
     SJ_TRY(tmp.alloc(&wv2, M));
     wl_keys_kernel<<<grid_for(M), kThreads, 0, s>>>(wload, M, ix.max_w, wk, wv);
+    note_launch();
     SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(ix.max_w), &qorder_keys, &qorder, s));
     uint32_t *mq, *qb;
     SJ_TRY(tmp.alloc(&mq, M));
     SJ_TRY(tmp.alloc(&qb, M));
     queue_m_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, cell_start, M, mq);
+    note_launch();
     SJ_TRY(scan_exclusive_u32(mq, qb, M, nullptr, s));
 
     // ---- final arrays
@@ -651,9 +662,14 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&qbr, M));
     cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, fbegin, cell_lid, M, ix.cellq, r2q,
                                                            qbr, ix.cell_lid);
-    if (E) fwd_convert_kernel<<<grid_for(E), kThreads, 0, s>>>(fwd_rank, E, qbr, cell_start, ix.fwd);
+    note_launch();
+    if (E) {
+        fwd_convert_kernel<<<grid_for(E), kThreads, 0, s>>>(fwd_rank, E, qbr, cell_start, ix.fwd);
+        note_launch();
+    }
     permute_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, dim, ix.pad, idx_sorted, cellof, cell_start, qbr, r2q,
                                                     ix.pts, ix.orig, ix.pcell);
+    note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));

@@ -252,6 +252,7 @@ int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaSt
         return SJ_EINVAL;
     }
     f<<<blocks, kJoinThreads, 0, s>>>(a);
+    note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     return SJ_OK;
 }

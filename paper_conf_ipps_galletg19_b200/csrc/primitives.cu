@@ -123,8 +123,11 @@ int scan_exclusive(const T *in, T *out, uint64_t n, T *d_total, cudaStream_t s) 
     T *partials = nullptr;
     SJ_TRY(dev_alloc_t(&partials, nt, s));
     scan_reduce_kernel<T><<<(unsigned)nt, kScanThreads, 0, s>>>(in, n, partials);
+    note_launch();
     scan_partials_kernel<T><<<1, 1024, 0, s>>>(partials, nt, d_total);
+    note_launch();
     scan_down_kernel<T><<<(unsigned)nt, kScanThreads, 0, s>>>(in, out, n, partials);
+    note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     dev_free(partials, s);
     return SJ_OK;
@@ -256,8 +259,10 @@ int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_
     uint32_t *va = vals, *vb = vals_alt;
     for (int shift = 0; shift < bits; shift += 8) {
         radix_hist_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, n, shift, hist, ntiles);
+        note_launch();
         SJ_TRY(scan_exclusive<uint32_t>(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s));
         radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, va, kb, vb, n, shift, hist, ntiles);
+        note_launch();
         SJ_CUDA_TRY(cudaGetLastError());
         K *tk = ka; ka = kb; kb = tk;
         uint32_t *tv = va; va = vb; vb = tv;

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <string>
 
 #include "../../include/sj.h"
@@ -36,6 +37,10 @@ struct Status {
         if (_rc < 0) return _rc;     \
     } while (0)
 
+// Process-wide count of kernels libsj.so launched (sj_kernel_launches()).
+extern std::atomic<unsigned long long> g_launches;
+inline void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
 // --------------------------------------------------------------------------- memory
 // Stream-ordered allocations from the device's default memory pool.  The pool's
 // release threshold is raised once, so repeated create/destroy cycles reuse memory
@@ -46,6 +51,12 @@ template <class T>
 inline int dev_alloc_t(T **p, size_t count, cudaStream_t s) {
     return dev_alloc(reinterpret_cast<void **>(p), count * sizeof(T) + 16, s);
 }
+
+// Process-wide free list of 4 KiB pinned host blocks ("mailboxes" for small D2H reads);
+// cudaMallocHost costs far more than a whole small join, so blocks are recycled.
+constexpr size_t kMailBytes = 4096;
+void *pinned_acquire();
+void pinned_release(void *p);
 
 // --------------------------------------------------------------------------- primitives
 // Exclusive scan of u32 (out may alias in).  total (device, optional) receives the sum.

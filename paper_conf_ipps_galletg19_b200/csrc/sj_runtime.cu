@@ -15,6 +15,8 @@
 
 namespace sj {
 
+std::atomic<unsigned long long> g_launches{0};
+
 // ------------------------------------------------------------------------- errors
 static thread_local char g_err[1024] = "";
 
@@ -54,6 +56,33 @@ int dev_alloc(void **p, size_t bytes, cudaStream_t s) {
 
 void dev_free(void *p, cudaStream_t s) {
     if (p) cudaFreeAsync(p, s);
+}
+
+static std::mutex g_pin_mu;
+static std::vector<void *> g_pin_free;
+
+void *pinned_acquire() {
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        if (!g_pin_free.empty()) {
+            void *p = g_pin_free.back();
+            g_pin_free.pop_back();
+            return p;
+        }
+    }
+    void *p = nullptr;
+    if (cudaMallocHost(&p, kMailBytes) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("pinned host allocation failed");
+        return nullptr;
+    }
+    return p;
+}
+
+void pinned_release(void *p) {
+    if (!p) return;
+    std::lock_guard<std::mutex> lk(g_pin_mu);
+    g_pin_free.push_back(p);
 }
 
 // ------------------------------------------------------------------------- small kernels
@@ -146,7 +175,8 @@ int handle_init_common(sj_handle *h) {
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_b));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_c));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_d));
-    SJ_CUDA_TRY(cudaMallocHost(&h->mail, 64 * sizeof(uint64_t)));
+    h->mail = static_cast<uint64_t *>(pinned_acquire());
+    if (!h->mail) return SJ_ENOMEM;
     SJ_TRY(dev_alloc_t(&h->d_ctr, 8, h->s_main));
     return SJ_OK;
 }
@@ -224,6 +254,7 @@ int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *
     cudaStream_t s = h->s_main;
     SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
     set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, v0);
+    note_launch();
     JoinArgs a = base_args(h);
     a.head = h->d_ctr + 1;
     a.v_end = v1;
@@ -250,6 +281,7 @@ int launch_job(sj_handle *h, Job &j, int slot_idx) {
     SJ_TRY(slot_buffer(h, s, h->batch_pairs));
     SJ_CUDA_TRY(cudaMemsetAsync(s.d_ctr, 0, 4 * sizeof(unsigned long long), s.stream));
     set_u64_kernel<<<1, 1, 0, s.stream>>>(s.d_ctr + 1, j.v0);
+    note_launch();
     JoinArgs a = base_args(h);
     a.head = s.d_ctr + 1;
     a.v_end = j.v1;
@@ -420,12 +452,17 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         set_error("sj_self_join: device out_pairs must be 16-byte aligned");
         return SJ_EINVAL;
     }
-    if (dev_out && h->fast_path && est <= 4.0 * (double)cap + 1e6) {
+    // The sample's own pairs are part of the result, so spairs is a strict lower bound of the
+    // total; the extrapolated estimate is NOT (the first 1% of D' is the heaviest part)
+    // and is only used to size the staged batches.
+    if (dev_out && h->fast_path && spairs <= cap) {
         // Fast path: the caller's HBM buffer is the result buffer; one persistent launch
-        // over the whole slice writes it in place (no staging, no D2D copy).
+        // over the whole slice writes it in place (no staging, no D2D copy).  Overflow is
+        // detected from the counter and falls back to the staged path.
         cudaStream_t s = h->s_main;
         SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
         set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, 0ull);
+        note_launch();
         JoinArgs a = base_args(h);
         a.head = h->d_ctr + 1;
         a.v_end = V;
@@ -486,6 +523,8 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
 extern "C" {
 
 int sj_abi_version(void) { return SJ_ABI_VERSION; }
+
+uint64_t sj_kernel_launches(void) { return g_launches.load(); }
 
 const char *sj_last_error(void) { return g_err; }
 
@@ -605,7 +644,7 @@ void sj_destroy(sj_handle *h) {
     if (h->ev_b) cudaEventDestroy(h->ev_b);
     if (h->ev_c) cudaEventDestroy(h->ev_c);
     if (h->ev_d) cudaEventDestroy(h->ev_d);
-    if (h->mail) cudaFreeHost(h->mail);
+    pinned_release(h->mail);
     delete h;
 }
 
