@@ -136,10 +136,10 @@ def load_profile_facts(cfg_name: str):
 
 def algorithmic_bytes(st: dict, pad: int) -> int:
     """Compulsory HBM bytes of one join launch: every ordered pair written once
-    (8 B) plus the index read once: points (pad*8 B), orig id and cell id (4+4 B) per point,
-    16 B per cell record, 8 B per forward-neighbour entry."""
-    n, m, e = st["n"], st["n_cells"], st["fwd_entries"]
-    return 8 * st["pairs"] + n * (8 * pad + 8) + 16 * m + 8 * e
+    (8 B) plus the index read once: points (pad*8 B), orig id (4 B) and the D' entry (8 B) per
+    point, 16 B per cell record, 8 B per forward run."""
+    n, m, e = st["n"], st["n_cells"], st["fwd_runs"]
+    return 8 * st["pairs"] + n * (8 * pad + 12) + 16 * m + 8 * e
 
 
 def oracle_baseline(pts, eps, d_alg: int, stride: int, budget_s: float = 20.0):
@@ -393,7 +393,7 @@ def main():
             "data": "synthetic, seeded (workloads/, SURVEY.md §8.0 recipe)",
             "config": {"workload": f"{cfg.name}: {cfg.note}", "n": cfg.n, "dim": cfg.dim, "eps": cfg.eps, "k": k,
                        "pairs": tot_pairs, "dist_calcs": d_alg, "n_cells": st0["n_cells"],
-                       "fwd_entries": st0["fwd_entries"], "parallelism": f"replicas+queue slices x{world}",
+                       "fwd_runs": st0["fwd_runs"], "parallelism": f"replicas+queue slices x{world}",
                        "l2": "flushed before every step (256 MiB write, outside the step events)",
                        "output": "HBM-resident pairs (uint32 x2), written in place"},
             "self_join_s": total_ms / args.steps / 1e3,

@@ -54,7 +54,7 @@ enum sj_option {
     SJ_OPT_BATCH_PAIRS = 2,    /* b_s, pairs per batch buffer; default 1e8                        */
     SJ_OPT_STREAMS = 3,        /* CUDA streams for batches, 1..8; default 3                       */
     SJ_OPT_SAMPLE_PPM = 4,     /* estimator sample of D' in parts per million; default 10000 = 1%*/
-    SJ_OPT_GRAB = 5,           /* queue positions one warp dequeues per atomic; multiple of 32/k; 32     */
+    SJ_OPT_GRAB = 5,           /* WorkQueue chunks one warp dequeues per atomic (1..1024); default 1     */
     SJ_OPT_COUNT_CALCS = 6,    /* 1 = instrument the join with a distance-calculation counter; default 0 */
     SJ_OPT_BLOCKS_PER_SM = 7,  /* persistent-grid CTAs per SM; 0 = occupancy maximum (default)           */
     SJ_OPT_FAST_PATH = 8       /* 1 = device output written in place when it fits (default); 0 = always
@@ -67,7 +67,9 @@ typedef struct sj_stats {
     uint32_t dim;             /* dimensionality                                      */
     uint32_t key_bits;        /* significant bits of the linear cell id              */
     uint64_t n_cells;         /* M, non-empty cells (|B|)                      */
-    uint64_t fwd_entries;     /* sum over cells of non-empty forward neighbours      */
+    uint64_t fwd_runs;        /* forward runs: per cell, the non-empty LID-UNICOMP
+                                 neighbour cells of one grid row form one contiguous
+                                 run of the lid-ordered points        */
     uint64_t dist_calcs;      /* D_alg: distance calculations of the LID-UNICOMP
                                  pattern, sum_A [C(m_A,2) + m_A * sum_fwd m_B]       */
     uint64_t calcs_measured;  /* instrumented counter of the last join (0 if off)    */
@@ -86,6 +88,9 @@ typedef struct sj_stats {
     double ms_total;          /* last sj_self_join call, device span                 */
     uint32_t fast_path;       /* 1 if the last join wrote the caller's device buffer in place */
     uint32_t nc[8];           /* cells per dimension                                 */
+    uint64_t n_chunks;        /* WorkQueue chunks of D'                              */
+    uint32_t tiled_min;       /* smallest cell (points) that gets shared-memory tiles */
+    uint32_t reserved;
 } sj_stats;
 
 /* Build the eps-grid index of `n` points of dimension `dim` (row-major AoS,
@@ -126,10 +131,11 @@ const char *sj_last_error(void);
 int sj_set_option(sj_handle *h, int opt, int64_t value);
 
 /* Restrict this handle to the queue slice of `rank` out of `world` replicas
- * (multi-GPU): D' is cut into chunks of SJ_OPT_GRAB positions and
- * chunk c belongs to rank c mod world.  Slices of all ranks are disjoint and
- * cover D'; each slice's pairs are disjoint (every unordered pair is evaluated
- * by exactly one query point).  world = 1 restores the whole queue. */
+ * (multi-GPU): D' is cut into WorkQueue chunks (at most 32
+ * positions, never straddling a cell of >= 8 points) and chunk c belongs to rank
+ * c mod world.  Slices of all ranks are disjoint and cover D'; each slice's pairs
+ * are disjoint (every unordered pair is evaluated by exactly one query point).
+ * world = 1 restores the whole queue. */
 int sj_set_slice(sj_handle *h, int rank, int world);
 
 /* Copy the statistics of the handle into *s. */
@@ -158,10 +164,10 @@ uint64_t sj_kernel_launches(void);
  * if out != NULL and cap >= F*dim.  Returns F, or SJ_EINVAL. */
 int sj_forward_offsets(int dim, int8_t *out, uint64_t cap);
 
-/* Queue positions of slice (rank, world) for n points and chunk `grab`:
+/* WorkQueue chunks of slice (rank, world) out of n_chunks (sj_stats.n_chunks):
  * writes them ascending into out (if out != NULL and cap is large enough) and
  * returns their number, or a negative sj_status. */
-int64_t sj_slice_positions(uint64_t n, uint32_t grab, int rank, int world, uint32_t *out, uint64_t cap);
+int64_t sj_slice_chunks(uint64_t n_chunks, int rank, int world, uint32_t *out, uint64_t cap);
 
 /* ---- diagnostics (GPU microbenchmarks for the roofline denominators) ------ */
 

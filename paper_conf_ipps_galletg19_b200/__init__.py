@@ -15,7 +15,7 @@ from ._lib import (  # noqa: F401
     SJError, SJStats, lib_path, header_functions,
     sj_abi_version, sj_kernel_launches, sj_last_error, sj_create, sj_create_from_index, sj_self_join, sj_destroy,
     sj_set_option, sj_set_slice, sj_get_stats, sj_export_index, sj_forward_offsets,
-    sj_slice_positions, sj_measure_fp64, sj_measure_atomics,
+    sj_slice_chunks, sj_measure_fp64, sj_measure_atomics,
     Handle, self_join_pairs,
 )
 

@@ -26,13 +26,14 @@ class SJError(RuntimeError):
 class SJStats(ctypes.Structure):
     _fields_ = [
         ("n", ctypes.c_uint64), ("dim", ctypes.c_uint32), ("key_bits", ctypes.c_uint32),
-        ("n_cells", ctypes.c_uint64), ("fwd_entries", ctypes.c_uint64), ("dist_calcs", ctypes.c_uint64),
+        ("n_cells", ctypes.c_uint64), ("fwd_runs", ctypes.c_uint64), ("dist_calcs", ctypes.c_uint64),
         ("calcs_measured", ctypes.c_uint64), ("pairs", ctypes.c_uint64), ("est_pairs", ctypes.c_uint64),
         ("batches", ctypes.c_uint32), ("retries", ctypes.c_uint32), ("join_launches", ctypes.c_uint32),
         ("k", ctypes.c_uint32), ("max_cell_load", ctypes.c_uint64),
         ("ms_build", ctypes.c_double), ("ms_estimate", ctypes.c_double), ("ms_join", ctypes.c_double),
         ("ms_join_sum", ctypes.c_double), ("ms_transfer", ctypes.c_double), ("ms_total", ctypes.c_double),
-        ("fast_path", ctypes.c_uint32), ("nc", ctypes.c_uint32 * 8),
+        ("fast_path", ctypes.c_uint32), ("nc", ctypes.c_uint32 * 8), ("n_chunks", ctypes.c_uint64),
+        ("tiled_min", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
     ]
 
     def as_dict(self) -> dict:
@@ -60,7 +61,7 @@ _sig = {
     "sj_export_index": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
     "sj_create_from_index": (_vp, [_vp, _u64]),
     "sj_forward_offsets": (_int, [_int, _vp, _u64]),
-    "sj_slice_positions": (_i64, [_u64, ctypes.c_uint32, _int, _int, _vp, _u64]),
+    "sj_slice_chunks": (_i64, [_u64, _int, _int, _vp, _u64]),
     "sj_measure_fp64": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
     "sj_measure_atomics": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
 }
@@ -182,12 +183,12 @@ def sj_forward_offsets(dim: int):
     return out
 
 
-def sj_slice_positions(n: int, grab: int, rank: int, world: int):
+def sj_slice_chunks(n_chunks: int, rank: int, world: int):
     import numpy as np
 
-    cnt = _check(_lib.sj_slice_positions(int(n), int(grab), int(rank), int(world), None, 0))
+    cnt = _check(_lib.sj_slice_chunks(int(n_chunks), int(rank), int(world), None, 0))
     out = np.zeros(max(cnt, 1), dtype=np.uint32)
-    _check(_lib.sj_slice_positions(int(n), int(grab), int(rank), int(world), out.ctypes.data, out.size))
+    _check(_lib.sj_slice_chunks(int(n_chunks), int(rank), int(world), out.ctypes.data, out.size))
     return out[:cnt]
 
 

@@ -6,9 +6,10 @@
 //      (readings c5, c6); lid = sum_d c_d * stride_d, row-major, dim 0 most significant (c7)
 //   a4 hand-written radix sort of (lid, point id) on the significant bits
 //   a5 run-length compaction -> non-empty cells B + point lookup
-//   a6 LID-UNICOMP forward neighbours (Alg. 3) resolved once per cell
+//   a6 LID-UNICOMP forward neighbours (Alg. 3) resolved once per cell into
+//      contiguous runs of the lid-ordered point storage
 //   a7 workload W(A) = ceil((m_A-1)/2) + sum_{B in fwd(A)} m_B and D_alg
-//   a8 SortByWL: cells in non-increasing W (stable, ties by lid, c10) -> D' storage order
+//   a8 SortByWL: cells in non-increasing W (stable, ties by lid, c10) -> D' (index array)
 #include <cmath>
 #include <cstring>
 #include <vector>
@@ -17,8 +18,7 @@
 
 namespace sj {
 
-__constant__ uint64_t c_fwd_off[SJ_MAX_FWD];   // packed int8 offsets, dim d in byte d
-__constant__ long long c_fwd_delta[SJ_MAX_FWD];  // sum_d o_d * stride_d
+__constant__ uint64_t c_fwd_off[SJ_MAX_FWD];  // forward rows (forward_rows()), packed int8
 
 namespace {
 
@@ -202,7 +202,7 @@ struct FwdGeom {
     unsigned long long nc[SJ_MAX_DIM];
     unsigned long long stride[SJ_MAX_DIM];
     int dim;
-    int F;
+    int rows;  // forward rows (see forward_rows())
 };
 
 struct BuildTotals {
@@ -213,22 +213,28 @@ struct BuildTotals {
     unsigned int pad;
 };
 
-// a6 + a7: count the non-empty forward neighbours of every cell (Alg. 3: neighbour
-// cells with a higher linear id) and its workload W:
-//   W(A) = ceil((m_A - 1)/2)          (balanced circulant home-cell half scan, reading c8)
-//        + sum_{B in fwd(A)} m_B       (forward cells)
-// plus the exact distance-calculation total D_alg = sum_A C(m_A,2) + m_A sum m_B.
+// a6 + a7.  LID-UNICOMP (Alg. 3) visits the neighbour cells with a higher linear
+// id.  With row-major ids those form "rows" along the last dimension: for every offset
+// o' of the first n-1 dimensions whose first non-zero component is +1, the three cells
+// o' x {-1, 0, +1}; plus, in the home row (o' = 0), the single cell +1.  The non-empty
+// cells of one row have consecutive ranks in the lid-sorted cell array, so their points
+// are ONE contiguous run of the lid-ordered point storage.  Each cell's forward
+// neighbourhood is therefore a short list of runs {begin, length}.
+//   W(A) = ceil((m_A - 1)/2)            (balanced circulant home-cell half scan, reading c8)
+//        + sum_{B in fwd(A)} m_B
+//   D_alg = sum_A C(m_A, 2) + m_A * sum_{B in fwd(A)} m_B
 template <bool FILL>
-__global__ void __launch_bounds__(kThreads) fwd_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
-                                                       const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *fcnt,
-                                                       uint32_t *wload, const uint32_t *fbegin, uint32_t *fwd_rank,
-                                                       BuildTotals *tot) {
+__global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
+                                                        const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *rcnt,
+                                                        uint32_t *wload, const uint32_t *rbegin, uint2 *runs,
+                                                        BuildTotals *tot) {
     const uint64_t M = *d_M;
     const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     unsigned long long calcs = 0;
     uint32_t w = 0;
     if (r < M) {
         const unsigned long long lid = cell_lid[r];
+        const int last = g.dim - 1;
         long long c[SJ_MAX_DIM];
 #pragma unroll
         for (int d = 0; d < SJ_MAX_DIM; ++d)
@@ -236,31 +242,45 @@ __global__ void __launch_bounds__(kThreads) fwd_kernel(const unsigned long long 
         const uint32_t m = cell_start[r + 1] - cell_start[r];
         uint32_t cnt = 0;
         unsigned long long summ = 0;
-        uint32_t out = FILL ? fbegin[r] : 0;
-        for (int j = 0; j < g.F; ++j) {
-            const unsigned long long off = c_fwd_off[j];
+        uint32_t out = FILL ? rbegin[r] : 0;
+        for (int j = 0; j < g.rows; ++j) {
+            const unsigned long long off = c_fwd_off[j];  // bytes 0..n-2: o'; byte 7: 1 = home row
             bool in = true;
+            long long base = 0;
 #pragma unroll
-            for (int d = 0; d < SJ_MAX_DIM; ++d) {
-                if (d < g.dim) {
+            for (int d = 0; d < SJ_MAX_DIM - 1; ++d) {
+                if (d < last) {
                     long long o = (long long)(signed char)((off >> (8 * d)) & 0xFF);
                     long long v = c[d] + o;
                     in = in && (v >= 0) && (v < (long long)g.nc[d]);
+                    base += v * (long long)g.stride[d];
                 }
             }
             if (!in) continue;
-            const uint32_t nb = lookup_cell(L, lid + (unsigned long long)c_fwd_delta[j]);
-            if (nb == 0xFFFFFFFFu) continue;
+            const bool home_row = (off >> 56) != 0;
+            long long lo = c[last] + (home_row ? 1 : -1);
+            long long hi = c[last] + 1;
+            if (lo < 0) lo = 0;
+            if (hi > (long long)g.nc[last] - 1) hi = (long long)g.nc[last] - 1;
+            uint32_t r_lo = 0xFFFFFFFFu, r_hi = 0;
+            for (long long x = lo; x <= hi; ++x) {
+                const uint32_t nb = lookup_cell(L, (unsigned long long)(base + x));
+                if (nb == 0xFFFFFFFFu) continue;
+                if (r_lo == 0xFFFFFFFFu) r_lo = nb;
+                r_hi = nb;
+            }
+            if (r_lo == 0xFFFFFFFFu) continue;
+            const uint32_t b = cell_start[r_lo], len = cell_start[r_hi + 1] - b;
             if (FILL) {
-                fwd_rank[out++] = nb;
+                runs[out++] = make_uint2(b, len);
             } else {
                 ++cnt;
-                summ += cell_start[nb + 1] - cell_start[nb];
+                summ += len;
             }
         }
         if (!FILL) {
-            fcnt[r] = cnt;
-            w = (uint32_t)((m - 1 + 1) / 2 + summ);  // ceil((m-1)/2) + sum m_B
+            rcnt[r] = cnt;
+            w = (uint32_t)(m / 2 + summ);  // ceil((m-1)/2) = floor(m/2) for m >= 1
             wload[r] = w;
             calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
         }
@@ -296,7 +316,8 @@ __global__ void __launch_bounds__(kThreads) queue_m_kernel(const uint32_t *qorde
 }
 
 __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t *qorder, const uint32_t *qb,
-                                                                  const uint32_t *cell_start, const uint32_t *fbegin,
+                                                                  const uint32_t *cell_start, const uint32_t *rbegin,
+                                                                  const uint32_t *wload,
                                                                   const unsigned long long *cell_lid, uint64_t M,
                                                                   uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
                                                                   uint64_t *lid_q) {
@@ -304,35 +325,59 @@ __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t
     if (i >= M) return;
     uint32_t r = qorder[i];
     uint32_t m = cell_start[r + 1] - cell_start[r];
-    cellq[i] = make_uint4(qb[i], m, fbegin[r], fbegin[r + 1]);
+    // {begin in the lid-ordered storage, m, first run, sum of the runs' lengths (= W - floor(m/2))}
+    cellq[i] = make_uint4(cell_start[r], m, rbegin[r], wload[r] - m / 2);
     r2q[r] = (uint32_t)i;
     qbr[r] = qb[i];
     lid_q[i] = cell_lid[r];
 }
 
-__global__ void __launch_bounds__(kThreads) fwd_convert_kernel(const uint32_t *fwd_rank, uint64_t E,
-                                                               const uint32_t *qbr, const uint32_t *cell_start,
-                                                               uint2 *fwd) {
-    uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (e >= E) return;
-    uint32_t nb = fwd_rank[e];
-    fwd[e] = make_uint2(qbr[nb], cell_start[nb + 1] - cell_start[nb]);
-}
-
-// Gather points into D' storage order (padded AoS, `pad` doubles per point).
+// Points gathered into lid (spatial) order, padded AoS, plus D' = the queue as an index
+// array: qmap[D' position] = {lid-storage position, queue-order cell}.
 __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, uint64_t n, int dim, int pad,
                                                            const uint32_t *idx_sorted, const uint32_t *cellof,
                                                            const uint32_t *cell_start, const uint32_t *qbr,
                                                            const uint32_t *r2q, double *pts, uint32_t *orig,
-                                                           uint32_t *pcell) {
+                                                           uint2 *qmap) {
     uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
     const uint32_t r = cellof[p];
-    const uint64_t dest = (uint64_t)qbr[r] + (p - cell_start[r]);
     const uint32_t src = idx_sorted[p];
-    for (int d = 0; d < pad; ++d) pts[dest * pad + d] = d < dim ? raw[(uint64_t)src * dim + d] : 0.0;
-    orig[dest] = src;
-    pcell[dest] = r2q[r];
+    if (pad == 2 && dim == 2) {
+        reinterpret_cast<double2 *>(pts)[p] = reinterpret_cast<const double2 *>(raw)[src];
+    } else {
+        for (int d = 0; d < pad; ++d) pts[p * pad + d] = d < dim ? raw[(uint64_t)src * dim + d] : 0.0;
+    }
+    orig[p] = src;
+    qmap[(uint64_t)qbr[r] + (p - cell_start[r])] = make_uint2((uint32_t)p, r2q[r]);
+}
+
+// WorkQueue chunks: D' is cut into chunks of at most kChunk positions so that
+// a chunk of a "big" cell (m >= big_min) never contains another cell, and consecutive small
+// cells are packed together.  A boundary sits at
+//   big cell:   every kChunk positions from the cell's first D' position;
+//   small cell: every kChunk-aligned position, and where a big cell ended.
+__global__ void __launch_bounds__(kThreads) chunk_flags_kernel(const uint2 *qmap, const uint4 *cellq, const uint32_t *qb,
+                                                               uint64_t n, uint32_t big_min, uint32_t *flags) {
+    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    const uint32_t iq = qmap[p].y;
+    const uint32_t m = cellq[iq].y, beg = qb[iq];
+    bool f;
+    if (m >= big_min) {
+        f = ((p - beg) % kChunk) == 0;
+    } else {
+        f = (p % kChunk) == 0 || (p == beg && p > 0 && cellq[qmap[p - 1].y].y >= big_min);
+    }
+    flags[p] = f ? 1u : 0u;
+}
+
+__global__ void __launch_bounds__(kThreads) chunk_write_kernel(const uint32_t *flags, const uint32_t *excl, uint64_t n,
+                                                               uint32_t *chunks) {
+    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    if (flags[p]) chunks[excl[p]] = (uint32_t)p;
+    if (p == n - 1) chunks[excl[p] + flags[p]] = (uint32_t)n;
 }
 
 int bits_for(unsigned long long maxval) {
@@ -384,15 +429,51 @@ int forward_offsets_public(int dim, int8_t *out, uint64_t cap) {
 void free_index(Index &ix, cudaStream_t s) {
     dev_free(ix.pts, s);
     dev_free(ix.orig, s);
-    dev_free(ix.pcell, s);
+    dev_free(ix.qmap, s);
     dev_free(ix.cellq, s);
-    dev_free(ix.fwd, s);
+    dev_free(ix.runs, s);
     dev_free(ix.cell_lid, s);
+    dev_free(ix.chunks, s);
+    ix.chunks = nullptr;
     ix.pts = nullptr;
-    ix.orig = ix.pcell = nullptr;
+    ix.orig = nullptr;
+    ix.qmap = nullptr;
     ix.cellq = nullptr;
-    ix.fwd = nullptr;
+    ix.runs = nullptr;
     ix.cell_lid = nullptr;
+}
+
+// Forward rows of LID-UNICOMP (see runs_kernel): the home row (o' = 0, last-dim offset +1
+// only) followed by every o' in {-1,0,1}^(dim-1) whose first non-zero component is +1 with
+// last-dim offsets -1..+1.  Packed: byte d = o'_d (d < dim-1 <= 7), byte 7 = 1 for the home row.
+static int forward_rows(int dim, std::vector<uint64_t> &rows) {
+    rows.clear();
+    auto pack = [](const int8_t *o, int nd, bool home) {
+        uint64_t p = 0;
+        for (int d = 0; d < nd; ++d) p |= (uint64_t)(uint8_t)o[d] << (8 * d);
+        if (home) p |= 1ull << 56;
+        return p;
+    };
+    int8_t zero[SJ_MAX_DIM] = {0};
+    rows.push_back(pack(zero, dim - 1, true));
+    int total = 1;
+    for (int d = 0; d < dim - 1; ++d) total *= 3;
+    for (int t = 0; t < total; ++t) {
+        int8_t o[SJ_MAX_DIM] = {0};
+        int v = t;
+        for (int d = dim - 2; d >= 0; --d) {
+            o[d] = (int8_t)(v % 3 - 1);
+            v /= 3;
+        }
+        int first = 0;
+        for (int d = 0; d < dim - 1; ++d)
+            if (o[d] != 0) {
+                first = o[d];
+                break;
+            }
+        if (first == 1) rows.push_back(pack(o, dim - 1, false));
+    }
+    return (int)rows.size();
 }
 
 namespace {
@@ -482,6 +563,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_CUDA_TRY(cudaGetLastError());
     SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_bb, sizeof(BBox), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    debug_mark("build: bbox sync");
     BBox bb;
     memcpy(&bb, mail, sizeof bb);
     if (bb.nonfinite) {
@@ -564,77 +646,59 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     }
     SJ_CUDA_TRY(cudaGetLastError());
 
-    // ---- a6 + a7: forward neighbour counts, workload, D_alg
-    std::vector<int8_t> offs;
-    const int F = forward_offsets(dim, offs);
-    {
-        std::vector<uint64_t> packed(F);
-        std::vector<long long> delta(F);
-        for (int j = 0; j < F; ++j) {
-            uint64_t p = 0;
-            long long dl = 0;
-            for (int d = 0; d < dim; ++d) {
-                p |= (uint64_t)(uint8_t)offs[(size_t)j * dim + d] << (8 * d);
-                dl += (long long)offs[(size_t)j * dim + d] * (long long)ix.stride[d];
-            }
-            packed[j] = p;
-            delta[j] = dl;
-        }
-        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, packed.data(), F * sizeof(uint64_t), 0,
-                                            cudaMemcpyHostToDevice, s));
-        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_delta, delta.data(), F * sizeof(long long), 0,
-                                            cudaMemcpyHostToDevice, s));
-    }
+    // ---- a6 + a7: forward runs, workload, D_alg
+    std::vector<uint64_t> rows;
+    const int R = forward_rows(dim, rows);
+    SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, rows.data(), R * sizeof(uint64_t), 0, cudaMemcpyHostToDevice, s));
     FwdGeom fg{};
     fg.dim = dim;
-    fg.F = F;
+    fg.rows = R;
     for (int d = 0; d < dim; ++d) {
         fg.nc[d] = ix.nc[d];
         fg.stride[d] = ix.stride[d];
     }
-    uint32_t *fcnt, *wload;
+    uint32_t *rcnt, *wload;
     BuildTotals *d_tot;
-    SJ_TRY(tmp.alloc(&fcnt, n + 1));
+    SJ_TRY(tmp.alloc(&rcnt, n + 1));
     SJ_TRY(tmp.alloc(&wload, n));
     SJ_TRY(tmp.alloc(&d_tot, 1));
     SJ_CUDA_TRY(cudaMemsetAsync(d_tot, 0, sizeof(BuildTotals), s));
-    fwd_kernel<false><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, fcnt, wload, nullptr,
-                                                       nullptr, d_tot);
+    runs_kernel<false><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload, nullptr,
+                                                        nullptr, d_tot);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
-    // fbegin = exclusive scan of fcnt over M (+1 entry for the end): scan n+1 entries with
-    // fcnt[r] = 0 for r >= M so fbegin[M] = E.
-    uint32_t *fbegin;
-    SJ_TRY(tmp.alloc(&fbegin, n + 1));
+    uint32_t *rbegin;
+    SJ_TRY(tmp.alloc(&rbegin, n + 1));
     SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_M, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    debug_mark("build: sort+rle+runcount sync");
     uint64_t M;
     memcpy(&M, mail, sizeof M);
     ix.n_cells = M;
     uint32_t *d_E32;
     SJ_TRY(tmp.alloc(&d_E32, 1));
-    SJ_CUDA_TRY(cudaMemsetAsync(fcnt + M, 0, sizeof(uint32_t), s));
-    SJ_TRY(scan_exclusive_u32(fcnt, fbegin, M + 1, d_E32, s));
+    SJ_CUDA_TRY(cudaMemsetAsync(rcnt + M, 0, sizeof(uint32_t), s));
+    SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s));
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, fbegin + M, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, rbegin + M, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    debug_mark("build: scan sync");
     BuildTotals bt;
     memcpy(&bt, mail, sizeof bt);
     uint32_t E32;
     memcpy(&E32, (char *)mail + 256, sizeof E32);
     const uint64_t E = E32;
-    ix.fwd_entries = E;
+    ix.n_runs = E;
     ix.dist_calcs = bt.dist_calcs;
     ix.max_w = bt.max_w;
 
-    uint32_t *fwd_rank;
-    SJ_TRY(tmp.alloc(&fwd_rank, E + 1));
-    fwd_kernel<true><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr, fbegin,
-                                                      fwd_rank, nullptr);
+    SJ_TRY(dev_alloc_t(&ix.runs, E + 2, s));
+    runs_kernel<true><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr, rbegin,
+                                                       ix.runs, nullptr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
-    // ---- a8: SortByWL over cells
+    // ---- a8: SortByWL over cells -> D' (queue of points in non-increasing W)
     uint32_t *wk, *wv, *wk2, *wv2, *qorder_keys, *qorder;
     SJ_TRY(tmp.alloc(&wk, M));
     SJ_TRY(tmp.alloc(&wv, M));
@@ -652,28 +716,42 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
 
     // ---- final arrays
     SJ_TRY(dev_alloc_t(&ix.cellq, M, s));
-    SJ_TRY(dev_alloc_t(&ix.fwd, E + 1, s));
     SJ_TRY(dev_alloc_t(&ix.cell_lid, M, s));
     SJ_TRY(dev_alloc_t(&ix.pts, n * ix.pad, s));
     SJ_TRY(dev_alloc_t(&ix.orig, n, s));
-    SJ_TRY(dev_alloc_t(&ix.pcell, n, s));
+    SJ_TRY(dev_alloc_t(&ix.qmap, n, s));
     uint32_t *r2q, *qbr;
     SJ_TRY(tmp.alloc(&r2q, M));
     SJ_TRY(tmp.alloc(&qbr, M));
-    cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, fbegin, cell_lid, M, ix.cellq, r2q,
-                                                           qbr, ix.cell_lid);
+    cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, rbegin, wload, cell_lid, M,
+                                                           ix.cellq, r2q, qbr, ix.cell_lid);
     note_launch();
-    if (E) {
-        fwd_convert_kernel<<<grid_for(E), kThreads, 0, s>>>(fwd_rank, E, qbr, cell_start, ix.fwd);
-        note_launch();
-    }
     permute_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, dim, ix.pad, idx_sorted, cellof, cell_start, qbr, r2q,
-                                                    ix.pts, ix.orig, ix.pcell);
+                                                    ix.pts, ix.orig, ix.qmap);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
+
+    // ---- WorkQueue chunks over D'
+    uint32_t *cflags, *cexcl, *d_nc;
+    SJ_TRY(tmp.alloc(&cflags, n));
+    SJ_TRY(tmp.alloc(&cexcl, n));
+    SJ_TRY(tmp.alloc(&d_nc, 1));
+    SJ_TRY(dev_alloc_t(&ix.chunks, n + 1, s));
+    chunk_flags_kernel<<<grid_for(n), kThreads, 0, s>>>(ix.qmap, ix.cellq, qb, n, kBigCell, cflags);
+    note_launch();
+    SJ_TRY(scan_exclusive_u32(cflags, cexcl, n, d_nc, s));
+    chunk_write_kernel<<<grid_for(n), kThreads, 0, s>>>(cflags, cexcl, n, ix.chunks);
+    note_launch();
+    SJ_CUDA_TRY(cudaGetLastError());
+    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
+    debug_mark("build: tail issued");
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    debug_mark("build: final sync");
     if (ms && ev0 && ev1) SJ_CUDA_TRY(cudaEventElapsedTime(ms, ev0, ev1));
+    uint32_t nchunks;
+    memcpy(&nchunks, (char *)mail + 512, sizeof nchunks);
+    ix.n_chunks = nchunks;
     return SJ_OK;
 }
 

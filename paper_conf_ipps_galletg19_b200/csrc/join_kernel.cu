@@ -8,8 +8,8 @@
 //   * WorkQueue, P:194-198 (§III-D): a global counter persistent for the batch is
 //     the queue head; an atomic increment hands D' (sorted by workload)
 //     out in order.  With k > 1 only a leader increments the counter and shuffles
-//     the result to its group; here the leader is lane 0 of the warp and
-//     the warp takes SJ_OPT_GRAB consecutive positions per atomic.
+//     the result to its group; here the leader is lane 0 of the warp, and a
+//     dequeue hands out a chunk of <= 32 consecutive D' positions.
 //   * k threads per query point, P:161-170 (§III-A, Fig. 4): the k lanes of a
 //     group split the query's candidates -- lane t takes candidates t, t+k, t+2k...
 //     of the concatenated candidate list, so the split stays balanced across cell
@@ -25,6 +25,10 @@
 //   * Emission: hits of a warp step are ranked with __ballot_sync/__popc into a
 //     per-warp shared-memory buffer; a full buffer is flushed with ONE atomicAdd on
 //     the batch's output counter and coalesced 16-byte streaming stores.
+//   * Cell tiles in shared memory: a chunk whose queries all lie in one cell of >= 8
+//     points shares that cell's forward runs; the warp stages them 32 candidates at a
+//     time in shared memory and every query of the chunk is evaluated against each
+//     tile (loads per distance calculation / (chunk size / k)).
 #include "sj_internal.cuh"
 
 namespace sj {
@@ -33,11 +37,22 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarps = kJoinThreads / 32;
-constexpr int kBufHits = 256;  // hits (= 2 pairs = 16 B) buffered per warp
+constexpr int kBufHits = 512;  // hits buffered per warp ({orig q, lid pos of c}, 8 B -> 4 KB)
 
 template <int DIM>
 struct PointPad {
     static constexpr int value = DIM == 1 ? 1 : ((DIM + 1) & ~1);
+};
+
+// Per-warp shared memory: emission buffer, the chunk's queries, one candidate tile.
+template <int DIM, bool EMIT>
+struct WarpSmem {
+    static constexpr int PAD = PointPad<DIM>::value;
+    alignas(16) double tile[32 * PAD];  // staged candidates (lid order)
+    alignas(16) double qry[32 * PAD];   // the chunk's query points
+    unsigned tile_pos[32];              // lid positions of the staged candidates
+    unsigned qorig[32];                 // input ids of the chunk's queries
+    alignas(16) uint2 buf[EMIT ? kBufHits : 2];
 };
 
 template <int DIM>
@@ -54,6 +69,32 @@ __device__ __forceinline__ void load_point(const double *__restrict__ p, double 
     }
 }
 
+template <int DIM>
+__device__ __forceinline__ void load_smem_point(const double *p, double (&x)[DIM]) {
+    if constexpr (DIM == 1) {
+        x[0] = p[0];
+    } else {
+#pragma unroll
+        for (int d = 0; d < DIM; d += 2) {
+            const double2 v = *reinterpret_cast<const double2 *>(p + d);
+            x[d] = v.x;
+            if (d + 1 < DIM) x[d + 1] = v.y;
+        }
+    }
+}
+
+template <int DIM>
+__device__ __forceinline__ void copy_point_to_smem(const double *__restrict__ src, double *dst) {
+    constexpr int PAD = PointPad<DIM>::value;
+    if constexpr (PAD == 1) {
+        dst[0] = __ldg(src);
+    } else {
+#pragma unroll
+        for (int d = 0; d < PAD; d += 2)
+            *reinterpret_cast<double2 *>(dst + d) = __ldg(reinterpret_cast<const double2 *>(src + d));
+    }
+}
+
 // s = fl(...fl(fl(t0*t0) + fl(t1*t1)) + ...), t_d = fl(q_d - c_d)  (readings c1/c2)
 template <int DIM>
 __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&c)[DIM]) {
@@ -67,37 +108,221 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
     return s;
 }
 
-__device__ __forceinline__ void flush(uint4 *buf, int nbuf, const JoinArgs &a, int lane) {
+// Flush a warp's staged hits: ONE atomicAdd reserves 2*nbuf output slots, then every lane
+// translates its entries' lid positions to input ids (independent loads -> memory-level
+// parallelism off the hot loop) and writes both mirrored pairs with one 16-B streaming store.
+__device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane) {
     __syncwarp();
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd(a.emit_ctr, 2ull * (unsigned long long)nbuf);
     base = __shfl_sync(kFull, base, 0);
     uint4 *out4 = reinterpret_cast<uint4 *>(a.out);
     uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
+#pragma unroll 4
     for (int k = lane; k < nbuf; k += 32) {
         const unsigned long long slot = base + 2ull * (unsigned long long)k;  // even
-        const uint4 v = buf[k];
+        const uint2 v = buf[k];                                              // {orig q, lid pos of c}
+        const unsigned oc = __ldg(a.orig + v.y);
         if (slot + 2 <= a.out_cap)
-            __stcs(out4 + (slot >> 1), v);
+            __stcs(out4 + (slot >> 1), make_uint4(v.x, oc, oc, v.x));  // (q,c) and (c,q)
         else if (slot < a.out_cap)
-            __stcs(out2 + slot, make_uint2(v.x, v.y));
+            __stcs(out2 + slot, make_uint2(v.x, oc));
     }
     __syncwarp();
+}
+
+// Warp-aggregated emission of one evaluation step (all 32 lanes call it).
+template <bool EMIT>
+__device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned cpos, uint2 *buf, int &nbuf,
+                                     unsigned long long &nhits, const JoinArgs &a, int lane, unsigned lt) {
+    if constexpr (EMIT) {
+        const unsigned hm = __ballot_sync(kFull, hit);
+        if (hm) {
+            if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, cpos);
+            nbuf += __popc(hm);
+            if (nbuf > kBufHits - 32) {
+                flush(buf, nbuf, a, lane);
+                nbuf = 0;
+            }
+        }
+    } else {
+        nhits += hit ? 2ull : 0ull;
+    }
+}
+
+// Home cell of one query: the balanced circulant half scan (reading c8) -- position rr
+// compares to rr+1 .. rr+floor((m-1)/2) (mod m), plus rr+m/2 when m is even and rr < m/2.
+__device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
+    return (m - 1u) / 2u + (((m & 1u) == 0u && rr < m / 2u) ? 1u : 0u);
+}
+
+// Generic path: rounds of 32/k queries (possibly from different cells); the k lanes of a
+// group walk their query's list -- forward runs first (identical for queries of one cell,
+// so their loads coincide), then the home half scan -- taking candidates t, t+k, ...
+template <int DIM, int K, bool EMIT>
+__device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint2 *buf, int &nbuf,
+                                              unsigned long long &nhits, unsigned long long &ncalcs, int lane,
+                                              unsigned lt) {
+    constexpr int PAD = PointPad<DIM>::value;
+    constexpr int QPW = 32 / K;
+    const int grp = lane / K;
+    const unsigned t = (unsigned)(lane % K);
+    for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+        const unsigned qi = r0 + grp;
+        const bool valid = qi < nq;
+        const unsigned qlid = __shfl_sync(kFull, qm_lane.x, qi & 31);
+        const unsigned qcell = __shfl_sync(kFull, qm_lane.y, qi & 31);
+        double qp[DIM];
+        unsigned oq = 0;
+        uint4 ci = make_uint4(0, 0, 0, 0);
+        if (valid) {
+            ci = __ldg(a.cellq + qcell);
+            load_point<DIM>(a.pts + (size_t)qlid * PAD, qp);
+            oq = __ldg(a.orig + qlid);
+        } else {
+#pragma unroll
+            for (int d = 0; d < DIM; ++d) qp[d] = 0.0;
+        }
+        const unsigned hb = ci.x, m = ci.y;
+        unsigned e = ci.z;
+        unsigned rem = ci.w;  // forward candidates not yet entered
+        const unsigned rr = qlid - hb;
+        const unsigned home_len = valid ? home_count(m, rr) : 0u;
+        const unsigned total = valid ? rem + home_len : 0u;
+        unsigned seg_base = 0, seg_len = 0;
+        bool home = false;
+        uint2 nxt = (valid && rem) ? __ldg(a.runs + e) : make_uint2(0, 0);  // prefetched next run
+        unsigned i = t;  // lane t takes candidates t, t+k, ... of the list (Fig. 4)
+        const unsigned my_iters = (total + (unsigned)K - 1u - t) / (unsigned)K;
+        const unsigned iters = __reduce_max_sync(kFull, my_iters);  // warp-uniform trip count
+        ncalcs += my_iters;
+        unsigned gi = t;
+        for (unsigned it = 0; it < iters; ++it, gi += K) {
+            bool hit = false;
+            unsigned cidx = 0;
+            if (gi < total) {
+                while (i >= seg_len) {  // step to the run holding candidate gi
+                    i -= seg_len;
+                    if (rem) {
+                        seg_base = nxt.x;
+                        seg_len = nxt.y;
+                        rem -= nxt.y;
+                        if (rem) nxt = __ldg(a.runs + (++e));
+                    } else {
+                        seg_base = hb;
+                        seg_len = home_len;
+                        home = true;
+                    }
+                }
+                if (home) {
+                    unsigned j = rr + 1u + i;
+                    if (j >= m) j -= m;
+                    cidx = hb + j;
+                } else {
+                    cidx = seg_base + i;
+                }
+                double cp[DIM];
+                load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
+                hit = sqdist<DIM>(qp, cp) <= a.e2;
+                i += K;
+            }
+            emit<EMIT>(hit, oq, cidx, buf, nbuf, nhits, a, lane, lt);
+        }
+    }
+}
+
+// Tiled path: all nq queries of the chunk lie in one cell (hb, m, runs rb.., S candidates).
+// The forward runs are staged 32 candidates at a time in shared memory; every round of
+// 32/k queries evaluates the whole tile (lane t of a group: tile slots t, t+k, ...).
+template <int DIM, int K, bool EMIT>
+__device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint4 ci,
+                                            WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
+                                            unsigned long long &ncalcs, int lane, unsigned lt) {
+    constexpr int PAD = PointPad<DIM>::value;
+    constexpr int QPW = 32 / K;
+    const int grp = lane / K;
+    const unsigned t = (unsigned)(lane % K);
+    const unsigned hb = ci.x, m = ci.y, S = ci.w;
+    __syncwarp();
+    if ((unsigned)lane < nq) {
+        copy_point_to_smem<DIM>(a.pts + (size_t)qm_lane.x * PAD, ws.qry + lane * PAD);
+        ws.qorig[lane] = __ldg(a.orig + qm_lane.x);
+    }
+    // ---- forward runs, staged
+    unsigned e = ci.z, seg_base = 0, seg_len = 0, i = (unsigned)lane;
+    for (unsigned tb = 0; tb < S; tb += 32) {
+        __syncwarp();
+        if (tb + (unsigned)lane < S) {
+            while (i >= seg_len) {
+                i -= seg_len;
+                const uint2 f = __ldg(a.runs + (e++));
+                seg_base = f.x;
+                seg_len = f.y;
+            }
+            const unsigned cidx = seg_base + i;
+            copy_point_to_smem<DIM>(a.pts + (size_t)cidx * PAD, ws.tile + lane * PAD);
+            ws.tile_pos[lane] = cidx;
+            i += 32;
+        }
+        __syncwarp();
+        const unsigned nt = min(32u, S - tb);
+        for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+            const unsigned qi = r0 + grp;
+            const bool qv = qi < nq;
+            double qq[DIM];
+            load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
+            const unsigned oq = ws.qorig[qi & 31];
+#pragma unroll
+            for (int s = 0; s < 32 / K; ++s) {
+                const unsigned j = t + (unsigned)(K * s);
+                bool hit = false;
+                if (qv && j < nt) {
+                    double cp[DIM];
+                    load_smem_point<DIM>(ws.tile + j * PAD, cp);
+                    hit = sqdist<DIM>(qq, cp) <= a.e2;
+                }
+                emit<EMIT>(hit, oq, hit ? ws.tile_pos[j] : 0u, ws.buf, nbuf, nhits, a, lane, lt);
+            }
+        }
+    }
+    // ---- home cell, per round, straight from global memory (the cell is small and hot in L1)
+    for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+        const unsigned qi = r0 + grp;
+        const bool qv = qi < nq;
+        const unsigned qlid = __shfl_sync(kFull, qm_lane.x, qi & 31);
+        const unsigned rr = qlid - hb;
+        const unsigned home_len = qv ? home_count(m, rr) : 0u;
+        double qq[DIM];
+        load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
+        const unsigned oq = ws.qorig[qi & 31];
+        if (qv && t == 0) ncalcs += (unsigned long long)S + home_len;
+        const unsigned iters = __reduce_max_sync(kFull, (home_len + (unsigned)K - 1u - t) / (unsigned)K);
+        for (unsigned it = 0; it < iters; ++it) {
+            const unsigned ii = t + (unsigned)K * it;
+            bool hit = false;
+            unsigned cidx = 0;
+            if (ii < home_len) {
+                unsigned j = rr + 1u + ii;
+                if (j >= m) j -= m;
+                cidx = hb + j;
+                double cp[DIM];
+                load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
+                hit = sqdist<DIM>(qq, cp) <= a.e2;
+            }
+            emit<EMIT>(hit, oq, cidx, ws.buf, nbuf, nhits, a, lane, lt);
+        }
+    }
 }
 
 template <int DIM, int K, bool EMIT>
 __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     static_assert(32 % K == 0, "k must divide 32");
-    constexpr int PAD = PointPad<DIM>::value;
-    constexpr int QPW = 32 / K;  // query points per warp step
-    __shared__ uint4 sbuf[EMIT ? kWarps : 1][EMIT ? kBufHits : 1];
-
+    constexpr int QPW = 32 / K;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    const int grp = lane / K;
-    const unsigned t = (unsigned)(lane % K);
     const unsigned lt = (1u << lane) - 1u;
-    uint4 *buf = sbuf[EMIT ? warp : 0];
+    WarpSmem<DIM, EMIT> &ws = reinterpret_cast<WarpSmem<DIM, EMIT> *>(smem_raw)[warp];
     int nbuf = 0;
     unsigned long long nhits = 0;
     unsigned long long ncalcs = 0;
@@ -108,89 +333,25 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         if (lane == 0) vb = atomicAdd(a.head, (unsigned long long)a.grab);
         vb = __shfl_sync(kFull, vb, 0);
         if (vb >= a.v_end) break;
-        // queue slice (multi-GPU): virtual chunk -> physical chunk
-        const unsigned long long pchunk = (vb / a.grab) * a.world + a.rank;
-        const unsigned long long qbase = pchunk * a.grab;
-        const unsigned long long qlim = min(qbase + a.grab, (unsigned long long)a.n);
-
-        for (unsigned r0 = 0; r0 < a.grab; r0 += QPW) {
-            const unsigned long long q = qbase + r0 + grp;
-            const bool valid = q < qlim;
-            if (!__any_sync(kFull, valid)) break;
-
-            double qp[DIM];
-            unsigned oq = 0;
-            uint4 ci = make_uint4(0, 0, 0, 0);
-            if (valid) {
-                load_point<DIM>(a.pts + q * PAD, qp);
-                oq = __ldg(a.orig + q);
-                ci = __ldg(a.cellq + __ldg(a.pcell + q));
-            } else {
-#pragma unroll
-                for (int d = 0; d < DIM; ++d) qp[d] = 0.0;
-            }
-            const unsigned hb = ci.x, m = ci.y;
-            unsigned e = ci.z;
-            const unsigned fe = ci.w;
-            const unsigned rr = (unsigned)(q - hb);
-            // home cell: balanced circulant half scan (reading c8)
-            unsigned seg_len = valid ? ((m - 1u) / 2u + (((m & 1u) == 0u && rr < m / 2u) ? 1u : 0u)) : 0u;
-            unsigned seg_base = hb;
-            bool home = true;
-            bool done = !valid;
-            unsigned i = t;  // lane t takes candidates t, t+k, ... (Fig. 4)
-
-            for (;;) {
-                while (!done && i >= seg_len) {
-                    i -= seg_len;
-                    if (e >= fe) {
-                        done = true;
-                    } else {
-                        const uint2 f = __ldg(a.fwd + e);  // next forward cell (LID-UNICOMP)
-                        ++e;
-                        seg_base = f.x;
-                        seg_len = f.y;
-                        home = false;
-                    }
-                }
-                if (__ballot_sync(kFull, !done) == 0u) break;
-                bool hit = false;
-                unsigned cidx = 0;
-                if (!done) {
-                    if (home) {
-                        unsigned j = rr + 1u + i;
-                        if (j >= m) j -= m;
-                        cidx = hb + j;
-                    } else {
-                        cidx = seg_base + i;
-                    }
-                    double cp[DIM];
-                    load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
-                    hit = sqdist<DIM>(qp, cp) <= a.e2;
-                    i += K;
-                    ++ncalcs;
-                }
-                if constexpr (EMIT) {
-                    const unsigned hm = __ballot_sync(kFull, hit);
-                    if (hm) {
-                        if (hit) {
-                            const unsigned oc = __ldg(a.orig + cidx);
-                            buf[nbuf + __popc(hm & lt)] = make_uint4(oq, oc, oc, oq);  // (q,c) and (c,q)
-                        }
-                        nbuf += __popc(hm);
-                        if (nbuf > kBufHits - 32) {
-                            flush(buf, nbuf, a, lane);
-                            nbuf = 0;
-                        }
-                    }
-                } else {
-                    nhits += hit ? 2ull : 0ull;
-                }
-            }
+        const unsigned long long vend = min(vb + a.grab, a.v_end);
+        for (unsigned long long v = vb; v < vend; ++v) {
+            const unsigned long long c = v * a.world + a.rank;  // queue slice (multi-GPU)
+            if (c >= a.n_chunks) break;
+            const unsigned qs = __ldg(a.chunks + c), qe = __ldg(a.chunks + c + 1);
+            const unsigned nq = qe - qs;  // 1..32 D' positions
+            const bool lv = (unsigned)lane < nq;
+            const uint2 qm = lv ? __ldg(a.qmap + qs + lane) : make_uint2(0, 0xFFFFFFFFu);
+            const unsigned cell0 = __shfl_sync(kFull, qm.y, 0);
+            const bool same = __all_sync(kFull, !lv || qm.y == cell0);
+            const uint4 ci0 = __ldg(a.cellq + cell0);
+            if (same && ci0.y >= kBigCell && nq >= 2u * QPW)
+                tiled_chunk<DIM, K, EMIT>(a, nq, qm, ci0, ws, nbuf, nhits, ncalcs, lane, lt);
+            else
+                generic_chunk<DIM, K, EMIT>(a, nq, qm, ws.buf, nbuf, nhits, ncalcs, lane, lt);
         }
     }
     if constexpr (EMIT) {
-        if (nbuf > 0) flush(buf, nbuf, a, lane);
+        if (nbuf > 0) flush(ws.buf, nbuf, a, lane);
     } else {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) nhits += __shfl_xor_sync(kFull, nhits, o);
@@ -205,21 +366,34 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
 
 typedef void (*join_fn)(const JoinArgs);
 
+struct KernelInfo {
+    join_fn f = nullptr;
+    size_t smem = 0;
+};
+
+template <int DIM, int K, bool EMIT>
+KernelInfo info() {
+    KernelInfo ki;
+    ki.f = join_kernel<DIM, K, EMIT>;
+    ki.smem = sizeof(WarpSmem<DIM, EMIT>) * kWarps;
+    return ki;
+}
+
 template <int DIM, bool EMIT>
-join_fn pick_k(int k) {
+KernelInfo pick_k(int k) {
     switch (k) {
-        case 1: return join_kernel<DIM, 1, EMIT>;
-        case 2: return join_kernel<DIM, 2, EMIT>;
-        case 4: return join_kernel<DIM, 4, EMIT>;
-        case 8: return join_kernel<DIM, 8, EMIT>;
-        case 16: return join_kernel<DIM, 16, EMIT>;
-        case 32: return join_kernel<DIM, 32, EMIT>;
+        case 1: return info<DIM, 1, EMIT>();
+        case 2: return info<DIM, 2, EMIT>();
+        case 4: return info<DIM, 4, EMIT>();
+        case 8: return info<DIM, 8, EMIT>();
+        case 16: return info<DIM, 16, EMIT>();
+        case 32: return info<DIM, 32, EMIT>();
     }
-    return nullptr;
+    return KernelInfo();
 }
 
 template <bool EMIT>
-join_fn pick(int dim, int k) {
+KernelInfo pick(int dim, int k) {
     switch (dim) {
         case 1: return pick_k<1, EMIT>(k);
         case 2: return pick_k<2, EMIT>(k);
@@ -230,28 +404,33 @@ join_fn pick(int dim, int k) {
         case 7: return pick_k<7, EMIT>(k);
         case 8: return pick_k<8, EMIT>(k);
     }
-    return nullptr;
+    return KernelInfo();
+}
+
+int prepare(int dim, int k, bool emit, KernelInfo *out) {
+    KernelInfo ki = emit ? pick<true>(dim, k) : pick<false>(dim, k);
+    if (!ki.f) {
+        set_error("join: unsupported dim=%d k=%d", dim, k);
+        return SJ_EINVAL;
+    }
+    SJ_CUDA_TRY(cudaFuncSetAttribute(ki.f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ki.smem));
+    *out = ki;
+    return SJ_OK;
 }
 
 }  // namespace
 
 int join_occupancy(int dim, int k, bool emit, int *blocks_per_sm) {
-    join_fn f = emit ? pick<true>(dim, k) : pick<false>(dim, k);
-    if (!f) {
-        set_error("join: unsupported dim=%d k=%d", dim, k);
-        return SJ_EINVAL;
-    }
-    SJ_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, f, kJoinThreads, 0));
+    KernelInfo ki;
+    SJ_TRY(prepare(dim, k, emit, &ki));
+    SJ_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, ki.f, kJoinThreads, ki.smem));
     return SJ_OK;
 }
 
 int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaStream_t s) {
-    join_fn f = emit ? pick<true>(dim, k) : pick<false>(dim, k);
-    if (!f) {
-        set_error("join: unsupported dim=%d k=%d", dim, k);
-        return SJ_EINVAL;
-    }
-    f<<<blocks, kJoinThreads, 0, s>>>(a);
+    KernelInfo ki;
+    SJ_TRY(prepare(dim, k, emit, &ki));
+    ki.f<<<blocks, kJoinThreads, ki.smem, s>>>(a);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     return SJ_OK;

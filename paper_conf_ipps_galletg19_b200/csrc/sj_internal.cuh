@@ -14,6 +14,11 @@
 #define SJ_MAX_DIM 8
 #define SJ_MAX_FWD 3280  // (3^8 - 1) / 2
 
+// WorkQueue chunk: at most kChunk D' positions; cells with at least kBigCell points get
+// chunks of their own.
+constexpr unsigned kChunk = 32;
+constexpr unsigned kBigCell = 8;
+
 namespace sj {
 
 // --------------------------------------------------------------------------- errors
@@ -40,6 +45,9 @@ struct Status {
 // Process-wide count of kernels libsj.so launched (sj_kernel_launches()).
 extern std::atomic<unsigned long long> g_launches;
 inline void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+// Host-side phase timer printed to stderr when SJ_DEBUG=1 (diagnostics only).
+void debug_mark(const char *label);
 
 // --------------------------------------------------------------------------- memory
 // Stream-ordered allocations from the device's default memory pool.  The pool's
@@ -87,16 +95,18 @@ struct Index {
     uint64_t stride[SJ_MAX_DIM] = {0};
     int key_bits = 0;
     uint64_t n_cells = 0;     // M
-    uint64_t fwd_entries = 0; // E
+    uint64_t n_runs = 0;      // E, forward runs over all cells
     uint64_t dist_calcs = 0;  // D_alg
     uint32_t max_w = 0;
 
-    double *pts = nullptr;      // [n * pad]  D' order
-    uint32_t *orig = nullptr;   // [n]        D' position -> input id
-    uint32_t *pcell = nullptr;  // [n]        D' position -> queue-order cell index
-    uint4 *cellq = nullptr;     // [M]        queue-order cell: {begin in D', m, fwd_begin, fwd_end}
-    uint2 *fwd = nullptr;       // [E]        forward neighbour cell: {begin in D', m}
+    double *pts = nullptr;      // [n * pad]  points in lid (spatial) order, padded AoS
+    uint32_t *orig = nullptr;   // [n]        lid position -> input id
+    uint2 *qmap = nullptr;      // [n]        D' (queue) position -> {lid position, queue-order cell}
+    uint4 *cellq = nullptr;     // [M]        queue-order cell: {lid begin, m, first run, sum of run lengths}
+    uint2 *runs = nullptr;      // [E]        forward run: {lid begin, length}
     uint64_t *cell_lid = nullptr; // [M]      queue-order cell -> linear id (export / tests)
+    uint32_t *chunks = nullptr; // [C+1]      WorkQueue chunk c = D' positions [chunks[c], chunks[c+1])
+    uint64_t n_chunks = 0;      // C
 };
 
 struct BuildTimes {
@@ -114,15 +124,16 @@ int forward_offsets_public(int dim, int8_t *out, uint64_t cap);
 struct JoinArgs {
     const double *pts;
     const uint32_t *orig;
-    const uint32_t *pcell;
+    const uint2 *qmap;
     const uint4 *cellq;
-    const uint2 *fwd;
+    const uint2 *runs;
+    const uint32_t *chunks;       // WorkQueue chunks of D'
+    uint32_t n_chunks;
     double e2;
-    unsigned long long *head;     // dequeue counter (virtual queue positions)
-    unsigned long long v_end;     // end of this batch (virtual)
-    uint32_t n;                   // points
-    uint32_t grab;                // positions per dequeue (= slice chunk)
-    uint32_t rank, world;         // queue slice
+    unsigned long long *head;     // dequeue counter (virtual chunk index of this slice)
+    unsigned long long v_end;     // end of this batch (virtual chunk index)
+    uint32_t grab;                // chunks per dequeue
+    uint32_t rank, world;         // queue slice: virtual chunk v -> chunk v*world + rank
     uint32_t *out;                // interleaved pairs, or nullptr (count-only)
     unsigned long long *emit_ctr; // pairs emitted (may exceed out_cap -> overflow)
     unsigned long long out_cap;   // capacity of out in pairs

@@ -3,6 +3,8 @@
 // batch loop, overflow retry, SJ_MORE continuation, statistics,
 // index export/import for the NCCL broadcast, and the host-only helpers.
 #include <algorithm>
+#include <chrono>
+#include <cstdlib>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -25,6 +27,18 @@ void set_error(const char *fmt, ...) {
     va_start(ap, fmt);
     vsnprintf(g_err, sizeof g_err, fmt, ap);
     va_end(ap);
+}
+
+void debug_mark(const char *label) {
+    static const bool on = [] {
+        const char *e = getenv("SJ_DEBUG");
+        return e && e[0] == '1';
+    }();
+    if (!on) return;
+    static thread_local std::chrono::steady_clock::time_point last = std::chrono::steady_clock::now();
+    auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "[sj] %-28s %9.3f ms\n", label, std::chrono::duration<double, std::milli>(now - last).count());
+    last = now;
 }
 
 // ------------------------------------------------------------------------- memory
@@ -98,7 +112,7 @@ namespace {
 constexpr int kMaxStreams = 8;
 
 struct Job {
-    uint64_t v0, v1;  // virtual queue range [v0, v1), multiples of grab
+    uint64_t v0, v1;  // virtual WorkQueue chunk range [v0, v1) of this handle's slice
     int slot = -1;
     bool launched = false, complete = false;
     uint64_t cnt = 0, consumed = 0;
@@ -129,7 +143,7 @@ struct sj_handle {
     uint64_t batch_pairs = 100000000ull;
     int streams = 3;
     uint32_t sample_ppm = 10000;
-    uint32_t grab = 32;
+    uint32_t grab = 1;
     int count_calcs = 0;
     int blocks_per_sm = 0;
     int fast_path = 1;
@@ -218,9 +232,9 @@ void slots_release(sj_handle *h) {
     }
 }
 
-// number of virtual queue positions of this handle's slice (multiple of grab)
+// number of WorkQueue chunks of this handle's slice (chunk c belongs to rank c mod world)
 uint64_t slice_chunks(const sj_handle *h) {
-    const uint64_t nchunks = (h->ix.n + h->grab - 1) / h->grab;
+    const uint64_t nchunks = h->ix.n_chunks;
     if (nchunks <= (uint64_t)h->rank) return 0;
     return (nchunks - (uint64_t)h->rank + (uint64_t)h->world - 1) / (uint64_t)h->world;
 }
@@ -229,11 +243,12 @@ JoinArgs base_args(const sj_handle *h) {
     JoinArgs a{};
     a.pts = h->ix.pts;
     a.orig = h->ix.orig;
-    a.pcell = h->ix.pcell;
+    a.qmap = h->ix.qmap;
     a.cellq = h->ix.cellq;
-    a.fwd = h->ix.fwd;
+    a.runs = h->ix.runs;
+    a.chunks = h->ix.chunks;
+    a.n_chunks = (uint32_t)h->ix.n_chunks;
     a.e2 = h->ix.e2;
-    a.n = (uint32_t)h->ix.n;
     a.grab = h->grab;
     a.rank = (uint32_t)h->rank;
     a.world = (uint32_t)h->world;
@@ -340,7 +355,7 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
                 h->st.retries++;
                 if (h->count_calcs) h->st.calcs_measured -= m[2];
                 const Job old = j;
-                const uint64_t chunks = (old.v1 - old.v0) / h->grab;
+                const uint64_t chunks = old.v1 - old.v0;
                 h->jobs.pop_front();
                 s.busy = false;
                 if (chunks <= 1) {
@@ -354,8 +369,8 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
                     const uint64_t parts = std::min<uint64_t>(chunks, old.cnt / s.cap + 2);
                     for (uint64_t p = parts; p-- > 0;) {
                         Job nj;
-                        nj.v0 = old.v0 + (chunks * p / parts) * h->grab;
-                        nj.v1 = old.v0 + (chunks * (p + 1) / parts) * h->grab;
+                        nj.v0 = old.v0 + chunks * p / parts;
+                        nj.v1 = old.v0 + chunks * (p + 1) / parts;
                         if (nj.v1 > nj.v0) h->jobs.push_front(nj);
                     }
                     h->st.batches += (uint32_t)(parts - 1);
@@ -411,7 +426,7 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     for (int i = 0; i < kMaxStreams; ++i) h->slots[i].busy = false;
 
     const uint64_t nch = slice_chunks(h);
-    const uint64_t V = nch * h->grab;
+    const uint64_t V = nch;
     SJ_CUDA_TRY(cudaEventRecord(h->ev_a, h->s_main));
 
     if (out == nullptr) {  // count-only (whole slice, one launch)
@@ -438,7 +453,9 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     if (sch > nch) sch = nch;
     uint64_t spairs = 0;
     float ms_est = 0;
-    if (nch) SJ_TRY(count_range(h, 0, sch * h->grab, &spairs, &ms_est));
+    debug_mark("join: enter");
+    if (nch) SJ_TRY(count_range(h, 0, sch, &spairs, &ms_est));
+    debug_mark("join: estimator");
     h->st.ms_estimate = ms_est;
     h->st.calcs_measured = 0;
     const double est = nch ? (double)spairs * (double)nch / (double)sch : 0.0;
@@ -483,6 +500,7 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         h->st.batches = 1;
         h->st.ms_join = h->st.ms_join_sum = ms;
         const uint64_t total = h->mail[0];
+        debug_mark("join: fast path");
         if (total <= cap) {
             if (h->count_calcs) h->st.calcs_measured = h->mail[2];
             h->st.pairs = total;
@@ -508,8 +526,8 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     for (int i = 0; i < h->streams; ++i) SJ_CUDA_TRY(cudaStreamWaitEvent(h->slots[i].stream, h->ev_c, 0));
     for (uint64_t b = 0; b < nb; ++b) {
         Job j;
-        j.v0 = (nch * b / nb) * h->grab;
-        j.v1 = (nch * (b + 1) / nb) * h->grab;
+        j.v0 = nch * b / nb;
+        j.v1 = nch * (b + 1) / nb;
         if (j.v1 > j.v0) h->jobs.push_back(j);
     }
     h->st.batches = (uint32_t)h->jobs.size();
@@ -549,11 +567,13 @@ static void fill_static_stats(sj_handle *h) {
     st.dim = (uint32_t)h->ix.dim;
     st.key_bits = (uint32_t)h->ix.key_bits;
     st.n_cells = h->ix.n_cells;
-    st.fwd_entries = h->ix.fwd_entries;
+    st.fwd_runs = h->ix.n_runs;
     st.dist_calcs = h->ix.dist_calcs;
     st.max_cell_load = h->ix.max_w;
     st.k = (uint32_t)h->k;
     for (int d = 0; d < SJ_MAX_DIM; ++d) st.nc[d] = d < h->ix.dim ? (uint32_t)h->ix.nc[d] : 0;
+    st.n_chunks = h->ix.n_chunks;
+    st.tiled_min = kBigCell;
 }
 
 sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
@@ -569,8 +589,10 @@ sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
         set_error("sj_create: no CUDA device available (the CUDA path has no CPU fallback)");
         return nullptr;
     }
+    debug_mark("create: enter");
     sj_handle *h = nullptr;
     if (create_common(&h) < 0) return nullptr;
+    debug_mark("create: handle init");
     cudaStream_t s = h->s_main;
     const double *d_raw = points;
     double *d_copy = nullptr;
@@ -588,7 +610,9 @@ sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
         d_raw = d_copy;
     }
     float ms = 0;
+    debug_mark("create: upload issued");
     if (rc == SJ_OK) rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_a, h->ev_b, &ms);
+    debug_mark("create: build_index");
     dev_free(d_copy, s);
     if (rc == SJ_OK && cudaStreamSynchronize(s) != cudaSuccess) {
         set_error("sj_create: %s", cudaGetErrorString(cudaGetLastError()));
@@ -631,6 +655,7 @@ int sj_self_join(sj_handle *h, uint32_t *out_pairs, uint64_t cap, uint64_t *coun
 
 void sj_destroy(sj_handle *h) {
     if (!h) return;
+    debug_mark("destroy: enter");
     cudaSetDevice(h->device);
     slots_release(h);
     if (h->s_main) {
@@ -646,6 +671,7 @@ void sj_destroy(sj_handle *h) {
     if (h->ev_d) cudaEventDestroy(h->ev_d);
     pinned_release(h->mail);
     delete h;
+    debug_mark("destroy: done");
 }
 
 int sj_set_option(sj_handle *h, int opt, int64_t v) {
@@ -654,7 +680,6 @@ int sj_set_option(sj_handle *h, int opt, int64_t v) {
         case SJ_OPT_K:
             if (v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32) break;
             h->k = (int)v;
-            if (h->grab % (32 / h->k)) h->grab = ((h->grab + 32 / h->k - 1) / (32 / h->k)) * (32 / h->k);
             h->st.k = (uint32_t)v;
             return SJ_OK;
         case SJ_OPT_BATCH_PAIRS:
@@ -670,7 +695,7 @@ int sj_set_option(sj_handle *h, int opt, int64_t v) {
             h->sample_ppm = (uint32_t)v;
             return SJ_OK;
         case SJ_OPT_GRAB:
-            if (v < 1 || v > (1 << 20) || (v % (32 / h->k)) != 0) break;
+            if (v < 1 || v > 1024) break;
             h->grab = (uint32_t)v;
             return SJ_OK;
         case SJ_OPT_COUNT_CALCS:
@@ -708,19 +733,19 @@ int sj_get_stats(const sj_handle *h, sj_stats *s) {
 // ---------------------------------------------------------------- index export / import
 namespace {
 struct BlobHeader {
-    uint64_t magic;  // "SJIDX001"
+    uint64_t magic;  // "SJIDX003"
     uint64_t n;
     int32_t dim, pad, key_bits, reserved;
     double eps, e2, w;
     double mins[SJ_MAX_DIM];
     uint64_t nc[SJ_MAX_DIM];
     uint64_t stride[SJ_MAX_DIM];
-    uint64_t n_cells, fwd_entries, dist_calcs;
+    uint64_t n_cells, n_runs, dist_calcs, n_chunks;
     uint32_t max_w, reserved2;
-    uint64_t off[6], bytes[6];  // pts, orig, pcell, cellq, fwd, cell_lid
+    uint64_t off[7], bytes[7];  // pts, orig, qmap, cellq, runs, cell_lid, chunks
     uint64_t total;
 };
-constexpr uint64_t kMagic = 0x3130305844494a53ull;  // "SJIDX001"
+constexpr uint64_t kMagic = 0x3330305844494a53ull;  // "SJIDX003"
 constexpr uint64_t kHdr = 1024;
 static_assert(sizeof(BlobHeader) <= kHdr, "header");
 
@@ -740,13 +765,15 @@ BlobHeader make_header(const Index &ix) {
         b.stride[d] = ix.stride[d];
     }
     b.n_cells = ix.n_cells;
-    b.fwd_entries = ix.fwd_entries;
+    b.n_runs = ix.n_runs;
+    b.n_chunks = ix.n_chunks;
     b.dist_calcs = ix.dist_calcs;
     b.max_w = ix.max_w;
-    const uint64_t sz[6] = {ix.n * ix.pad * sizeof(double), ix.n * sizeof(uint32_t), ix.n * sizeof(uint32_t),
-                            ix.n_cells * sizeof(uint4), ix.fwd_entries * sizeof(uint2), ix.n_cells * sizeof(uint64_t)};
+    const uint64_t sz[7] = {ix.n * ix.pad * sizeof(double), ix.n * sizeof(uint32_t), ix.n * sizeof(uint2),
+                            ix.n_cells * sizeof(uint4), ix.n_runs * sizeof(uint2), ix.n_cells * sizeof(uint64_t),
+                            (ix.n_chunks + 1) * sizeof(uint32_t)};
     uint64_t o = kHdr;
-    for (int i = 0; i < 6; ++i) {
+    for (int i = 0; i < 7; ++i) {
         b.off[i] = o;
         b.bytes[i] = sz[i];
         o += (sz[i] + 255) & ~255ull;
@@ -767,9 +794,9 @@ int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes
     }
     SJ_TRY(ensure_device(h));
     char *d = static_cast<char *>(dst);
-    const void *src[6] = {h->ix.pts, h->ix.orig, h->ix.pcell, h->ix.cellq, h->ix.fwd, h->ix.cell_lid};
+    const void *src[7] = {h->ix.pts, h->ix.orig, h->ix.qmap, h->ix.cellq, h->ix.runs, h->ix.cell_lid, h->ix.chunks};
     SJ_CUDA_TRY(cudaMemcpyAsync(d, &b, sizeof b, cudaMemcpyDefault, h->s_main));
-    for (int i = 0; i < 6; ++i)
+    for (int i = 0; i < 7; ++i)
         if (b.bytes[i]) SJ_CUDA_TRY(cudaMemcpyAsync(d + b.off[i], src[i], b.bytes[i], cudaMemcpyDefault, h->s_main));
     SJ_CUDA_TRY(cudaStreamSynchronize(h->s_main));
     return SJ_OK;
@@ -812,15 +839,16 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
         ix.stride[d] = b.stride[d];
     }
     ix.n_cells = b.n_cells;
-    ix.fwd_entries = b.fwd_entries;
+    ix.n_runs = b.n_runs;
+    ix.n_chunks = b.n_chunks;
     ix.dist_calcs = b.dist_calcs;
     ix.max_w = b.max_w;
     cudaStream_t s = h->s_main;
-    void **dst[6] = {(void **)&ix.pts, (void **)&ix.orig, (void **)&ix.pcell, (void **)&ix.cellq, (void **)&ix.fwd,
-                     (void **)&ix.cell_lid};
+    void **dst[7] = {(void **)&ix.pts,  (void **)&ix.orig,     (void **)&ix.qmap,  (void **)&ix.cellq,
+                     (void **)&ix.runs, (void **)&ix.cell_lid, (void **)&ix.chunks};
     int rc = SJ_OK;
-    for (int i = 0; i < 6 && rc == SJ_OK; ++i) {
-        rc = dev_alloc(dst[i], b.bytes[i] + 16, s);
+    for (int i = 0; i < 7 && rc == SJ_OK; ++i) {
+        rc = dev_alloc(dst[i], b.bytes[i] + 32, s);
         if (rc == SJ_OK && b.bytes[i] &&
             cudaMemcpyAsync(*dst[i], static_cast<const char *>(blob) + b.off[i], b.bytes[i], cudaMemcpyDefault, s) !=
                 cudaSuccess) {
@@ -842,19 +870,15 @@ int sj_forward_offsets(int dim, int8_t *out, uint64_t cap) {
     return sj::forward_offsets_public(dim, out, cap);
 }
 
-int64_t sj_slice_positions(uint64_t n, uint32_t grab, int rank, int world, uint32_t *out, uint64_t cap) {
-    if (grab == 0 || world < 1 || rank < 0 || rank >= world || n >= (1ull << 32)) return SJ_EINVAL;
-    const uint64_t nchunks = (n + grab - 1) / grab;
+int64_t sj_slice_chunks(uint64_t n_chunks, int rank, int world, uint32_t *out, uint64_t cap) {
+    if (world < 1 || rank < 0 || rank >= world || n_chunks >= (1ull << 32)) return SJ_EINVAL;
     int64_t cnt = 0;
-    for (uint64_t c = (uint64_t)rank; c < nchunks; c += (uint64_t)world) {
-        const uint64_t b = c * grab, e = std::min<uint64_t>(n, b + grab);
-        for (uint64_t q = b; q < e; ++q) {
-            if (out) {
-                if ((uint64_t)cnt >= cap) return SJ_EINVAL;
-                out[cnt] = (uint32_t)q;
-            }
-            ++cnt;
+    for (uint64_t c = (uint64_t)rank; c < n_chunks; c += (uint64_t)world) {
+        if (out) {
+            if ((uint64_t)cnt >= cap) return SJ_EINVAL;
+            out[cnt] = (uint32_t)c;
         }
+        ++cnt;
     }
     return cnt;
 }

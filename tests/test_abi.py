@@ -58,17 +58,19 @@ def test_forward_offsets_rejects_bad_dim():
         sj.sj_forward_offsets(9)
 
 
-@pytest.mark.parametrize("n,grab,world", [(10, 3, 2), (1000, 32, 3), (1001, 4, 8), (5, 32, 4), (64, 32, 2)])
-def test_slice_positions_disjoint_cover(n, grab, world):
-    allpos = []
+@pytest.mark.parametrize("nch,world", [(10, 2), (1000, 3), (1001, 8), (5, 4), (64, 2), (1, 1)])
+def test_slice_chunks_disjoint_cover(nch, world):
+    allc = []
     for r in range(world):
-        p = sj.sj_slice_positions(n, grab, r, world)
-        assert np.all(np.diff(p.astype(np.int64)) > 0)
+        c = sj.sj_slice_chunks(nch, r, world)
+        assert np.all(np.diff(c.astype(np.int64)) > 0)
         # chunk c belongs to rank c mod world
-        assert np.all((p // grab) % world == r)
-        allpos.append(p)
-    cat = np.concatenate(allpos)
-    assert np.array_equal(np.sort(cat), np.arange(n, dtype=np.uint32))
+        assert np.all(c % world == r)
+        allc.append(c)
+    cat = np.concatenate(allc)
+    assert np.array_equal(np.sort(cat), np.arange(nch, dtype=np.uint32))
+    sizes = [len(c) for c in allc]
+    assert max(sizes) - min(sizes) <= 1
 
 
 def test_fails_loudly_without_gpu():

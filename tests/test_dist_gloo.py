@@ -41,8 +41,8 @@ def _worker(rank, world, port, q):
         res["sum"] = sjdist.allreduce_counts([rank + 1, 10 * rank], device="cpu")
         res["max"] = sjdist.allreduce_counts([100 + rank], device="cpu", op=dist.ReduceOp.MAX)
         # 3. queue slices of this rank, gathered
-        n, grab = 10_007, 32
-        mine = torch.from_numpy(sj.sj_slice_positions(n, grab, rank, world).astype(np.int64))
+        n = 10_007  # WorkQueue chunks
+        mine = torch.from_numpy(sj.sj_slice_chunks(n, rank, world).astype(np.int64))
         sizes = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
         dist.all_gather(sizes, torch.tensor([mine.numel()]))
         maxlen = int(max(s.item() for s in sizes))
@@ -79,4 +79,4 @@ def test_gloo_plumbing(world):
         assert res["sum"] == [sum(i + 1 for i in range(world)), sum(10 * i for i in range(world))]
         assert res["max"] == [100 + world - 1]
         assert res["cover"] and res["disjoint"]
-        assert res["balanced"] <= 32  # ranks differ by at most one chunk
+        assert res["balanced"] <= 1  # ranks differ by at most one chunk
