@@ -37,7 +37,7 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarps = kJoinThreads / 32;
-constexpr int kBufHits = 512;  // hits buffered per warp ({orig q, lid pos of c}, 8 B -> 4 KB)
+constexpr int kBufHits = 512;  // hits buffered per warp ({orig q, orig c}, 8 B -> 4 KB)
 
 template <int DIM>
 struct PointPad {
@@ -50,7 +50,7 @@ struct WarpSmem {
     static constexpr int PAD = PointPad<DIM>::value;
     alignas(16) double tile[32 * PAD];  // staged candidates (lid order)
     alignas(16) double qry[32 * PAD];   // the chunk's query points
-    unsigned tile_pos[32];              // lid positions of the staged candidates
+    unsigned tile_orig[32];             // input ids of the staged candidates
     unsigned qorig[32];                 // input ids of the chunk's queries
     alignas(16) uint2 buf[EMIT ? kBufHits : 2];
 };
@@ -108,45 +108,57 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
     return s;
 }
 
-// Flush a warp's staged hits: ONE atomicAdd reserves 2*nbuf output slots, then every lane
-// translates its entries' lid positions to input ids (independent loads -> memory-level
-// parallelism off the hot loop) and writes both mirrored pairs with one 16-B streaming store.
+// Flush a warp's staged hits: ONE atomicAdd reserves 2*nbuf output slots, then the lanes
+// write both mirrored pairs of each hit with one 16-B streaming store (coalesced).
 __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane) {
     __syncwarp();
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd(a.emit_ctr, 2ull * (unsigned long long)nbuf);
     base = __shfl_sync(kFull, base, 0);
-    uint4 *out4 = reinterpret_cast<uint4 *>(a.out);
-    uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
+    uint4 *out4 = reinterpret_cast<uint4 *>(a.out) + (base >> 1);  // base is even
+    if (base + 2ull * (unsigned long long)nbuf <= a.out_cap) {
 #pragma unroll 4
-    for (int k = lane; k < nbuf; k += 32) {
-        const unsigned long long slot = base + 2ull * (unsigned long long)k;  // even
-        const uint2 v = buf[k];                                              // {orig q, lid pos of c}
-        const unsigned oc = __ldg(a.orig + v.y);
-        if (slot + 2 <= a.out_cap)
-            __stcs(out4 + (slot >> 1), make_uint4(v.x, oc, oc, v.x));  // (q,c) and (c,q)
-        else if (slot < a.out_cap)
-            __stcs(out2 + slot, make_uint2(v.x, oc));
+        for (int k = lane; k < nbuf; k += 32) {
+            const uint2 v = buf[k];  // {orig q, orig c}
+            __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));  // (q,c) and (c,q)
+        }
+    } else {  // overflow: keep what fits, the counter still reports the total
+        uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
+        for (int k = lane; k < nbuf; k += 32) {
+            const unsigned long long slot = base + 2ull * (unsigned long long)k;
+            const uint2 v = buf[k];
+            if (slot + 2 <= a.out_cap)
+                __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));
+            else if (slot < a.out_cap)
+                __stcs(out2 + slot, make_uint2(v.x, v.y));
+        }
     }
     __syncwarp();
 }
 
-// Warp-aggregated emission of one evaluation step (all 32 lanes call it).
+// Warp-aggregated emission of one evaluation step (all 32 lanes call it): the hits are
+// ranked with __ballot_sync/__popc into the warp's shared buffer.  Before each round the
+// caller makes room for the round's maximum number of hits (flush_if) instead of checking
+// after every step.
 template <bool EMIT>
-__device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned cpos, uint2 *buf, int &nbuf,
-                                     unsigned long long &nhits, const JoinArgs &a, int lane, unsigned lt) {
+__device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *buf, int &nbuf,
+                                     unsigned long long &nhits, unsigned lt) {
     if constexpr (EMIT) {
         const unsigned hm = __ballot_sync(kFull, hit);
-        if (hm) {
-            if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, cpos);
-            nbuf += __popc(hm);
-            if (nbuf > kBufHits - 32) {
-                flush(buf, nbuf, a, lane);
-                nbuf = 0;
-            }
-        }
+        if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, oc);
+        nbuf += __popc(hm);
     } else {
         nhits += hit ? 2ull : 0ull;
+    }
+}
+
+template <bool EMIT>
+__device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane) {
+    if constexpr (EMIT) {
+        if (nbuf > kBufHits - room) {
+            flush(buf, nbuf, a, lane);
+            nbuf = 0;
+        }
     }
 }
 
@@ -226,20 +238,25 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, ui
                 hit = sqdist<DIM>(qp, cp) <= a.e2;
                 i += K;
             }
-            emit<EMIT>(hit, oq, cidx, buf, nbuf, nhits, a, lane, lt);
+            const unsigned oc = (EMIT && hit) ? __ldg(a.orig + cidx) : 0u;
+            flush_if<EMIT>(buf, nbuf, 32, a, lane);
+            emit<EMIT>(hit, oq, oc, buf, nbuf, nhits, lt);
         }
     }
 }
 
 // Tiled path: all nq queries of the chunk lie in one cell (hb, m, runs rb.., S candidates).
-// The forward runs are staged 32 candidates at a time in shared memory; every round of
-// 32/k queries evaluates the whole tile (lane t of a group: tile slots t, t+k, ...).
+// The forward runs are staged 32 candidates at a time in shared memory (points + input
+// ids); lane t of a group holds tile slots t, t+k, ... in registers and evaluates them
+// against one query per round of 32/k queries, so each staged candidate serves the whole
+// chunk.
 template <int DIM, int K, bool EMIT>
 __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint4 ci,
                                             WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
                                             unsigned long long &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
+    constexpr int SPL = 32 / K;  // tile slots per lane
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
     const unsigned hb = ci.x, m = ci.y, S = ci.w;
@@ -261,27 +278,53 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint
             }
             const unsigned cidx = seg_base + i;
             copy_point_to_smem<DIM>(a.pts + (size_t)cidx * PAD, ws.tile + lane * PAD);
-            ws.tile_pos[lane] = cidx;
+            ws.tile_orig[lane] = __ldg(a.orig + cidx);
             i += 32;
         }
         __syncwarp();
         const unsigned nt = min(32u, S - tb);
-        for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
-            const unsigned qi = r0 + grp;
-            const bool qv = qi < nq;
-            double qq[DIM];
-            load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
-            const unsigned oq = ws.qorig[qi & 31];
+        if constexpr (SPL <= 4 && DIM <= 3) {  // tile slots in registers (register budget)
+            double cp[SPL][DIM];
+            unsigned co[SPL];
+            bool cv[SPL];
 #pragma unroll
-            for (int s = 0; s < 32 / K; ++s) {
+            for (int s = 0; s < SPL; ++s) {
                 const unsigned j = t + (unsigned)(K * s);
-                bool hit = false;
-                if (qv && j < nt) {
-                    double cp[DIM];
-                    load_smem_point<DIM>(ws.tile + j * PAD, cp);
-                    hit = sqdist<DIM>(qq, cp) <= a.e2;
+                cv[s] = j < nt;
+                load_smem_point<DIM>(ws.tile + (j & 31) * PAD, cp[s]);
+                co[s] = ws.tile_orig[j & 31];
+            }
+            for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+                const unsigned qi = r0 + grp;
+                const bool qv = qi < nq;
+                double qq[DIM];
+                load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
+                const unsigned oq = ws.qorig[qi & 31];
+                flush_if<EMIT>(ws.buf, nbuf, 32 * SPL, a, lane);
+#pragma unroll
+                for (int s = 0; s < SPL; ++s) {
+                    const bool hit = qv && cv[s] && sqdist<DIM>(qq, cp[s]) <= a.e2;
+                    emit<EMIT>(hit, oq, co[s], ws.buf, nbuf, nhits, lt);
                 }
-                emit<EMIT>(hit, oq, hit ? ws.tile_pos[j] : 0u, ws.buf, nbuf, nhits, a, lane, lt);
+            }
+        } else {
+            for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+                const unsigned qi = r0 + grp;
+                const bool qv = qi < nq;
+                double qq[DIM];
+                load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
+                const unsigned oq = ws.qorig[qi & 31];
+                for (int s = 0; s < SPL; ++s) {
+                    const unsigned j = t + (unsigned)(K * s);
+                    bool hit = false;
+                    if (qv && j < nt) {
+                        double cp[DIM];
+                        load_smem_point<DIM>(ws.tile + j * PAD, cp);
+                        hit = sqdist<DIM>(qq, cp) <= a.e2;
+                    }
+                    flush_if<EMIT>(ws.buf, nbuf, 32, a, lane);
+                    emit<EMIT>(hit, oq, ws.tile_orig[j & 31], ws.buf, nbuf, nhits, lt);
+                }
             }
         }
     }
@@ -309,7 +352,9 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint
                 load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
                 hit = sqdist<DIM>(qq, cp) <= a.e2;
             }
-            emit<EMIT>(hit, oq, cidx, ws.buf, nbuf, nhits, a, lane, lt);
+            const unsigned oc = (EMIT && hit) ? __ldg(a.orig + cidx) : 0u;
+            flush_if<EMIT>(ws.buf, nbuf, 32, a, lane);
+            emit<EMIT>(hit, oq, oc, ws.buf, nbuf, nhits, lt);
         }
     }
 }
