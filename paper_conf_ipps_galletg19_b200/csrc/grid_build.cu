@@ -14,6 +14,7 @@
 #include <cstring>
 #include <vector>
 
+#include "scan.cuh"
 #include "sj_internal.cuh"
 
 namespace sj {
@@ -123,28 +124,36 @@ __global__ void __launch_bounds__(kThreads) cell_id_kernel(const double *raw, ui
     vals[i] = (uint32_t)i;
 }
 
-// a5: run-length flags over the sorted ids
+// a5: run-length compaction of the sorted ids, fused into one single-pass scan:
+// flag(p) = (p == 0 || key[p] != key[p-1]); a flagged p starts cell ex = excl(p).
 template <class K>
-__global__ void __launch_bounds__(kThreads) rle_flags_kernel(const K *ks, uint64_t n, uint32_t *flags) {
-    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (p >= n) return;
-    flags[p] = (p == 0 || ks[p] != ks[p - 1]) ? 1u : 0u;
-}
-
+struct RleLoad {
+    const K *ks;
+    __device__ unsigned operator()(uint64_t p) const { return (p == 0 || ks[p] != ks[p - 1]) ? 1u : 0u; }
+};
 template <class K>
-__global__ void __launch_bounds__(kThreads) rle_write_kernel(const K *ks, uint64_t n, uint32_t *excl_to_cellof,
-                                                             unsigned long long *cell_lid, uint32_t *cell_start) {
-    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (p >= n) return;
-    const bool flag = (p == 0 || ks[p] != ks[p - 1]);
-    const uint32_t ex = excl_to_cellof[p];
-    if (flag) {
-        cell_lid[ex] = (unsigned long long)ks[p];
-        cell_start[ex] = (uint32_t)p;
+struct RleStore {
+    const K *ks;
+    uint32_t *cellof;
+    unsigned long long *cell_lid;
+    uint32_t *cell_start;
+    __device__ void operator()(uint64_t p, unsigned ex, unsigned flag) const {
+        if (flag) {
+            cell_lid[ex] = (unsigned long long)ks[p];
+            cell_start[ex] = (uint32_t)p;
+        }
+        cellof[p] = flag ? ex : ex - 1;  // point (sorted position) -> cell rank
     }
-    excl_to_cellof[p] = flag ? ex : ex - 1;  // point (sorted position) -> cell rank
-    if (p == n - 1) cell_start[ex + (flag ? 1 : 0)] = (uint32_t)n;
-}
+};
+struct RleDone {
+    uint64_t n;
+    uint32_t *cell_start;
+    uint64_t *d_M;
+    __device__ void operator()(unsigned total) const {
+        cell_start[total] = (uint32_t)n;
+        *d_M = total;
+    }
+};
 
 // ---------------------------------------------------------------- lid -> cell rank lookup
 struct Lookup {
@@ -202,7 +211,8 @@ struct FwdGeom {
     unsigned long long nc[SJ_MAX_DIM];
     unsigned long long stride[SJ_MAX_DIM];
     int dim;
-    int rows;  // forward rows (see forward_rows())
+    int rows;   // forward rows (see forward_rows())
+    int small;  // prod(nc) < 2^32: 32-bit lid arithmetic
 };
 
 struct BuildTotals {
@@ -223,77 +233,157 @@ struct BuildTotals {
 //   W(A) = ceil((m_A - 1)/2)            (balanced circulant home-cell half scan, reading c8)
 //        + sum_{B in fwd(A)} m_B
 //   D_alg = sum_A C(m_A, 2) + m_A * sum_{B in fwd(A)} m_B
-template <bool FILL>
+// Cell coordinates from a row-major linear id (c_0 most significant): n-1 divisions,
+// 32-bit when the whole grid has < 2^32 cells.
+__device__ __forceinline__ void decode_lid(unsigned long long lid, const FwdGeom &g, long long (&c)[SJ_MAX_DIM]) {
+    if (g.small) {
+        unsigned rem = (unsigned)lid;
+#pragma unroll
+        for (int d = 0; d < SJ_MAX_DIM; ++d) {
+            if (d < g.dim - 1) {
+                const unsigned st = (unsigned)g.stride[d];
+                const unsigned q = rem / st;
+                c[d] = q;
+                rem -= q * st;
+            } else if (d == g.dim - 1) {
+                c[d] = rem;
+            }
+        }
+    } else {
+        unsigned long long rem = lid;
+#pragma unroll
+        for (int d = 0; d < SJ_MAX_DIM; ++d) {
+            if (d < g.dim - 1) {
+                const unsigned long long q = rem / g.stride[d];
+                c[d] = (long long)q;
+                rem -= q * g.stride[d];
+            } else if (d == g.dim - 1) {
+                c[d] = (long long)rem;
+            }
+        }
+    }
+}
+
+// One forward row of cell c (see forward_rows()): the non-empty cells among the row's <= 3
+// cells have consecutive ranks, so their points are one run [b, b+len) of the lid-ordered
+// storage.  The <= 3 lookups are issued together.
+__device__ __forceinline__ bool eval_row(int j, const long long (&c)[SJ_MAX_DIM], const FwdGeom &g, const Lookup &L,
+                                         const uint32_t *cell_start, uint32_t &b, uint32_t &len) {
+    const unsigned long long off = c_fwd_off[j];  // bytes 0..n-2: o'; byte 7: 1 = home row
+    const int last = g.dim - 1;
+    bool in = true;
+    long long base = 0;
+#pragma unroll
+    for (int d = 0; d < SJ_MAX_DIM - 1; ++d) {
+        if (d < last) {
+            const long long o = (long long)(signed char)((off >> (8 * d)) & 0xFF);
+            const long long v = c[d] + o;
+            in = in && (v >= 0) && (v < (long long)g.nc[d]);
+            base += v * (long long)g.stride[d];
+        }
+    }
+    if (!in) return false;
+    const bool home_row = (off >> 56) != 0;
+    const long long x0 = c[last] + (home_row ? 1 : -1);
+    const int nx = home_row ? 1 : 3;
+    uint32_t nb[3];
+#pragma unroll
+    for (int u = 0; u < 3; ++u) {
+        const long long x = x0 + u;
+        const bool ok = u < nx && x >= 0 && x < (long long)g.nc[last];
+        nb[u] = ok ? lookup_cell(L, (unsigned long long)(base + x)) : 0xFFFFFFFFu;
+    }
+    uint32_t r_lo = 0xFFFFFFFFu, r_hi = 0xFFFFFFFFu;
+#pragma unroll
+    for (int u = 2; u >= 0; --u)
+        if (nb[u] != 0xFFFFFFFFu) r_lo = nb[u];
+#pragma unroll
+    for (int u = 0; u < 3; ++u)
+        if (nb[u] != 0xFFFFFFFFu) r_hi = nb[u];
+    if (r_lo == 0xFFFFFFFFu) return false;
+    b = cell_start[r_lo];
+    len = cell_start[r_hi + 1] - b;
+    return true;
+}
+
+// a6 + a7 over the forward rows; LPC lanes per cell (1, or 32 when there are many rows:
+// 6-D has 122) so the independent lookups of a cell run in parallel.
+template <bool FILL, int LPC>
 __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
                                                         const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *rcnt,
                                                         uint32_t *wload, const uint32_t *rbegin, uint2 *runs,
                                                         BuildTotals *tot) {
     const uint64_t M = *d_M;
-    const uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t gt = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t r = gt / LPC;
+    const unsigned sub = (unsigned)(gt % LPC);
+    const unsigned lane = threadIdx.x & 31;
     unsigned long long calcs = 0;
     uint32_t w = 0;
-    if (r < M) {
-        const unsigned long long lid = cell_lid[r];
-        const int last = g.dim - 1;
+    const bool valid = r < M;  // uniform across the LPC lanes of a cell
+    if (LPC == 1 ? valid : __any_sync(0xffffffffu, valid)) {
         long long c[SJ_MAX_DIM];
-#pragma unroll
-        for (int d = 0; d < SJ_MAX_DIM; ++d)
-            if (d < g.dim) c[d] = (long long)((lid / g.stride[d]) % g.nc[d]);
-        const uint32_t m = cell_start[r + 1] - cell_start[r];
+        uint32_t m = 0, out = 0;
+        if (valid) {
+            decode_lid(cell_lid[r], g, c);
+            m = cell_start[r + 1] - cell_start[r];
+            if (FILL) out = rbegin[r];
+        }
         uint32_t cnt = 0;
         unsigned long long summ = 0;
-        uint32_t out = FILL ? rbegin[r] : 0;
-        for (int j = 0; j < g.rows; ++j) {
-            const unsigned long long off = c_fwd_off[j];  // bytes 0..n-2: o'; byte 7: 1 = home row
-            bool in = true;
-            long long base = 0;
-#pragma unroll
-            for (int d = 0; d < SJ_MAX_DIM - 1; ++d) {
-                if (d < last) {
-                    long long o = (long long)(signed char)((off >> (8 * d)) & 0xFF);
-                    long long v = c[d] + o;
-                    in = in && (v >= 0) && (v < (long long)g.nc[d]);
-                    base += v * (long long)g.stride[d];
-                }
-            }
-            if (!in) continue;
-            const bool home_row = (off >> 56) != 0;
-            long long lo = c[last] + (home_row ? 1 : -1);
-            long long hi = c[last] + 1;
-            if (lo < 0) lo = 0;
-            if (hi > (long long)g.nc[last] - 1) hi = (long long)g.nc[last] - 1;
-            uint32_t r_lo = 0xFFFFFFFFu, r_hi = 0;
-            for (long long x = lo; x <= hi; ++x) {
-                const uint32_t nb = lookup_cell(L, (unsigned long long)(base + x));
-                if (nb == 0xFFFFFFFFu) continue;
-                if (r_lo == 0xFFFFFFFFu) r_lo = nb;
-                r_hi = nb;
-            }
-            if (r_lo == 0xFFFFFFFFu) continue;
-            const uint32_t b = cell_start[r_lo], len = cell_start[r_hi + 1] - b;
+        for (int jb = 0; jb < g.rows; jb += LPC) {
+            const int j = jb + (int)sub;
+            uint32_t b = 0, len = 0;
+            const bool found = valid && j < g.rows && eval_row(j, c, g, L, cell_start, b, len);
             if (FILL) {
-                runs[out++] = make_uint2(b, len);
-            } else {
+                if (LPC == 1) {
+                    if (found) runs[out++] = make_uint2(b, len);
+                } else {
+                    const unsigned fm = __ballot_sync(0xffffffffu, found);
+                    if (found) runs[out + __popc(fm & ((1u << lane) - 1u))] = make_uint2(b, len);
+                    out += __popc(fm);
+                }
+            } else if (found) {
                 ++cnt;
                 summ += len;
             }
         }
         if (!FILL) {
-            rcnt[r] = cnt;
-            w = (uint32_t)(m / 2 + summ);  // ceil((m-1)/2) = floor(m/2) for m >= 1
-            wload[r] = w;
-            calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
+            if (LPC == 32) {
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+                    summ += __shfl_xor_sync(0xffffffffu, summ, o);
+                }
+            }
+            if (valid && sub == 0) {
+                rcnt[r] = cnt;
+                w = (uint32_t)(m / 2 + summ);  // ceil((m-1)/2) = floor(m/2) for m >= 1
+                wload[r] = w;
+                calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
+            }
         }
     }
-    if (!FILL) {
+    if (!FILL) {  // block reduction, then ONE pair of global atomics per block
+        __shared__ unsigned long long s_calcs[kThreads / 32];
+        __shared__ uint32_t s_w[kThreads / 32];
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             calcs += __shfl_xor_sync(0xffffffffu, calcs, o);
             w = max(w, __shfl_xor_sync(0xffffffffu, w, o));
         }
-        if ((threadIdx.x & 31) == 0) {
+        if (lane == 0) {
+            s_calcs[threadIdx.x >> 5] = calcs;
+            s_w[threadIdx.x >> 5] = w;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int i = 1; i < kThreads / 32; ++i) {
+                calcs += s_calcs[i];
+                w = max(w, s_w[i]);
+            }
             if (calcs) atomicAdd(&tot->dist_calcs, calcs);
-            atomicMax(&tot->max_w, w);
+            if (w) atomicMax(&tot->max_w, w);
         }
     }
 }
@@ -357,28 +447,38 @@ __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, ui
 // cells are packed together.  A boundary sits at
 //   big cell:   every kChunk positions from the cell's first D' position;
 //   small cell: every kChunk-aligned position, and where a big cell ended.
-__global__ void __launch_bounds__(kThreads) chunk_flags_kernel(const uint2 *qmap, const uint4 *cellq, const uint32_t *qb,
-                                                               uint64_t n, uint32_t big_min, uint32_t *flags) {
-    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (p >= n) return;
-    const uint32_t iq = qmap[p].y;
-    const uint32_t m = cellq[iq].y, beg = qb[iq];
-    bool f;
-    if (m >= big_min) {
-        f = ((p - beg) % kChunk) == 0;
-    } else {
-        f = (p % kChunk) == 0 || (p == beg && p > 0 && cellq[qmap[p - 1].y].y >= big_min);
+// Flags, their scan and the boundary scatter are one fused single-pass scan.
+struct ChunkLoad {
+    const uint2 *qmap;
+    const uint4 *cellq;
+    const uint32_t *qb;
+    uint32_t big_min;
+    __device__ unsigned operator()(uint64_t p) const {
+        const uint32_t iq = qmap[p].y;
+        const uint32_t m = cellq[iq].y, beg = qb[iq];
+        bool f;
+        if (m >= big_min)
+            f = ((p - beg) % kChunk) == 0;
+        else
+            f = (p % kChunk) == 0 || (p == beg && p > 0 && cellq[qmap[p - 1].y].y >= big_min);
+        return f ? 1u : 0u;
     }
-    flags[p] = f ? 1u : 0u;
-}
-
-__global__ void __launch_bounds__(kThreads) chunk_write_kernel(const uint32_t *flags, const uint32_t *excl, uint64_t n,
-                                                               uint32_t *chunks) {
-    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (p >= n) return;
-    if (flags[p]) chunks[excl[p]] = (uint32_t)p;
-    if (p == n - 1) chunks[excl[p] + flags[p]] = (uint32_t)n;
-}
+};
+struct ChunkStore {
+    uint32_t *chunks;
+    __device__ void operator()(uint64_t p, unsigned ex, unsigned flag) const {
+        if (flag) chunks[ex] = (uint32_t)p;
+    }
+};
+struct ChunkDone {
+    uint64_t n;
+    uint32_t *chunks;
+    uint32_t *d_nc;
+    __device__ void operator()(unsigned total) const {
+        chunks[total] = (uint32_t)n;
+        *d_nc = total;
+    }
+};
 
 int bits_for(unsigned long long maxval) {
     int b = 0;
@@ -514,20 +614,11 @@ static int sort_points(Temps &tmp, const double *d_raw, uint64_t n, const GridGe
 }
 
 template <class K>
-static int rle(Temps &tmp, const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *cell_lid,
-               uint32_t *cell_start, uint64_t *d_M, cudaStream_t s) {
-    rle_flags_kernel<K><<<grid_for(n), kThreads, 0, s>>>(ks, n, cellof);
-    note_launch();
-    uint32_t *d_m32;
-    SJ_TRY(tmp.alloc(&d_m32, 1));
-    SJ_TRY(scan_exclusive_u32(cellof, cellof, n, d_m32, s));
-    rle_write_kernel<K><<<grid_for(n), kThreads, 0, s>>>(ks, n, cellof, cell_lid, cell_start);
-    note_launch();
-    // d_M (u64) <- d_m32
+static int rle(const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *cell_lid, uint32_t *cell_start,
+               uint64_t *d_M, cudaStream_t s) {
     SJ_CUDA_TRY(cudaMemsetAsync(d_M, 0, sizeof(uint64_t), s));
-    SJ_CUDA_TRY(cudaMemcpyAsync(d_M, d_m32, sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
-    SJ_CUDA_TRY(cudaGetLastError());
-    return SJ_OK;
+    return scan_fused(n, RleLoad<K>{ks}, RleStore<K>{ks, cellof, cell_lid, cell_start}, s,
+                      RleDone{n, cell_start, d_M});
 }
 
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s, cudaEvent_t ev0,
@@ -613,11 +704,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     if (ix.key_bits <= 32) {
         uint32_t *ks;
         SJ_TRY(sort_points<uint32_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
-        SJ_TRY(rle<uint32_t>(tmp, ks, n, cellof, cell_lid, cell_start, d_M, s));
+        SJ_TRY(rle<uint32_t>(ks, n, cellof, cell_lid, cell_start, d_M, s));
     } else {
         uint64_t *ks;
         SJ_TRY(sort_points<uint64_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
-        SJ_TRY(rle<uint64_t>(tmp, ks, n, cellof, cell_lid, cell_start, d_M, s));
+        SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s));
     }
 
     // ---- lid -> rank lookup: dense table when prod(nc) is small, else a hash table
@@ -653,6 +744,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     FwdGeom fg{};
     fg.dim = dim;
     fg.rows = R;
+    fg.small = ncells_total <= 0xFFFFFFFFull ? 1 : 0;
     for (int d = 0; d < dim; ++d) {
         fg.nc[d] = ix.nc[d];
         fg.stride[d] = ix.stride[d];
@@ -663,8 +755,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wload, n));
     SJ_TRY(tmp.alloc(&d_tot, 1));
     SJ_CUDA_TRY(cudaMemsetAsync(d_tot, 0, sizeof(BuildTotals), s));
-    runs_kernel<false><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload, nullptr,
-                                                        nullptr, d_tot);
+    const bool wide = R >= 16;  // one warp per cell for many rows
+    if (wide)
+        runs_kernel<false, 32><<<grid_for(n * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
+                                                                     nullptr, nullptr, d_tot);
+    else
+        runs_kernel<false, 1><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload, nullptr,
+                                                               nullptr, d_tot);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin;
@@ -693,8 +790,12 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     ix.max_w = bt.max_w;
 
     SJ_TRY(dev_alloc_t(&ix.runs, E + 2, s));
-    runs_kernel<true><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr, rbegin,
-                                                       ix.runs, nullptr);
+    if (wide)
+        runs_kernel<true, 32><<<grid_for(M * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
+                                                                    rbegin, ix.runs, nullptr);
+    else
+        runs_kernel<true, 1><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
+                                                              rbegin, ix.runs, nullptr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
@@ -732,17 +833,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_CUDA_TRY(cudaGetLastError());
 
     // ---- WorkQueue chunks over D'
-    uint32_t *cflags, *cexcl, *d_nc;
-    SJ_TRY(tmp.alloc(&cflags, n));
-    SJ_TRY(tmp.alloc(&cexcl, n));
+    uint32_t *d_nc;
     SJ_TRY(tmp.alloc(&d_nc, 1));
     SJ_TRY(dev_alloc_t(&ix.chunks, n + 1, s));
-    chunk_flags_kernel<<<grid_for(n), kThreads, 0, s>>>(ix.qmap, ix.cellq, qb, n, kBigCell, cflags);
-    note_launch();
-    SJ_TRY(scan_exclusive_u32(cflags, cexcl, n, d_nc, s));
-    chunk_write_kernel<<<grid_for(n), kThreads, 0, s>>>(cflags, cexcl, n, ix.chunks);
-    note_launch();
-    SJ_CUDA_TRY(cudaGetLastError());
+    SJ_TRY(scan_fused(n, ChunkLoad{ix.qmap, ix.cellq, qb, kBigCell}, ChunkStore{ix.chunks}, s,
+                      ChunkDone{n, ix.chunks, d_nc}));
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
     debug_mark("build: tail issued");

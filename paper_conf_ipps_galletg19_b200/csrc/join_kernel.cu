@@ -303,7 +303,10 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint
                 flush_if<EMIT>(ws.buf, nbuf, 32 * SPL, a, lane);
 #pragma unroll
                 for (int s = 0; s < SPL; ++s) {
-                    const bool hit = qv && cv[s] && sqdist<DIM>(qq, cp[s]) <= a.e2;
+                    // evaluated unconditionally and masked after (invalid slots may hold stale or
+                    // uninitialised bits; FP64 arithmetic on them cannot trap)
+                    const bool close = sqdist<DIM>(qq, cp[s]) <= a.e2;
+                    const bool hit = close & qv & cv[s];
                     emit<EMIT>(hit, oq, co[s], ws.buf, nbuf, nhits, lt);
                 }
             }

@@ -3,22 +3,22 @@
 // The radix sort orders point->cell ids for the eps-grid index ("GPU Grid
 // Index", north_star "a hand-written radix sort of point-to-cell IDs") and orders
 // cells by workload for SortByWL.  Per 8-bit pass:
-//   1. tile histogram (2048 keys per CTA, shared-memory counters),
-//   2. exclusive scan of the digit-major histogram [256 x tiles] -> global starts,
-//   3. stable scatter: per-warp ranks with __match_any_sync, a block-wide
-//      prefix over warps and digits, a shared-memory reorder of the tile so the
-//      global writes of one digit run are contiguous (coalesced).
+//   1. tile histogram (2048 keys per CTA, shared-memory counters), digit-major,
+//   2. single-pass exclusive scan (decoupled look-back) of the [256 x tiles] histogram,
+//   3. stable scatter: per-warp ranks with __match_any_sync, a block-wide prefix over
+//      warps and digits, a shared-memory reorder of the tile so the global writes of one
+//      digit run are contiguous (coalesced).
 #include <cstdio>
 
+#include <algorithm>
+
+#include "scan.cuh"
 #include "sj_internal.cuh"
 
 namespace sj {
 
 namespace {
 
-constexpr int kScanThreads = 256;
-constexpr int kScanItems = 8;
-constexpr int kScanTile = kScanThreads * kScanItems;
 
 template <class T>
 __device__ __forceinline__ T warp_inclusive_scan(T x) {
@@ -52,87 +52,6 @@ __device__ __forceinline__ T block_exclusive_scan(T v, T *total) {
     return pre + x - v;
 }
 
-template <class T>
-__global__ void __launch_bounds__(kScanThreads) scan_reduce_kernel(const T *in, uint64_t n, T *partials) {
-    const uint64_t base = (uint64_t)blockIdx.x * kScanTile;
-    T s = 0;
-#pragma unroll
-    for (int it = 0; it < kScanItems; ++it) {
-        uint64_t i = base + (uint64_t)it * kScanThreads + threadIdx.x;
-        if (i < n) s += in[i];
-    }
-    T tot;
-    block_exclusive_scan<T>(s, &tot);
-    if (threadIdx.x == 0) partials[blockIdx.x] = tot;
-}
-
-template <class T>
-__global__ void __launch_bounds__(1024) scan_partials_kernel(T *partials, uint64_t nt, T *d_total) {
-    T carry = 0;
-    for (uint64_t b = 0; b < nt; b += blockDim.x) {
-        uint64_t i = b + threadIdx.x;
-        T v = i < nt ? partials[i] : T(0);
-        T tot;
-        T ex = block_exclusive_scan<T>(v, &tot);
-        if (i < nt) partials[i] = carry + ex;
-        carry += tot;
-    }
-    if (threadIdx.x == 0 && d_total) *d_total = carry;
-}
-
-template <class T>
-__global__ void __launch_bounds__(kScanThreads) scan_down_kernel(const T *in, T *out, uint64_t n, const T *partials) {
-    __shared__ T tile[kScanTile];
-    const uint64_t base = (uint64_t)blockIdx.x * kScanTile;
-    // coalesced load into shared memory, then blocked per-thread scan
-#pragma unroll
-    for (int it = 0; it < kScanItems; ++it) {
-        uint64_t i = base + (uint64_t)it * kScanThreads + threadIdx.x;
-        tile[it * kScanThreads + threadIdx.x] = i < n ? in[i] : T(0);
-    }
-    __syncthreads();
-    T v[kScanItems];
-    T s = 0;
-#pragma unroll
-    for (int j = 0; j < kScanItems; ++j) {
-        v[j] = tile[threadIdx.x * kScanItems + j];
-        s += v[j];
-    }
-    T ex = block_exclusive_scan<T>(s, nullptr) + partials[blockIdx.x];
-    // block_exclusive_scan ends with __syncthreads before its final read; tile reuse is safe
-#pragma unroll
-    for (int j = 0; j < kScanItems; ++j) {
-        tile[threadIdx.x * kScanItems + j] = ex;
-        ex += v[j];
-    }
-    __syncthreads();
-#pragma unroll
-    for (int it = 0; it < kScanItems; ++it) {
-        uint64_t i = base + (uint64_t)it * kScanThreads + threadIdx.x;
-        if (i < n) out[i] = tile[it * kScanThreads + threadIdx.x];
-    }
-}
-
-template <class T>
-int scan_exclusive(const T *in, T *out, uint64_t n, T *d_total, cudaStream_t s) {
-    if (n == 0) {
-        if (d_total) SJ_CUDA_TRY(cudaMemsetAsync(d_total, 0, sizeof(T), s));
-        return SJ_OK;
-    }
-    uint64_t nt = (n + kScanTile - 1) / kScanTile;
-    T *partials = nullptr;
-    SJ_TRY(dev_alloc_t(&partials, nt, s));
-    scan_reduce_kernel<T><<<(unsigned)nt, kScanThreads, 0, s>>>(in, n, partials);
-    note_launch();
-    scan_partials_kernel<T><<<1, 1024, 0, s>>>(partials, nt, d_total);
-    note_launch();
-    scan_down_kernel<T><<<(unsigned)nt, kScanThreads, 0, s>>>(in, out, n, partials);
-    note_launch();
-    SJ_CUDA_TRY(cudaGetLastError());
-    dev_free(partials, s);
-    return SJ_OK;
-}
-
 // ------------------------------------------------------------------ radix sort
 
 constexpr int kRadixThreads = 256;
@@ -141,6 +60,7 @@ constexpr int kRadixItems = 8;  // per lane
 constexpr int kRadixTile = kRadixThreads * kRadixItems;
 constexpr int kRadixBins = 256;
 
+// Per-tile digit counts, digit-major: hist[d * ntiles + tile].
 template <class K>
 __global__ void __launch_bounds__(kRadixThreads) radix_hist_kernel(const K *keys, uint64_t n, int shift,
                                                                    uint32_t *hist, uint32_t ntiles) {
@@ -157,6 +77,9 @@ __global__ void __launch_bounds__(kRadixThreads) radix_hist_kernel(const K *keys
     hist[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
 }
 
+// Stable scatter of one tile: per-warp ranks with __match_any_sync, a block-wide prefix
+// over warps and digits, global starts from the scanned digit-major histogram, and a
+// shared-memory reorder so each digit's run is written contiguously.
 template <class K>
 __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *keys_in, const uint32_t *vals_in,
                                                                       K *keys_out, uint32_t *vals_out, uint64_t n,
@@ -193,7 +116,6 @@ __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *k
         }
     }
     __syncthreads();
-    // per-warp stable ranks in (it, lane) order
 #pragma unroll
     for (int it = 0; it < kRadixItems; ++it) {
         const uint32_t d = dig[it];
@@ -206,18 +128,16 @@ __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *k
         __syncwarp();
     }
     __syncthreads();
-    // prefix over warps for digit d = threadIdx.x, then over digits
     {
         const uint32_t d = threadIdx.x;
-        uint32_t s = 0;
+        uint32_t tc = 0;
 #pragma unroll
         for (int w = 0; w < kRadixWarps; ++w) {
-            uint32_t t = cnt[w][d];
-            cnt[w][d] = s;
-            s += t;
+            const uint32_t t = cnt[w][d];
+            cnt[w][d] = tc;
+            tc += t;
         }
-        uint32_t ex = block_exclusive_scan<uint32_t>(s, nullptr);
-        dstart[d] = ex;
+        dstart[d] = block_exclusive_scan<uint32_t>(tc, nullptr);
         gstart[d] = hist_scanned[(uint64_t)d * ntiles + blockIdx.x];
     }
     __syncthreads();
@@ -225,7 +145,7 @@ __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *k
     for (int it = 0; it < kRadixItems; ++it) {
         const uint32_t d = dig[it];
         if (d < kRadixBins) {
-            uint32_t lpos = dstart[d] + cnt[warp][d] + rank[it];
+            const uint32_t lpos = dstart[d] + cnt[warp][d] + rank[it];
             skeys[lpos] = key[it];
             svals[lpos] = val[it];
         }
@@ -234,9 +154,9 @@ __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *k
     const uint64_t rem = n - base;
     const uint32_t tcount = rem < (uint64_t)kRadixTile ? (uint32_t)rem : (uint32_t)kRadixTile;
     for (uint32_t i = threadIdx.x; i < tcount; i += kRadixThreads) {
-        K k = skeys[i];
-        uint32_t d = (uint32_t)(k >> shift) & 0xFFu;
-        uint64_t dest = (uint64_t)gstart[d] + (i - dstart[d]);
+        const K k = skeys[i];
+        const uint32_t d = (uint32_t)(k >> shift) & 0xFFu;
+        const uint64_t dest = (uint64_t)gstart[d] + (i - dstart[d]);
         keys_out[dest] = k;
         vals_out[dest] = svals[i];
     }
@@ -260,7 +180,7 @@ int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_
     for (int shift = 0; shift < bits; shift += 8) {
         radix_hist_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, n, shift, hist, ntiles);
         note_launch();
-        SJ_TRY(scan_exclusive<uint32_t>(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s));
+        SJ_TRY(scan_exclusive_u32(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s));
         radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, va, kb, vb, n, shift, hist, ntiles);
         note_launch();
         SJ_CUDA_TRY(cudaGetLastError());
@@ -273,13 +193,29 @@ int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_
     return SJ_OK;
 }
 
+struct LoadArr {
+    const uint32_t *in;
+    __device__ unsigned operator()(uint64_t i) const { return in[i]; }
+};
+struct StoreArr {
+    uint32_t *out;
+    __device__ void operator()(uint64_t i, unsigned ex, unsigned) const { out[i] = ex; }
+};
+struct DoneTotal {
+    uint32_t *total;
+    __device__ void operator()(unsigned t) const {
+        if (total) *total = t;
+    }
+};
+
 }  // namespace
 
 int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s) {
-    return scan_exclusive<uint32_t>(in, out, n, d_total, s);
-}
-int scan_exclusive_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s) {
-    return scan_exclusive<uint64_t>(in, out, n, d_total, s);
+    if (n == 0) {
+        if (d_total) SJ_CUDA_TRY(cudaMemsetAsync(d_total, 0, sizeof(uint32_t), s));
+        return SJ_OK;
+    }
+    return scan_fused(n, LoadArr{in}, StoreArr{out}, s, DoneTotal{d_total});
 }
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
                    uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s) {

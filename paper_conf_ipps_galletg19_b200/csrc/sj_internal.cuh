@@ -69,8 +69,6 @@ void pinned_release(void *p);
 // --------------------------------------------------------------------------- primitives
 // Exclusive scan of u32 (out may alias in).  total (device, optional) receives the sum.
 int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s);
-// u64 variant
-int scan_exclusive_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s);
 
 // Stable LSD radix sort of (key, value) pairs on the low `bits` bits of the keys.
 // Hand-written: per 8-bit pass a tile histogram, a digit-major scan and a stable
