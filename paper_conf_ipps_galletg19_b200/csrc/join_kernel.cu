@@ -52,6 +52,7 @@ struct WarpSmem {
     alignas(16) double qry[32 * PAD];   // the chunk's query points
     unsigned tile_orig[32];             // input ids of the staged candidates
     unsigned qorig[32];                 // input ids of the chunk's queries
+    unsigned qrr[32];                   // the queries' positions in their (common) cell
     alignas(16) uint2 buf[EMIT ? kBufHits : 2];
 };
 
@@ -187,10 +188,12 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, ui
         double qp[DIM];
         unsigned oq = 0;
         uint4 ci = make_uint4(0, 0, 0, 0);
+        uint2 nxt = make_uint2(0, 0);
         if (valid) {
             ci = __ldg(a.cellq + qcell);
             load_point<DIM>(a.pts + (size_t)qlid * PAD, qp);
             oq = __ldg(a.orig + qlid);
+            if (ci.w) nxt = __ldg(a.runs + ci.z);  // prefetched next run
         } else {
 #pragma unroll
             for (int d = 0; d < DIM; ++d) qp[d] = 0.0;
@@ -203,7 +206,6 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, ui
         const unsigned total = valid ? rem + home_len : 0u;
         unsigned seg_base = 0, seg_len = 0;
         bool home = false;
-        uint2 nxt = (valid && rem) ? __ldg(a.runs + e) : make_uint2(0, 0);  // prefetched next run
         unsigned i = t;  // lane t takes candidates t, t+k, ... of the list (Fig. 4)
         const unsigned my_iters = (total + (unsigned)K - 1u - t) / (unsigned)K;
         const unsigned iters = __reduce_max_sync(kFull, my_iters);  // warp-uniform trip count
@@ -245,27 +247,108 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, ui
     }
 }
 
-// Tiled path: all nq queries of the chunk lie in one cell (hb, m, runs rb.., S candidates).
-// The forward runs are staged 32 candidates at a time in shared memory (points + input
-// ids); lane t of a group holds tile slots t, t+k, ... in registers and evaluates them
-// against one query per round of 32/k queries, so each staged candidate serves the whole
-// chunk.
-template <int DIM, int K, bool EMIT>
-__device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint4 ci,
-                                            WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
-                                            unsigned long long &ncalcs, int lane, unsigned lt) {
+// Evaluate one staged tile against every query of the chunk.  HOME: the tile holds home-cell
+// positions tb.. and a (query, slot) pair is inside the query's circulant half scan iff
+// (p - rr - 1) mod m < home_count(m, rr) (reading c8).
+template <int DIM, int K, bool EMIT, bool HOME>
+__device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
+                                            WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits, int lane,
+                                            unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     constexpr int SPL = 32 / K;  // tile slots per lane
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
+    if constexpr (SPL <= 4 && DIM <= 3) {  // tile slots in registers (register budget)
+        double cp[SPL][DIM];
+        unsigned co[SPL];
+        bool cv[SPL];
+#pragma unroll
+        for (int s = 0; s < SPL; ++s) {
+            const unsigned j = t + (unsigned)(K * s);
+            cv[s] = j < nt;
+            load_smem_point<DIM>(ws.tile + (j & 31) * PAD, cp[s]);
+            co[s] = ws.tile_orig[j & 31];
+        }
+        for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+            const unsigned qi = (r0 + grp) & 31;
+            const bool qv = r0 + grp < nq;
+            double qq[DIM];
+            load_smem_point<DIM>(ws.qry + qi * PAD, qq);
+            const unsigned oq = ws.qorig[qi];
+            unsigned rr = 0, hl = 0;
+            if (HOME) {
+                rr = ws.qrr[qi];
+                hl = home_count(m, rr);
+            }
+            flush_if<EMIT>(ws.buf, nbuf, 32 * SPL, a, lane);
+#pragma unroll
+            for (int s = 0; s < SPL; ++s) {
+                // evaluated unconditionally and masked after (invalid slots may hold stale or
+                // uninitialised bits; FP64 arithmetic on them cannot trap)
+                const bool close = sqdist<DIM>(qq, cp[s]) <= a.e2;
+                bool ok = qv & cv[s];
+                if (HOME) {
+                    int d = (int)(tb + t + (unsigned)(K * s)) - (int)rr - 1;
+                    if (d < 0) d += (int)m;
+                    ok = ok & ((unsigned)d < hl);
+                }
+                emit<EMIT>(close & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
+            }
+        }
+    } else {
+        for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+            const unsigned qi = (r0 + grp) & 31;
+            const bool qv = r0 + grp < nq;
+            double qq[DIM];
+            load_smem_point<DIM>(ws.qry + qi * PAD, qq);
+            const unsigned oq = ws.qorig[qi];
+            unsigned rr = 0, hl = 0;
+            if (HOME) {
+                rr = ws.qrr[qi];
+                hl = home_count(m, rr);
+            }
+            for (int s = 0; s < SPL; ++s) {
+                const unsigned j = t + (unsigned)(K * s);
+                bool ok = qv && j < nt;
+                if (HOME && ok) {
+                    int d = (int)(tb + j) - (int)rr - 1;
+                    if (d < 0) d += (int)m;
+                    ok = (unsigned)d < hl;
+                }
+                bool hit = false;
+                if (ok) {
+                    double cp[DIM];
+                    load_smem_point<DIM>(ws.tile + j * PAD, cp);
+                    hit = sqdist<DIM>(qq, cp) <= a.e2;
+                }
+                flush_if<EMIT>(ws.buf, nbuf, 32, a, lane);
+                emit<EMIT>(hit, oq, ws.tile_orig[j & 31], ws.buf, nbuf, nhits, lt);
+            }
+        }
+    }
+}
+
+// Tiled path: all nq queries of the chunk lie in one cell (hb, m, runs rb.., S forward
+// candidates).  The forward runs, then the home cell, are staged 32 candidates at a time in
+// shared memory (points + input ids); lane t of a group holds tile slots t, t+k, ... and
+// evaluates them against one query per round of 32/k queries, so each staged candidate
+// serves the whole chunk.
+template <int DIM, int K, bool EMIT>
+__device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint4 ci,
+                                            WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
+                                            unsigned long long &ncalcs, int lane, unsigned lt) {
+    constexpr int PAD = PointPad<DIM>::value;
     const unsigned hb = ci.x, m = ci.y, S = ci.w;
     __syncwarp();
     if ((unsigned)lane < nq) {
         copy_point_to_smem<DIM>(a.pts + (size_t)qm_lane.x * PAD, ws.qry + lane * PAD);
         ws.qorig[lane] = __ldg(a.orig + qm_lane.x);
+        const unsigned rr = qm_lane.x - hb;
+        ws.qrr[lane] = rr;
+        ncalcs += (unsigned long long)S + home_count(m, rr);  // this query's distance calculations
     }
-    // ---- forward runs, staged
+    // ---- forward runs (LID-UNICOMP)
     unsigned e = ci.z, seg_base = 0, seg_len = 0, i = (unsigned)lane;
     for (unsigned tb = 0; tb < S; tb += 32) {
         __syncwarp();
@@ -282,83 +365,18 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint
             i += 32;
         }
         __syncwarp();
-        const unsigned nt = min(32u, S - tb);
-        if constexpr (SPL <= 4 && DIM <= 3) {  // tile slots in registers (register budget)
-            double cp[SPL][DIM];
-            unsigned co[SPL];
-            bool cv[SPL];
-#pragma unroll
-            for (int s = 0; s < SPL; ++s) {
-                const unsigned j = t + (unsigned)(K * s);
-                cv[s] = j < nt;
-                load_smem_point<DIM>(ws.tile + (j & 31) * PAD, cp[s]);
-                co[s] = ws.tile_orig[j & 31];
-            }
-            for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
-                const unsigned qi = r0 + grp;
-                const bool qv = qi < nq;
-                double qq[DIM];
-                load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
-                const unsigned oq = ws.qorig[qi & 31];
-                flush_if<EMIT>(ws.buf, nbuf, 32 * SPL, a, lane);
-#pragma unroll
-                for (int s = 0; s < SPL; ++s) {
-                    // evaluated unconditionally and masked after (invalid slots may hold stale or
-                    // uninitialised bits; FP64 arithmetic on them cannot trap)
-                    const bool close = sqdist<DIM>(qq, cp[s]) <= a.e2;
-                    const bool hit = close & qv & cv[s];
-                    emit<EMIT>(hit, oq, co[s], ws.buf, nbuf, nhits, lt);
-                }
-            }
-        } else {
-            for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
-                const unsigned qi = r0 + grp;
-                const bool qv = qi < nq;
-                double qq[DIM];
-                load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
-                const unsigned oq = ws.qorig[qi & 31];
-                for (int s = 0; s < SPL; ++s) {
-                    const unsigned j = t + (unsigned)(K * s);
-                    bool hit = false;
-                    if (qv && j < nt) {
-                        double cp[DIM];
-                        load_smem_point<DIM>(ws.tile + j * PAD, cp);
-                        hit = sqdist<DIM>(qq, cp) <= a.e2;
-                    }
-                    flush_if<EMIT>(ws.buf, nbuf, 32, a, lane);
-                    emit<EMIT>(hit, oq, ws.tile_orig[j & 31], ws.buf, nbuf, nhits, lt);
-                }
-            }
-        }
+        tile_rounds<DIM, K, EMIT, false>(a, nq, min(32u, S - tb), tb, m, ws, nbuf, nhits, lane, lt);
     }
-    // ---- home cell, per round, straight from global memory (the cell is small and hot in L1)
-    for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
-        const unsigned qi = r0 + grp;
-        const bool qv = qi < nq;
-        const unsigned qlid = __shfl_sync(kFull, qm_lane.x, qi & 31);
-        const unsigned rr = qlid - hb;
-        const unsigned home_len = qv ? home_count(m, rr) : 0u;
-        double qq[DIM];
-        load_smem_point<DIM>(ws.qry + (qi & 31) * PAD, qq);
-        const unsigned oq = ws.qorig[qi & 31];
-        if (qv && t == 0) ncalcs += (unsigned long long)S + home_len;
-        const unsigned iters = __reduce_max_sync(kFull, (home_len + (unsigned)K - 1u - t) / (unsigned)K);
-        for (unsigned it = 0; it < iters; ++it) {
-            const unsigned ii = t + (unsigned)K * it;
-            bool hit = false;
-            unsigned cidx = 0;
-            if (ii < home_len) {
-                unsigned j = rr + 1u + ii;
-                if (j >= m) j -= m;
-                cidx = hb + j;
-                double cp[DIM];
-                load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
-                hit = sqdist<DIM>(qq, cp) <= a.e2;
-            }
-            const unsigned oc = (EMIT && hit) ? __ldg(a.orig + cidx) : 0u;
-            flush_if<EMIT>(ws.buf, nbuf, 32, a, lane);
-            emit<EMIT>(hit, oq, oc, ws.buf, nbuf, nhits, lt);
+    // ---- home cell: balanced circulant half scan as a mask over staged home tiles
+    for (unsigned tb = 0; tb < m; tb += 32) {
+        __syncwarp();
+        if (tb + (unsigned)lane < m) {
+            const unsigned cidx = hb + tb + (unsigned)lane;
+            copy_point_to_smem<DIM>(a.pts + (size_t)cidx * PAD, ws.tile + lane * PAD);
+            ws.tile_orig[lane] = __ldg(a.orig + cidx);
         }
+        __syncwarp();
+        tile_rounds<DIM, K, EMIT, true>(a, nq, min(32u, m - tb), tb, m, ws, nbuf, nhits, lane, lt);
     }
 }
 

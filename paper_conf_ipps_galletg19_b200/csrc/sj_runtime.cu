@@ -350,6 +350,10 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
             float ms = 0;
             SJ_CUDA_TRY(cudaEventElapsedTime(&ms, s.ev_start, s.ev_stop));
             h->st.ms_join_sum += ms;
+            if (getenv("SJ_DEBUG_BATCH"))
+                fprintf(stderr, "[sj] batch chunks [%llu, %llu) pairs %llu  %.3f ms  %.1f GB/s\n",
+                        (unsigned long long)j.v0, (unsigned long long)j.v1, (unsigned long long)j.cnt, ms,
+                        j.cnt * 8.0 / (ms * 1e6));
             if (j.cnt > s.cap) {
                 // overflow (estimate too low): split the range, or grow the buffer if it is one chunk
                 h->st.retries++;
@@ -477,12 +481,17 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         // over the whole slice writes it in place (no staging, no D2D copy).  Overflow is
         // detected from the counter and falls back to the staged path.
         cudaStream_t s = h->s_main;
+        unsigned long long dv0 = 0, dv1 = V;
+        if (const char *r = getenv("SJ_DEBUG_VRANGE")) {  // diagnostics: join a sub-range only
+            sscanf(r, "%llu,%llu", &dv0, &dv1);
+            dv1 = std::min<unsigned long long>(dv1, V);
+        }
         SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
-        set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, 0ull);
+        set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, dv0);
         note_launch();
         JoinArgs a = base_args(h);
         a.head = h->d_ctr + 1;
-        a.v_end = V;
+        a.v_end = dv1;
         a.out = out;
         a.emit_ctr = h->d_ctr;
         a.out_cap = cap;
