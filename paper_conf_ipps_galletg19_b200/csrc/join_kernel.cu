@@ -38,22 +38,32 @@ namespace {
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarps = kJoinThreads / 32;
 constexpr int kBufHits = 512;  // hits buffered per warp ({orig q, orig c}, 8 B -> 4 KB)
+// A cell segment of >= 2 queries is tiled when its forward list has at least this many
+// candidates (6-D: ~1300 per cell of ~4 points), so staging pays for itself.
+constexpr unsigned kTileMinCand = 128;
 
 template <int DIM>
 struct PointPad {
     static constexpr int value = DIM == 1 ? 1 : ((DIM + 1) & ~1);
 };
 
+template <int DIM>
+struct BufCap {
+    static constexpr int value = DIM <= 3 ? kBufHits : kBufHits / 2;
+};
+
 // Per-warp shared memory: emission buffer, the chunk's queries, one candidate tile.
 template <int DIM, bool EMIT>
 struct WarpSmem {
     static constexpr int PAD = PointPad<DIM>::value;
-    alignas(16) double tile[32 * PAD];  // staged candidates (lid order)
+    alignas(16) double tile[2][32 * PAD];  // staged candidates (lid order), double-buffered
     alignas(16) double qry[32 * PAD];   // the chunk's query points
-    unsigned tile_orig[32];             // input ids of the staged candidates
+    unsigned tile_orig[2][32];             // input ids of the staged candidates
     unsigned qorig[32];                 // input ids of the chunk's queries
     unsigned qrr[32];                   // the queries' positions in their (common) cell
-    alignas(16) uint2 buf[EMIT ? kBufHits : 2];
+    // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
+    // and the smaller footprint buys occupancy)
+    alignas(16) uint2 buf[EMIT ? (DIM <= 3 ? kBufHits : kBufHits / 2) : 2];
 };
 
 template <int DIM>
@@ -93,6 +103,35 @@ __device__ __forceinline__ void copy_point_to_smem(const double *__restrict__ sr
 #pragma unroll
         for (int d = 0; d < PAD; d += 2)
             *reinterpret_cast<double2 *>(dst + d) = __ldg(reinterpret_cast<const double2 *>(src + d));
+    }
+}
+
+// Asynchronous global->shared copies (cp.async, LDGSTS): tile staging without registers.
+__device__ __forceinline__ void cp_async_16(void *smem, const void *gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_8(void *smem, const void *gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sa), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_4(void *smem, const void *gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sa), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
+}
+template <int DIM>
+__device__ __forceinline__ void cp_async_point(double *dst, const double *src) {
+    constexpr int PAD = PointPad<DIM>::value;
+    if constexpr (PAD == 1) {
+        cp_async_8(dst, src);
+    } else {
+#pragma unroll
+        for (int d = 0; d < PAD; d += 2) cp_async_16(dst + d, src + d);
     }
 }
 
@@ -153,10 +192,10 @@ __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *
     }
 }
 
-template <bool EMIT>
+template <bool EMIT, int CAP = kBufHits>
 __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane) {
     if constexpr (EMIT) {
-        if (nbuf > kBufHits - room) {
+        if (nbuf > CAP - room) {
             flush(buf, nbuf, a, lane);
             nbuf = 0;
         }
@@ -173,18 +212,20 @@ __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
 // group walk their query's list -- forward runs first (identical for queries of one cell,
 // so their loads coincide), then the home half scan -- taking candidates t, t+k, ...
 template <int DIM, int K, bool EMIT>
-__device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint2 *buf, int &nbuf,
-                                              unsigned long long &nhits, unsigned long long &ncalcs, int lane,
-                                              unsigned lt) {
+__device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint2 *buf,
+                                              int &nbuf, unsigned long long &nhits, unsigned long long &ncalcs,
+                                              int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
+    const unsigned nq = __popc(gmask);  // the chunk's queries handled here: lanes in gmask
     for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
         const unsigned qi = r0 + grp;
         const bool valid = qi < nq;
-        const unsigned qlid = __shfl_sync(kFull, qm_lane.x, qi & 31);
-        const unsigned qcell = __shfl_sync(kFull, qm_lane.y, qi & 31);
+        const int src = valid ? (int)__fns(gmask, 0, (int)qi + 1) : 0;  // lane of the qi-th query
+        const unsigned qlid = __shfl_sync(kFull, qm_lane.x, src);
+        const unsigned qcell = __shfl_sync(kFull, qm_lane.y, src);
         double qp[DIM];
         unsigned oq = 0;
         uint4 ci = make_uint4(0, 0, 0, 0);
@@ -241,7 +282,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, ui
                 i += K;
             }
             const unsigned oc = (EMIT && hit) ? __ldg(a.orig + cidx) : 0u;
-            flush_if<EMIT>(buf, nbuf, 32, a, lane);
+            flush_if<EMIT, BufCap<DIM>::value>(buf, nbuf, 32, a, lane);
             emit<EMIT>(hit, oq, oc, buf, nbuf, nhits, lt);
         }
     }
@@ -252,8 +293,10 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned nq, ui
 // (p - rr - 1) mod m < home_count(m, rr) (reading c8).
 template <int DIM, int K, bool EMIT, bool HOME>
 __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
-                                            WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits, int lane,
-                                            unsigned lt) {
+                                            WarpSmem<DIM, EMIT> &ws, int b, int &nbuf, unsigned long long &nhits,
+                                            int lane, unsigned lt) {
+    const double *tile = ws.tile[b];
+    const unsigned *tile_orig = ws.tile_orig[b];
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     constexpr int SPL = 32 / K;  // tile slots per lane
@@ -267,8 +310,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
         for (int s = 0; s < SPL; ++s) {
             const unsigned j = t + (unsigned)(K * s);
             cv[s] = j < nt;
-            load_smem_point<DIM>(ws.tile + (j & 31) * PAD, cp[s]);
-            co[s] = ws.tile_orig[j & 31];
+            load_smem_point<DIM>(tile + (j & 31) * PAD, cp[s]);
+            co[s] = tile_orig[j & 31];
         }
         for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
             const unsigned qi = (r0 + grp) & 31;
@@ -281,22 +324,25 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 rr = ws.qrr[qi];
                 hl = home_count(m, rr);
             }
-            flush_if<EMIT>(ws.buf, nbuf, 32 * SPL, a, lane);
+            flush_if<EMIT, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
+            // all SPL distances first (independent FP64 chains -> ILP), then the emissions;
+            // evaluated unconditionally and masked after (invalid slots may hold stale or
+            // uninitialised bits; FP64 arithmetic on them cannot trap)
+            bool close[SPL];
+#pragma unroll
+            for (int s = 0; s < SPL; ++s) close[s] = sqdist<DIM>(qq, cp[s]) <= a.e2;
 #pragma unroll
             for (int s = 0; s < SPL; ++s) {
-                // evaluated unconditionally and masked after (invalid slots may hold stale or
-                // uninitialised bits; FP64 arithmetic on them cannot trap)
-                const bool close = sqdist<DIM>(qq, cp[s]) <= a.e2;
                 bool ok = qv & cv[s];
                 if (HOME) {
                     int d = (int)(tb + t + (unsigned)(K * s)) - (int)rr - 1;
                     if (d < 0) d += (int)m;
                     ok = ok & ((unsigned)d < hl);
                 }
-                emit<EMIT>(close & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
+                emit<EMIT>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
             }
         }
-    } else {
+    } else {  // tile slots read from shared memory each step (higher dimensions)
         for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
             const unsigned qi = (r0 + grp) & 31;
             const bool qv = r0 + grp < nq;
@@ -308,22 +354,27 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 rr = ws.qrr[qi];
                 hl = home_count(m, rr);
             }
-            for (int s = 0; s < SPL; ++s) {
-                const unsigned j = t + (unsigned)(K * s);
-                bool ok = qv && j < nt;
-                if (HOME && ok) {
-                    int d = (int)(tb + j) - (int)rr - 1;
-                    if (d < 0) d += (int)m;
-                    ok = (unsigned)d < hl;
+            flush_if<EMIT, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
+#pragma unroll 2
+            for (int s = 0; s < SPL; s += 2) {  // two slots per step: two independent FP64 chains
+                const unsigned j0 = t + (unsigned)(K * s), j1 = j0 + (unsigned)K;
+                double c0[DIM], c1[DIM];
+                load_smem_point<DIM>(tile + (j0 & 31) * PAD, c0);
+                load_smem_point<DIM>(tile + (j1 & 31) * PAD, c1);
+                // evaluated unconditionally and masked after (see above)
+                const bool close0 = sqdist<DIM>(qq, c0) <= a.e2;
+                const bool close1 = sqdist<DIM>(qq, c1) <= a.e2;
+                bool ok0 = qv & (j0 < nt), ok1 = qv & (s + 1 < SPL) & (j1 < nt);
+                if (HOME) {
+                    int d0 = (int)(tb + j0) - (int)rr - 1, d1 = (int)(tb + j1) - (int)rr - 1;
+                    if (d0 < 0) d0 += (int)m;
+                    if (d1 < 0) d1 += (int)m;
+                    ok0 = ok0 & ((unsigned)d0 < hl);
+                    ok1 = ok1 & ((unsigned)d1 < hl);
                 }
-                bool hit = false;
-                if (ok) {
-                    double cp[DIM];
-                    load_smem_point<DIM>(ws.tile + j * PAD, cp);
-                    hit = sqdist<DIM>(qq, cp) <= a.e2;
-                }
-                flush_if<EMIT>(ws.buf, nbuf, 32, a, lane);
-                emit<EMIT>(hit, oq, ws.tile_orig[j & 31], ws.buf, nbuf, nhits, lt);
+                const bool hit0 = close0 & ok0, hit1 = close1 & ok1;
+                emit<EMIT>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt);
+                emit<EMIT>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt);
             }
         }
     }
@@ -335,23 +386,24 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
 // evaluates them against one query per round of 32/k queries, so each staged candidate
 // serves the whole chunk.
 template <int DIM, int K, bool EMIT>
-__device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint2 qm_lane, uint4 ci,
+__device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsigned nq, uint2 qm_lane, uint4 ci,
                                             WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
                                             unsigned long long &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     const unsigned hb = ci.x, m = ci.y, S = ci.w;
     __syncwarp();
-    if ((unsigned)lane < nq) {
-        copy_point_to_smem<DIM>(a.pts + (size_t)qm_lane.x * PAD, ws.qry + lane * PAD);
-        ws.qorig[lane] = __ldg(a.orig + qm_lane.x);
+    const unsigned slot = (unsigned)lane - s0;  // the segment's queries are lanes s0 .. s0+nq-1
+    if (slot < nq) {
+        copy_point_to_smem<DIM>(a.pts + (size_t)qm_lane.x * PAD, ws.qry + slot * PAD);
+        ws.qorig[slot] = __ldg(a.orig + qm_lane.x);
         const unsigned rr = qm_lane.x - hb;
-        ws.qrr[lane] = rr;
+        ws.qrr[slot] = rr;
         ncalcs += (unsigned long long)S + home_count(m, rr);  // this query's distance calculations
     }
-    // ---- forward runs (LID-UNICOMP)
+    // ---- forward runs (LID-UNICOMP): tiles staged with cp.async, double-buffered, so the
+    // next tile's global loads overlap this tile's distance calculations
     unsigned e = ci.z, seg_base = 0, seg_len = 0, i = (unsigned)lane;
-    for (unsigned tb = 0; tb < S; tb += 32) {
-        __syncwarp();
+    auto stage_fwd = [&](int b, unsigned tb) {
         if (tb + (unsigned)lane < S) {
             while (i >= seg_len) {
                 i -= seg_len;
@@ -360,23 +412,46 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned nq, uint
                 seg_len = f.y;
             }
             const unsigned cidx = seg_base + i;
-            copy_point_to_smem<DIM>(a.pts + (size_t)cidx * PAD, ws.tile + lane * PAD);
-            ws.tile_orig[lane] = __ldg(a.orig + cidx);
+            cp_async_point<DIM>(ws.tile[b] + lane * PAD, a.pts + (size_t)cidx * PAD);
+            cp_async_4(ws.tile_orig[b] + lane, a.orig + cidx);
             i += 32;
         }
+        cp_async_commit();
+    };
+    if (S) stage_fwd(0, 0);
+    int it = 0;
+    for (unsigned tb = 0; tb < S; tb += 32, ++it) {
+        const bool more = tb + 32 < S;
+        if (more) stage_fwd((it + 1) & 1, tb + 32);
+        if (more)
+            cp_async_wait<1>();
+        else
+            cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, EMIT, false>(a, nq, min(32u, S - tb), tb, m, ws, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, EMIT, false>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        __syncwarp();
     }
     // ---- home cell: balanced circulant half scan as a mask over staged home tiles
-    for (unsigned tb = 0; tb < m; tb += 32) {
-        __syncwarp();
+    auto stage_home = [&](int b, unsigned tb) {
         if (tb + (unsigned)lane < m) {
             const unsigned cidx = hb + tb + (unsigned)lane;
-            copy_point_to_smem<DIM>(a.pts + (size_t)cidx * PAD, ws.tile + lane * PAD);
-            ws.tile_orig[lane] = __ldg(a.orig + cidx);
+            cp_async_point<DIM>(ws.tile[b] + lane * PAD, a.pts + (size_t)cidx * PAD);
+            cp_async_4(ws.tile_orig[b] + lane, a.orig + cidx);
         }
+        cp_async_commit();
+    };
+    stage_home(0, 0);
+    it = 0;
+    for (unsigned tb = 0; tb < m; tb += 32, ++it) {
+        const bool more = tb + 32 < m;
+        if (more) stage_home((it + 1) & 1, tb + 32);
+        if (more)
+            cp_async_wait<1>();
+        else
+            cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, EMIT, true>(a, nq, min(32u, m - tb), tb, m, ws, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, EMIT, true>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        __syncwarp();
     }
 }
 
@@ -407,13 +482,35 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
             const unsigned nq = qe - qs;  // 1..32 D' positions
             const bool lv = (unsigned)lane < nq;
             const uint2 qm = lv ? __ldg(a.qmap + qs + lane) : make_uint2(0, 0xFFFFFFFFu);
-            const unsigned cell0 = __shfl_sync(kFull, qm.y, 0);
-            const bool same = __all_sync(kFull, !lv || qm.y == cell0);
-            const uint4 ci0 = __ldg(a.cellq + cell0);
-            if (same && ci0.y >= kBigCell && nq >= 2u * QPW)
-                tiled_chunk<DIM, K, EMIT>(a, nq, qm, ci0, ws, nbuf, nhits, ncalcs, lane, lt);
-            else
-                generic_chunk<DIM, K, EMIT>(a, nq, qm, ws.buf, nbuf, nhits, ncalcs, lane, lt);
+            // The chunk's queries form segments of one cell each (D' keeps cells contiguous).
+            // A segment whose cell has a long candidate list is evaluated tile by tile from
+            // shared memory (each staged candidate serves every query of the segment); the
+            // remaining queries go through the generic per-query path together.
+            const unsigned prev = __shfl_up_sync(kFull, qm.y, 1);
+            const bool head = lv && (lane == 0 || qm.y != prev);
+            const unsigned heads = __ballot_sync(kFull, head);
+            // every lane fetches its own cell record in parallel; heads decide for their segment
+            const uint4 ci = lv ? __ldg(a.cellq + qm.y) : make_uint4(0, 0, 0, 0);
+            const unsigned later = heads & ~(0xffffffffu >> (31 - lane));  // heads after this lane
+            const unsigned seg_end = later ? (unsigned)(__ffs(later) - 1) : nq;
+            const unsigned nseg = seg_end - (unsigned)lane;  // meaningful on head lanes
+            const bool tiled = head && ((nseg >= 2u * QPW && ci.y >= kBigCell) ||
+                                        (DIM >= 4 && nseg >= 2u && ci.w >= kTileMinCand));
+            unsigned theads = __ballot_sync(kFull, tiled);
+            const int my_head = 31 - __clz(heads & (0xffffffffu >> (31 - lane)));
+            const unsigned gmask = __ballot_sync(kFull, lv && !((theads >> (my_head & 31)) & 1u));
+            while (theads) {
+                const int s0 = __ffs(theads) - 1;
+                theads &= theads - 1;
+                uint4 cs;
+                cs.x = __shfl_sync(kFull, ci.x, s0);
+                cs.y = __shfl_sync(kFull, ci.y, s0);
+                cs.z = __shfl_sync(kFull, ci.z, s0);
+                cs.w = __shfl_sync(kFull, ci.w, s0);
+                const unsigned n0 = __shfl_sync(kFull, nseg, s0);
+                tiled_chunk<DIM, K, EMIT>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
+            }
+            if (gmask) generic_chunk<DIM, K, EMIT>(a, gmask, qm, ws.buf, nbuf, nhits, ncalcs, lane, lt);
         }
     }
     if constexpr (EMIT) {
