@@ -195,9 +195,24 @@ int handle_init_common(sj_handle *h) {
     return SJ_OK;
 }
 
+// Staged-path slots (stream + events + b_s result buffer) are recycled process-wide per
+// device: creating/destroying streams and multi-GB buffers per join costs tens of ms.
+std::mutex g_slot_mu;
+std::vector<std::pair<int, Slot>> g_slot_cache;  // (device, idle slot)
+
 int slot_init(sj_handle *h, int i) {
     Slot &s = h->slots[i];
     if (s.stream) return SJ_OK;
+    {
+        std::lock_guard<std::mutex> lk(g_slot_mu);
+        for (size_t k = 0; k < g_slot_cache.size(); ++k)
+            if (g_slot_cache[k].first == h->device) {
+                s = g_slot_cache[k].second;
+                g_slot_cache.erase(g_slot_cache.begin() + (long)k);
+                s.busy = false;
+                return SJ_OK;
+            }
+    }
     SJ_CUDA_TRY(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
     SJ_CUDA_TRY(cudaEventCreate(&s.ev_start));
     SJ_CUDA_TRY(cudaEventCreate(&s.ev_stop));
@@ -221,6 +236,14 @@ void slots_release(sj_handle *h) {
         Slot &s = h->slots[i];
         if (!s.stream) continue;
         cudaStreamSynchronize(s.stream);
+        {
+            std::lock_guard<std::mutex> lk(g_slot_mu);
+            if (g_slot_cache.size() < 2 * kMaxStreams) {
+                g_slot_cache.emplace_back(h->device, s);
+                s = Slot();
+                continue;
+            }
+        }
         dev_free(s.buf, s.stream);
         dev_free(s.d_ctr, s.stream);
         cudaStreamSynchronize(s.stream);
