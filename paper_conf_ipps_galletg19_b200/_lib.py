@@ -7,7 +7,7 @@ import re
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _ROOT = os.path.dirname(_HERE)
-lib_path = os.path.join(_HERE, "libsj.so")
+lib_path = os.environ.get("SJ_LIB_PATH") or os.path.join(_HERE, "libsj.so")  # override: experiments only
 HEADER = os.path.join(_ROOT, "include", "sj.h")
 
 SJ_OK, SJ_MORE, SJ_EINVAL, SJ_ENOMEM, SJ_ECUDA, SJ_EGRID, SJ_ESTATE = 0, 1, -1, -2, -3, -4, -5

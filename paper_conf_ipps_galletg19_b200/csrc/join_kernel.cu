@@ -212,9 +212,9 @@ __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
 // group walk their query's list -- forward runs first (identical for queries of one cell,
 // so their loads coincide), then the home half scan -- taking candidates t, t+k, ...
 template <int DIM, int K, bool EMIT>
-__device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint2 *buf,
-                                              int &nbuf, unsigned long long &nhits, unsigned long long &ncalcs,
-                                              int lane, unsigned lt) {
+__device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
+                                              uint2 *buf, int &nbuf, unsigned long long &nhits,
+                                              unsigned long long &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     const int grp = lane / K;
@@ -225,13 +225,17 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         const bool valid = qi < nq;
         const int src = valid ? (int)__fns(gmask, 0, (int)qi + 1) : 0;  // lane of the qi-th query
         const unsigned qlid = __shfl_sync(kFull, qm_lane.x, src);
-        const unsigned qcell = __shfl_sync(kFull, qm_lane.y, src);
+        // the cell record was fetched per lane at chunk start: shuffle, do not reload
+        uint4 ci;
+        ci.x = __shfl_sync(kFull, ci_lane.x, src);
+        ci.y = __shfl_sync(kFull, ci_lane.y, src);
+        ci.z = __shfl_sync(kFull, ci_lane.z, src);
+        ci.w = __shfl_sync(kFull, ci_lane.w, src);
         double qp[DIM];
         unsigned oq = 0;
-        uint4 ci = make_uint4(0, 0, 0, 0);
         uint2 nxt = make_uint2(0, 0);
+        if (!valid) ci = make_uint4(0, 0, 0, 0);
         if (valid) {
-            ci = __ldg(a.cellq + qcell);
             load_point<DIM>(a.pts + (size_t)qlid * PAD, qp);
             oq = __ldg(a.orig + qlid);
             if (ci.w) nxt = __ldg(a.runs + ci.z);  // prefetched next run
@@ -254,7 +258,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         unsigned gi = t;
         for (unsigned it = 0; it < iters; ++it, gi += K) {
             bool hit = false;
-            unsigned cidx = 0;
+            unsigned cidx = 0, oc = 0;
             if (gi < total) {
                 while (i >= seg_len) {  // step to the run holding candidate gi
                     i -= seg_len;
@@ -278,10 +282,10 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                 }
                 double cp[DIM];
                 load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
+                if (EMIT) oc = __ldg(a.orig + cidx);  // issued with the point, not after the test
                 hit = sqdist<DIM>(qp, cp) <= a.e2;
                 i += K;
             }
-            const unsigned oc = (EMIT && hit) ? __ldg(a.orig + cidx) : 0u;
             flush_if<EMIT, BufCap<DIM>::value>(buf, nbuf, 32, a, lane);
             emit<EMIT>(hit, oq, oc, buf, nbuf, nhits, lt);
         }
@@ -510,7 +514,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
                 const unsigned n0 = __shfl_sync(kFull, nseg, s0);
                 tiled_chunk<DIM, K, EMIT>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
             }
-            if (gmask) generic_chunk<DIM, K, EMIT>(a, gmask, qm, ws.buf, nbuf, nhits, ncalcs, lane, lt);
+            if (gmask) generic_chunk<DIM, K, EMIT>(a, gmask, qm, ci, ws.buf, nbuf, nhits, ncalcs, lane, lt);
         }
     }
     if constexpr (EMIT) {
