@@ -57,43 +57,57 @@ __global__ void bbox_init_kernel(BBox *bb) {
     if (t == 0) bb->nonfinite = 0;
 }
 
-// a2: exact per-dimension min/max (order-independent) + non-finite check (a1 validation)
+// a2: exact per-dimension min/max (order-independent) + non-finite check (a1 validation).
+// The coordinates are read as a flat array of double2; the total thread count T is chosen
+// with 2T % dim == 0, so every thread always sees the same two dimensions.
 __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint64_t n, int dim, BBox *bb) {
-    unsigned long long mn[SJ_MAX_DIM], mx[SJ_MAX_DIM];
-#pragma unroll
-    for (int d = 0; d < SJ_MAX_DIM; ++d) {
-        mn[d] = ~0ull;
-        mx[d] = 0ull;
-    }
+    const uint64_t total = n * (uint64_t)dim;  // doubles
+    const uint64_t T = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int d0 = (int)((2 * t) % dim), d1 = (int)((2 * t + 1) % dim);
+    unsigned long long mn0 = ~0ull, mx0 = 0, mn1 = ~0ull, mx1 = 0;
     unsigned bad = 0;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-#pragma unroll
-        for (int d = 0; d < SJ_MAX_DIM; ++d) {
-            if (d < dim) {
-                double x = raw[i * dim + d];
-                if (!isfinite(x)) bad = 1;
-                unsigned long long k = ordered_key(x);
-                mn[d] = min(mn[d], k);
-                mx[d] = max(mx[d], k);
-            }
-        }
+    const double2 *r2 = reinterpret_cast<const double2 *>(raw);
+    const uint64_t pairs = total / 2;
+#pragma unroll 4
+    for (uint64_t e = t; e < pairs; e += T) {
+        const double2 v = __ldg(r2 + e);
+        bad |= !isfinite(v.x) | !isfinite(v.y);
+        const unsigned long long k0 = ordered_key(v.x), k1 = ordered_key(v.y);
+        mn0 = min(mn0, k0);
+        mx0 = max(mx0, k0);
+        mn1 = min(mn1, k1);
+        mx1 = max(mx1, k1);
     }
-#pragma unroll
-    for (int d = 0; d < SJ_MAX_DIM; ++d) {
-        if (d < dim) {
-            unsigned long long a = mn[d], b = mx[d];
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                a = min(a, __shfl_xor_sync(0xffffffffu, a, o));
-                b = max(b, __shfl_xor_sync(0xffffffffu, b, o));
-            }
-            if ((threadIdx.x & 31) == 0) {
-                atomicMin(&bb->mn[d], a);
-                atomicMax(&bb->mx[d], b);
-            }
-        }
+    if ((total & 1) && t == 0) {  // odd element count: the last double (dimension dim-1)
+        const double x = raw[total - 1];
+        bad |= !isfinite(x);
+        const unsigned long long k = ordered_key(x);
+        atomicMin(&bb->mn[dim - 1], k);
+        atomicMax(&bb->mx[dim - 1], k);
     }
-    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(&bb->nonfinite, 1u);
+    // block reduction per dimension in shared memory, then ONE atomic per dimension and block
+    __shared__ unsigned long long s_mn[SJ_MAX_DIM], s_mx[SJ_MAX_DIM];
+    __shared__ unsigned s_bad;
+    if (threadIdx.x < SJ_MAX_DIM) {
+        s_mn[threadIdx.x] = ~0ull;
+        s_mx[threadIdx.x] = 0;
+    }
+    if (threadIdx.x == 0) s_bad = 0;
+    __syncthreads();
+    if (t < pairs) {
+        atomicMin(&s_mn[d0], mn0);
+        atomicMax(&s_mx[d0], mx0);
+        atomicMin(&s_mn[d1], mn1);
+        atomicMax(&s_mx[d1], mx1);
+    }
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) s_bad = 1;
+    __syncthreads();
+    if (threadIdx.x < (unsigned)dim) {
+        atomicMin(&bb->mn[threadIdx.x], s_mn[threadIdx.x]);
+        atomicMax(&bb->mx[threadIdx.x], s_mx[threadIdx.x]);
+    }
+    if (threadIdx.x == 0 && s_bad) atomicOr(&bb->nonfinite, 1u);
 }
 
 struct GridGeom {
@@ -647,7 +661,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     bbox_init_kernel<<<1, 32, 0, s>>>(d_bb);
     note_launch();
     {
-        unsigned blocks = (unsigned)std::min<uint64_t>(grid_for(n), 148ull * 8);
+        // 2 * threads must be a multiple of dim (see bbox_kernel): blocks a multiple of dim
+        const uint64_t pairs = n * (uint64_t)dim / 2;
+        unsigned blocks = (unsigned)std::min<uint64_t>((pairs + kThreads * 8 - 1) / (kThreads * 8), 148ull * 8);
+        blocks = std::max(1u, blocks);
+        blocks = ((blocks + dim - 1) / dim) * dim;
         bbox_kernel<<<blocks, kThreads, 0, s>>>(d_raw, n, dim, d_bb);
         note_launch();
     }

@@ -112,13 +112,22 @@ __global__ void __launch_bounds__(kThreads) scan_kernel(uint64_t n, Load load, S
     }
     __syncthreads();
     ex += s_prefix;
+    // per-item exclusive prefixes back to shared memory (blocked), then the stores run in the
+    // same striped (coalesced) order as the loads
+    __shared__ unsigned exs[kTile];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
-        const uint64_t i = base + (uint64_t)threadIdx.x * kItems + j;
-        if (i < n) store(i, ex, v[j]);
+        exs[threadIdx.x * kItems + j] = ex;
         ex += v[j];
     }
     if (base + kTile >= n && threadIdx.x == kThreads - 1) done(ex);  // ex = grand total here
+    __syncthreads();
+#pragma unroll
+    for (int it = 0; it < kItems; ++it) {
+        const int k = it * kThreads + threadIdx.x;
+        const uint64_t i = base + (uint64_t)k;
+        if (i < n) store(i, exs[k], vals[k]);
+    }
 }
 
 }  // namespace scan_detail

@@ -629,7 +629,8 @@ sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
     const double *d_raw = points;
     double *d_copy = nullptr;
     int rc = SJ_OK;
-    if (!is_device_ptr(points, h->device)) {
+    // host input, or a device pointer that is not 16-byte aligned (the build reads double2)
+    if (!is_device_ptr(points, h->device) || (reinterpret_cast<uintptr_t>(points) & 15u)) {
         // a1: upload (the library owns its copy; caller keeps `points`)
         rc = dev_alloc_t(&d_copy, n * (uint64_t)dim, s);
         if (rc == SJ_OK) {

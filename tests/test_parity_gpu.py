@@ -163,6 +163,21 @@ def test_host_and_device_pointers(device_out, points_on_device):
     np.testing.assert_array_equal(canon(got), want)
 
 
+def test_misaligned_device_input_and_odd_sizes():
+    # a device pointer 8 bytes into an allocation (not 16-byte aligned) and an odd number of
+    # coordinates (3-D, odd n) exercise the bbox reader's edge cases
+    for dim, n in ((3, 10_001), (1, 9_999), (5, 3_333)):
+        pts = workloads.uniform(n, dim, 900 + dim)
+        eps = workloads.eps_for_k("uniform", n, dim, 10)
+        big = torch.empty(n * dim + 1, dtype=torch.float64, device=DEV)
+        big[1:] = torch.from_numpy(pts.ravel()).to(DEV)
+        view = big[1:].view(n, dim)
+        assert view.data_ptr() % 16 == 8
+        with sj.Handle(view, eps, k=8) as h:
+            got = sj.self_join_pairs(h, DEV).cpu().numpy().view(np.uint32)
+        np.testing.assert_array_equal(canon(got), oracle.grid_pairs(pts, eps))
+
+
 def test_count_only_matches_oracle():
     cfg = workloads.get_config("c3k64").scaled(100_000)
     pts = cfg.points()
