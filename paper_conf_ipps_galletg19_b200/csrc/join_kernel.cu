@@ -476,7 +476,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         // WorkQueue dequeue: one atomic per warp, result shuffled
         unsigned long long vb = 0;
         if (lane == 0) vb = atomicAdd(a.head, (unsigned long long)a.grab);
-        vb = __shfl_sync(kFull, vb, 0);
+        vb = __shfl_sync(kFull, vb, 0) + a.v_begin;
         if (vb >= a.v_end) break;
         const unsigned long long vend = min(vb + a.grab, a.v_end);
         for (unsigned long long v = vb; v < vend; ++v) {

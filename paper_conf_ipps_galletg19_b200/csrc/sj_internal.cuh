@@ -128,8 +128,9 @@ struct JoinArgs {
     const uint32_t *chunks;       // WorkQueue chunks of D'
     uint32_t n_chunks;
     double e2;
-    unsigned long long *head;     // dequeue counter (virtual chunk index of this slice)
-    unsigned long long v_end;     // end of this batch (virtual chunk index)
+    unsigned long long *head;     // WorkQueue counter (chunks taken), zeroed before the launch
+    unsigned long long v_begin;   // batch = virtual chunk range [v_begin, v_end) of this slice
+    unsigned long long v_end;
     uint32_t grab;                // chunks per dequeue
     uint32_t rank, world;         // queue slice: virtual chunk v -> chunk v*world + rank
     uint32_t *out;                // interleaved pairs, or nullptr (count-only)

@@ -291,10 +291,9 @@ int join_blocks(const sj_handle *h, bool emit, int *blocks) {
 int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms) {
     cudaStream_t s = h->s_main;
     SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
-    set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, v0);
-    note_launch();
     JoinArgs a = base_args(h);
-    a.head = h->d_ctr + 1;
+    a.head = h->d_ctr + 1;  // zeroed above
+    a.v_begin = v0;
     a.v_end = v1;
     a.out = nullptr;
     a.emit_ctr = h->d_ctr;
@@ -318,10 +317,9 @@ int launch_job(sj_handle *h, Job &j, int slot_idx) {
     Slot &s = h->slots[slot_idx];
     SJ_TRY(slot_buffer(h, s, h->batch_pairs));
     SJ_CUDA_TRY(cudaMemsetAsync(s.d_ctr, 0, 4 * sizeof(unsigned long long), s.stream));
-    set_u64_kernel<<<1, 1, 0, s.stream>>>(s.d_ctr + 1, j.v0);
-    note_launch();
     JoinArgs a = base_args(h);
-    a.head = s.d_ctr + 1;
+    a.head = s.d_ctr + 1;  // zeroed above
+    a.v_begin = j.v0;
     a.v_end = j.v1;
     a.out = s.buf;
     a.emit_ctr = s.d_ctr;
@@ -510,10 +508,9 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
             dv1 = std::min<unsigned long long>(dv1, V);
         }
         SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
-        set_u64_kernel<<<1, 1, 0, s>>>(h->d_ctr + 1, dv0);
-        note_launch();
         JoinArgs a = base_args(h);
-        a.head = h->d_ctr + 1;
+        a.head = h->d_ctr + 1;  // zeroed above
+        a.v_begin = dv0;
         a.v_end = dv1;
         a.out = out;
         a.emit_ctr = h->d_ctr;
@@ -741,6 +738,7 @@ int sj_set_option(sj_handle *h, int opt, int64_t v) {
         case SJ_OPT_FAST_PATH:
             h->fast_path = v ? 1 : 0;
             return SJ_OK;
+
     }
     set_error("sj_set_option: invalid option %d or value %lld", opt, (long long)v);
     return SJ_EINVAL;
