@@ -61,6 +61,21 @@ enum sj_option {
                                   stage per batch (the paper's scheme)                             */
 };
 
+/* Cell access patterns (sj_create_ex).  The paper's variants, Table II:
+ *   SJ_PATTERN_LID_UNICOMP -- neighbour cells with a higher linear id, mirrored emission
+ *                             (Alg. 3); the default and the hot path;
+ *   SJ_PATTERN_GCG         -- GPUCALCGLOBAL's full 3^n neighbourhood, one pair per
+ *                             distance calculation (Alg. 1): twice the calculations;
+ *   SJ_PATTERN_UNICOMP     -- the odd-coordinate pattern of [18] (Alg. 2), mirrored.
+ * All three return the same pair set. */
+enum sj_pattern { SJ_PATTERN_LID_UNICOMP = 0, SJ_PATTERN_GCG = 1, SJ_PATTERN_UNICOMP = 2 };
+
+/* Order of the query queue D' (sj_create_ex):
+ *   SJ_ORDER_WORKLOAD -- SortByWL: cells by non-increasing workload; default;
+ *   SJ_ORDER_CELL     -- cells in linear-id order (no sort by workload);
+ *   SJ_ORDER_INPUT    -- the input order of the points (the unsorted D of GPUCALCGLOBAL). */
+enum sj_order { SJ_ORDER_WORKLOAD = 0, SJ_ORDER_CELL = 1, SJ_ORDER_INPUT = 2 };
+
 /* Statistics of the handle (sj_get_stats).  Times are CUDA-event milliseconds. */
 typedef struct sj_stats {
     uint64_t n;               /* points                                              */
@@ -90,6 +105,8 @@ typedef struct sj_stats {
     uint32_t nc[8];           /* cells per dimension                                 */
     uint64_t n_chunks;        /* WorkQueue chunks of D'                              */
     uint32_t tiled_min;       /* smallest cell (points) that gets shared-memory tiles */
+    uint32_t pattern;         /* enum sj_pattern of the index                        */
+    uint32_t order;           /* enum sj_order of the index                          */
     uint32_t reserved;
 } sj_stats;
 
@@ -104,6 +121,11 @@ typedef struct sj_stats {
  * Returns NULL on error (see sj_last_error): NaN/Inf coordinate or bad argument
  * (SJ_EINVAL), grid overflow (SJ_EGRID), allocation (SJ_ENOMEM), CUDA (SJ_ECUDA). */
 sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps);
+
+/* sj_create with an explicit cell pattern (enum sj_pattern) and queue order (enum sj_order),
+ * for the paper's ablations (Tables III-V).  sj_create(...) == sj_create_ex(..., 0, 0).
+ * SJ_EINVAL for an unknown pattern or order. */
+sj_handle *sj_create_ex(const double *points, uint64_t n, int dim, double eps, int pattern, int order);
 
 /* Run (or continue) the self-join.
  *   out_pairs : caller-owned uint32[2*cap], interleaved (i, j) of 0-based input ids,

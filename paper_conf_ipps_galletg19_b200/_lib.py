@@ -11,6 +11,10 @@ lib_path = os.environ.get("SJ_LIB_PATH") or os.path.join(_HERE, "libsj.so")  # o
 HEADER = os.path.join(_ROOT, "include", "sj.h")
 
 SJ_OK, SJ_MORE, SJ_EINVAL, SJ_ENOMEM, SJ_ECUDA, SJ_EGRID, SJ_ESTATE = 0, 1, -1, -2, -3, -4, -5
+SJ_PATTERN_LID_UNICOMP, SJ_PATTERN_GCG, SJ_PATTERN_UNICOMP = 0, 1, 2
+SJ_ORDER_WORKLOAD, SJ_ORDER_CELL, SJ_ORDER_INPUT = 0, 1, 2
+PATTERNS = {"lid_unicomp": SJ_PATTERN_LID_UNICOMP, "gcg": SJ_PATTERN_GCG, "unicomp": SJ_PATTERN_UNICOMP}
+ORDERS = {"workload": SJ_ORDER_WORKLOAD, "cell": SJ_ORDER_CELL, "input": SJ_ORDER_INPUT}
 (SJ_OPT_K, SJ_OPT_BATCH_PAIRS, SJ_OPT_STREAMS, SJ_OPT_SAMPLE_PPM, SJ_OPT_GRAB, SJ_OPT_COUNT_CALCS,
  SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH) = range(1, 9)
 _NAMES = {0: "SJ_OK", 1: "SJ_MORE", -1: "SJ_EINVAL", -2: "SJ_ENOMEM", -3: "SJ_ECUDA", -4: "SJ_EGRID",
@@ -33,7 +37,8 @@ class SJStats(ctypes.Structure):
         ("ms_build", ctypes.c_double), ("ms_estimate", ctypes.c_double), ("ms_join", ctypes.c_double),
         ("ms_join_sum", ctypes.c_double), ("ms_transfer", ctypes.c_double), ("ms_total", ctypes.c_double),
         ("fast_path", ctypes.c_uint32), ("nc", ctypes.c_uint32 * 8), ("n_chunks", ctypes.c_uint64),
-        ("tiled_min", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
+        ("tiled_min", ctypes.c_uint32), ("pattern", ctypes.c_uint32), ("order", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32),
     ]
 
     def as_dict(self) -> dict:
@@ -53,6 +58,7 @@ _sig = {
     "sj_kernel_launches": (_u64, []),
     "sj_last_error": (ctypes.c_char_p, []),
     "sj_create": (_vp, [_vp, _u64, _int, _dbl]),
+    "sj_create_ex": (_vp, [_vp, _u64, _int, _dbl, _int, _int]),
     "sj_self_join": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
     "sj_destroy": (None, [_vp]),
     "sj_set_option": (_int, [_vp, _int, _i64]),
@@ -115,8 +121,7 @@ def sj_last_error() -> str:
     return (_lib.sj_last_error() or b"").decode()
 
 
-def sj_create(points, n: int | None = None, dim: int | None = None, eps: float | None = None) -> int:
-    """sj_create(points, eps) or sj_create(ptr, n, dim, eps).  Returns the raw handle (int)."""
+def _shape(points, n, dim, eps):
     if eps is None:  # (points, eps) form
         eps = n
         shape = tuple(points.shape)
@@ -129,7 +134,22 @@ def sj_create(points, n: int | None = None, dim: int | None = None, eps: float |
             raise ValueError("points must be contiguous")
         if hasattr(points, "flags") and not points.flags["C_CONTIGUOUS"]:
             raise ValueError("points must be C-contiguous")
+    return n, dim, eps
+
+
+def sj_create(points, n: int | None = None, dim: int | None = None, eps: float | None = None) -> int:
+    """sj_create(points, eps) or sj_create(ptr, n, dim, eps).  Returns the raw handle (int)."""
+    n, dim, eps = _shape(points, n, dim, eps)
     h = _lib.sj_create(_ptr(points), int(n), int(dim), float(eps))
+    if not h:
+        raise SJError(SJ_EINVAL, sj_last_error())
+    return h
+
+
+def sj_create_ex(points, n=None, dim=None, eps=None, pattern: int = 0, order: int = 0) -> int:
+    """sj_create_ex(points, eps, pattern=, order=) or (ptr, n, dim, eps, pattern, order)."""
+    n, dim, eps = _shape(points, n, dim, eps)
+    h = _lib.sj_create_ex(_ptr(points), int(n), int(dim), float(eps), int(pattern), int(order))
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
     return h
@@ -209,8 +229,16 @@ def sj_measure_atomics():
 class Handle:
     """Owning wrapper of an sj_handle*."""
 
-    def __init__(self, points=None, eps: float | None = None, *, raw: int | None = None, **options):
-        self.h = raw if raw is not None else sj_create(points, eps)
+    def __init__(self, points=None, eps: float | None = None, *, raw: int | None = None, pattern=None, order=None,
+                 **options):
+        if raw is not None:
+            self.h = raw
+        elif pattern is None and order is None:
+            self.h = sj_create(points, eps)
+        else:
+            pat = PATTERNS.get(pattern, pattern) if pattern is not None else 0
+            odr = ORDERS.get(order, order) if order is not None else 0
+            self.h = sj_create_ex(points, eps, pattern=pat, order=odr)
         for k, v in options.items():
             self.set_option(k, v)
 

@@ -19,7 +19,7 @@
 
 namespace sj {
 
-__constant__ uint64_t c_fwd_off[SJ_MAX_FWD];  // forward rows (forward_rows()), packed int8
+__constant__ uint64_t c_fwd_off[SJ_MAX_FWD];  // rows of the cell pattern (pattern_rows()), packed
 
 namespace {
 
@@ -225,8 +225,9 @@ struct FwdGeom {
     unsigned long long nc[SJ_MAX_DIM];
     unsigned long long stride[SJ_MAX_DIM];
     int dim;
-    int rows;   // forward rows (see forward_rows())
+    int rows;   // rows of the cell pattern (see pattern_rows())
     int small;  // prod(nc) < 2^32: 32-bit lid arithmetic
+    int full;   // GCG: the rows cover the whole 3^n neighbourhood incl. the home cell
 };
 
 struct BuildTotals {
@@ -278,13 +279,24 @@ __device__ __forceinline__ void decode_lid(unsigned long long lid, const FwdGeom
     }
 }
 
-// One forward row of cell c (see forward_rows()): the non-empty cells among the row's <= 3
-// cells have consecutive ranks, so their points are one run [b, b+len) of the lid-ordered
-// storage.  The <= 3 lookups are issued together.
+// One row of cell c (see pattern_rows()): the non-empty cells among the row's <= 3 cells
+// (consecutive along the last dimension) have consecutive ranks, so their points are one
+// run [b, b+len) of the lid-ordered storage.  The <= 3 lookups are issued together.
+// Row encoding: byte d = o'_d (d < dim-1 <= 7); byte 7 = lo+1 | (hi+1) << 2 | (pdim+1) << 4,
+// the last-dimension offsets lo..hi and (UNICOMP) the dimension whose coordinate must be odd.
 __device__ __forceinline__ bool eval_row(int j, const long long (&c)[SJ_MAX_DIM], const FwdGeom &g, const Lookup &L,
                                          const uint32_t *cell_start, uint32_t &b, uint32_t &len) {
-    const unsigned long long off = c_fwd_off[j];  // bytes 0..n-2: o'; byte 7: 1 = home row
+    const unsigned long long off = c_fwd_off[j];
     const int last = g.dim - 1;
+    const unsigned meta = (unsigned)(off >> 56);
+    const int pdim = (int)(meta >> 4) - 1;
+    if (pdim >= 0) {  // UNICOMP rule (Alg. 2): only cells with an odd coordinate in pdim
+        long long cp = 0;
+#pragma unroll
+        for (int d = 0; d < SJ_MAX_DIM; ++d)
+            if (d == pdim) cp = c[d];
+        if ((cp & 1) == 0) return false;
+    }
     bool in = true;
     long long base = 0;
 #pragma unroll
@@ -297,9 +309,9 @@ __device__ __forceinline__ bool eval_row(int j, const long long (&c)[SJ_MAX_DIM]
         }
     }
     if (!in) return false;
-    const bool home_row = (off >> 56) != 0;
-    const long long x0 = c[last] + (home_row ? 1 : -1);
-    const int nx = home_row ? 1 : 3;
+    const int lo = (int)(meta & 3u) - 1, hi = (int)((meta >> 2) & 3u) - 1;
+    const long long x0 = c[last] + lo;
+    const int nx = hi - lo + 1;
     uint32_t nb[3];
 #pragma unroll
     for (int u = 0; u < 3; ++u) {
@@ -372,9 +384,14 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
             }
             if (valid && sub == 0) {
                 rcnt[r] = cnt;
-                w = (uint32_t)(m / 2 + summ);  // ceil((m-1)/2) = floor(m/2) for m >= 1
+                if (g.full) {  // GCG: every candidate of the 3^n neighbourhood but the query itself
+                    w = (uint32_t)(summ - 1);
+                    calcs = (unsigned long long)m * (summ - 1);
+                } else {       // half patterns: ceil((m-1)/2) = floor(m/2) home + the forward runs
+                    w = (uint32_t)(m / 2 + summ);
+                    calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
+                }
                 wload[r] = w;
-                calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
             }
         }
     }
@@ -423,26 +440,28 @@ __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t
                                                                   const uint32_t *cell_start, const uint32_t *rbegin,
                                                                   const uint32_t *wload,
                                                                   const unsigned long long *cell_lid, uint64_t M,
-                                                                  uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
+                                                                  int full, uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
                                                                   uint64_t *lid_q) {
     uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= M) return;
     uint32_t r = qorder[i];
     uint32_t m = cell_start[r + 1] - cell_start[r];
-    // {begin in the lid-ordered storage, m, first run, sum of the runs' lengths (= W - floor(m/2))}
-    cellq[i] = make_uint4(cell_start[r], m, rbegin[r], wload[r] - m / 2);
+    // {begin in the lid-ordered storage, m, first run, S = sum of the runs' lengths}
+    // (half patterns: W = floor(m/2) + S; GCG: W = S - 1, the query itself excluded)
+    cellq[i] = make_uint4(cell_start[r], m, rbegin[r], full ? wload[r] + 1 : wload[r] - m / 2);
     r2q[r] = (uint32_t)i;
     qbr[r] = qb[i];
     lid_q[i] = cell_lid[r];
 }
 
 // Points gathered into lid (spatial) order, padded AoS, plus D' = the queue as an index
-// array: qmap[D' position] = {lid-storage position, queue-order cell}.
+// array: qmap[D' position] = {lid-storage position, queue-order cell}.  With
+// input_order the queue is the input order itself (the ablation's unsorted D).
 __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, uint64_t n, int dim, int pad,
                                                            const uint32_t *idx_sorted, const uint32_t *cellof,
                                                            const uint32_t *cell_start, const uint32_t *qbr,
                                                            const uint32_t *r2q, double *pts, uint32_t *orig,
-                                                           uint2 *qmap) {
+                                                           uint2 *qmap, int input_order) {
     uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
     const uint32_t r = cellof[p];
@@ -453,7 +472,8 @@ __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, ui
         for (int d = 0; d < pad; ++d) pts[p * pad + d] = d < dim ? raw[(uint64_t)src * dim + d] : 0.0;
     }
     orig[p] = src;
-    qmap[(uint64_t)qbr[r] + (p - cell_start[r])] = make_uint2((uint32_t)p, r2q[r]);
+    const uint64_t dest = input_order ? (uint64_t)src : (uint64_t)qbr[r] + (p - cell_start[r]);
+    qmap[dest] = make_uint2((uint32_t)p, r2q[r]);
 }
 
 // WorkQueue chunks: D' is cut into chunks of at most kChunk positions so that
@@ -557,35 +577,71 @@ void free_index(Index &ix, cudaStream_t s) {
     ix.cell_lid = nullptr;
 }
 
-// Forward rows of LID-UNICOMP (see runs_kernel): the home row (o' = 0, last-dim offset +1
-// only) followed by every o' in {-1,0,1}^(dim-1) whose first non-zero component is +1 with
-// last-dim offsets -1..+1.  Packed: byte d = o'_d (d < dim-1 <= 7), byte 7 = 1 for the home row.
-static int forward_rows(int dim, std::vector<uint64_t> &rows) {
+// Rows of a cell pattern (see eval_row for the encoding):
+//  * LID-UNICOMP (Alg. 3): the home row's +1 cell, then every o' in {-1,0,1}^(dim-1)
+//    whose first non-zero component is +1, with last-dimension offsets -1..+1 -- exactly the
+//    neighbours with a higher row-major linear id (reading c7);
+//  * GCG (GPUCALCGLOBAL, Alg. 1): every o' with offsets -1..+1 -- the whole 3^n
+//    neighbourhood including the home cell;
+//  * UNICOMP ([18] as given in Alg. 2): a cell whose coordinate in dimension j is
+//    odd compares to the neighbours that differ in dimension j, are free in the dimensions
+//    before j and equal in the dimensions after it; one single-cell row per such offset.
+static int pattern_rows(int dim, int pattern, std::vector<uint64_t> &rows) {
     rows.clear();
-    auto pack = [](const int8_t *o, int nd, bool home) {
+    auto pack = [dim](const int8_t *o, int lo, int hi, int pdim) {
         uint64_t p = 0;
-        for (int d = 0; d < nd; ++d) p |= (uint64_t)(uint8_t)o[d] << (8 * d);
-        if (home) p |= 1ull << 56;
-        return p;
+        for (int d = 0; d < dim - 1; ++d) p |= (uint64_t)(uint8_t)o[d] << (8 * d);
+        const unsigned meta = (unsigned)(lo + 1) | ((unsigned)(hi + 1) << 2) | ((unsigned)(pdim + 1) << 4);
+        return p | ((uint64_t)meta << 56);
     };
-    int8_t zero[SJ_MAX_DIM] = {0};
-    rows.push_back(pack(zero, dim - 1, true));
     int total = 1;
     for (int d = 0; d < dim - 1; ++d) total *= 3;
+    auto prefix = [dim](int t, int8_t *o) {
+        for (int d = dim - 2; d >= 0; --d) {
+            o[d] = (int8_t)(t % 3 - 1);
+            t /= 3;
+        }
+    };
+    if (pattern == SJ_PATTERN_UNICOMP) {
+        int all = total * 3;
+        for (int t = 0; t < all; ++t) {
+            int8_t o[SJ_MAX_DIM] = {0};
+            int v = t;
+            for (int d = dim - 1; d >= 0; --d) {
+                o[d] = (int8_t)(v % 3 - 1);
+                v /= 3;
+            }
+            int j = -1;
+            for (int d = dim - 1; d >= 0; --d)
+                if (o[d] != 0) {
+                    j = d;
+                    break;
+                }
+            if (j < 0) continue;  // the home cell: circulant half scan in the kernel
+            rows.push_back(pack(o, o[dim - 1], o[dim - 1], j));
+        }
+        return (int)rows.size();
+    }
+    if (pattern == SJ_PATTERN_GCG) {
+        for (int t = 0; t < total; ++t) {
+            int8_t o[SJ_MAX_DIM] = {0};
+            prefix(t, o);
+            rows.push_back(pack(o, -1, 1, -1));
+        }
+        return (int)rows.size();
+    }
+    int8_t zero[SJ_MAX_DIM] = {0};
+    rows.push_back(pack(zero, 1, 1, -1));
     for (int t = 0; t < total; ++t) {
         int8_t o[SJ_MAX_DIM] = {0};
-        int v = t;
-        for (int d = dim - 2; d >= 0; --d) {
-            o[d] = (int8_t)(v % 3 - 1);
-            v /= 3;
-        }
+        prefix(t, o);
         int first = 0;
         for (int d = 0; d < dim - 1; ++d)
             if (o[d] != 0) {
                 first = o[d];
                 break;
             }
-        if (first == 1) rows.push_back(pack(o, dim - 1, false));
+        if (first == 1) rows.push_back(pack(o, -1, 1, -1));
     }
     return (int)rows.size();
 }
@@ -757,12 +813,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
 
     // ---- a6 + a7: forward runs, workload, D_alg
     std::vector<uint64_t> rows;
-    const int R = forward_rows(dim, rows);
+    const int R = pattern_rows(dim, ix.pattern, rows);
     SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, rows.data(), R * sizeof(uint64_t), 0, cudaMemcpyHostToDevice, s));
     FwdGeom fg{};
     fg.dim = dim;
     fg.rows = R;
     fg.small = ncells_total <= 0xFFFFFFFFull ? 1 : 0;
+    fg.full = ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
     for (int d = 0; d < dim; ++d) {
         fg.nc[d] = ix.nc[d];
         fg.stride[d] = ix.stride[d];
@@ -825,7 +882,12 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wv2, M));
     wl_keys_kernel<<<grid_for(M), kThreads, 0, s>>>(wload, M, ix.max_w, wk, wv);
     note_launch();
-    SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(ix.max_w), &qorder_keys, &qorder, s));
+    if (ix.order == SJ_ORDER_WORKLOAD) {
+        SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(ix.max_w), &qorder_keys, &qorder, s));
+    } else {  // ablation orders: cells stay in lid order (no SortByWL)
+        qorder_keys = wk;
+        qorder = wv;
+    }
     uint32_t *mq, *qb;
     SJ_TRY(tmp.alloc(&mq, M));
     SJ_TRY(tmp.alloc(&qb, M));
@@ -843,10 +905,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&r2q, M));
     SJ_TRY(tmp.alloc(&qbr, M));
     cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, rbegin, wload, cell_lid, M,
-                                                           ix.cellq, r2q, qbr, ix.cell_lid);
+                                                           fg.full, ix.cellq, r2q, qbr, ix.cell_lid);
     note_launch();
     permute_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, dim, ix.pad, idx_sorted, cellof, cell_start, qbr, r2q,
-                                                    ix.pts, ix.orig, ix.qmap);
+                                                    ix.pts, ix.orig, ix.qmap, ix.order == SJ_ORDER_INPUT ? 1 : 0);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
@@ -854,7 +916,9 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     uint32_t *d_nc;
     SJ_TRY(tmp.alloc(&d_nc, 1));
     SJ_TRY(dev_alloc_t(&ix.chunks, n + 1, s));
-    SJ_TRY(scan_fused(n, ChunkLoad{ix.qmap, ix.cellq, qb, kBigCell}, ChunkStore{ix.chunks}, s,
+    // in input order a cell's points are scattered: no chunk may claim a cell
+    const uint32_t big_min = ix.order == SJ_ORDER_INPUT ? 0xFFFFFFFFu : kBigCell;
+    SJ_TRY(scan_fused(n, ChunkLoad{ix.qmap, ix.cellq, qb, big_min}, ChunkStore{ix.chunks}, s,
                       ChunkDone{n, ix.chunks, d_nc}));
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));

@@ -148,29 +148,38 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
     return s;
 }
 
-// Flush a warp's staged hits: ONE atomicAdd reserves 2*nbuf output slots, then the lanes
-// write both mirrored pairs of each hit with one 16-B streaming store (coalesced).
+// Flush a warp's staged hits: ONE atomicAdd reserves the output slots, then the lanes write
+// coalesced streaming stores: both mirrored pairs of a hit as one 16-B store {q, c, c, q}
+// (half patterns), or the single pair {q, c} (GCG, which meets every pair twice).
+template <bool GCG>
 __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane) {
     __syncwarp();
+    constexpr unsigned long long kPer = GCG ? 1ull : 2ull;  // pairs per buffered hit
     unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(a.emit_ctr, 2ull * (unsigned long long)nbuf);
+    if (lane == 0) base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)nbuf);
     base = __shfl_sync(kFull, base, 0);
-    uint4 *out4 = reinterpret_cast<uint4 *>(a.out) + (base >> 1);  // base is even
-    if (base + 2ull * (unsigned long long)nbuf <= a.out_cap) {
+    uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
+    if constexpr (GCG) {
+        const bool fits = base + (unsigned long long)nbuf <= a.out_cap;
+        for (int k = lane; k < nbuf; k += 32)
+            if (fits || base + (unsigned long long)k < a.out_cap) __stcs(out2 + base + k, buf[k]);
+    } else {
+        uint4 *out4 = reinterpret_cast<uint4 *>(a.out) + (base >> 1);  // base is even
+        if (base + 2ull * (unsigned long long)nbuf <= a.out_cap) {
 #pragma unroll 4
-        for (int k = lane; k < nbuf; k += 32) {
-            const uint2 v = buf[k];  // {orig q, orig c}
-            __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));  // (q,c) and (c,q)
-        }
-    } else {  // overflow: keep what fits, the counter still reports the total
-        uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
-        for (int k = lane; k < nbuf; k += 32) {
-            const unsigned long long slot = base + 2ull * (unsigned long long)k;
-            const uint2 v = buf[k];
-            if (slot + 2 <= a.out_cap)
-                __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));
-            else if (slot < a.out_cap)
-                __stcs(out2 + slot, make_uint2(v.x, v.y));
+            for (int k = lane; k < nbuf; k += 32) {
+                const uint2 v = buf[k];  // {orig q, orig c}
+                __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));  // (q,c) and (c,q)
+            }
+        } else {  // overflow: keep what fits, the counter still reports the total
+            for (int k = lane; k < nbuf; k += 32) {
+                const unsigned long long slot = base + 2ull * (unsigned long long)k;
+                const uint2 v = buf[k];
+                if (slot + 2 <= a.out_cap)
+                    __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));
+                else if (slot < a.out_cap)
+                    __stcs(out2 + slot, make_uint2(v.x, v.y));
+            }
         }
     }
     __syncwarp();
@@ -180,7 +189,7 @@ __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs
 // ranked with __ballot_sync/__popc into the warp's shared buffer.  Before each round the
 // caller makes room for the round's maximum number of hits (flush_if) instead of checking
 // after every step.
-template <bool EMIT>
+template <bool EMIT, bool GCG>
 __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *buf, int &nbuf,
                                      unsigned long long &nhits, unsigned lt) {
     if constexpr (EMIT) {
@@ -188,15 +197,15 @@ __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *
         if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, oc);
         nbuf += __popc(hm);
     } else {
-        nhits += hit ? 2ull : 0ull;
+        nhits += hit ? (GCG ? 1ull : 2ull) : 0ull;
     }
 }
 
-template <bool EMIT, int CAP = kBufHits>
+template <bool EMIT, bool GCG, int CAP = kBufHits>
 __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane) {
     if constexpr (EMIT) {
         if (nbuf > CAP - room) {
-            flush(buf, nbuf, a, lane);
+            flush<GCG>(buf, nbuf, a, lane);
             nbuf = 0;
         }
     }
@@ -211,7 +220,7 @@ __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
 // Generic path: rounds of 32/k queries (possibly from different cells); the k lanes of a
 // group walk their query's list -- forward runs first (identical for queries of one cell,
 // so their loads coincide), then the home half scan -- taking candidates t, t+k, ...
-template <int DIM, int K, bool EMIT>
+template <int DIM, int K, bool EMIT, bool GCG>
 __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
                                               uint2 *buf, int &nbuf, unsigned long long &nhits,
                                               unsigned long long &ncalcs, int lane, unsigned lt) {
@@ -247,7 +256,8 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         unsigned e = ci.z;
         unsigned rem = ci.w;  // forward candidates not yet entered
         const unsigned rr = qlid - hb;
-        const unsigned home_len = valid ? home_count(m, rr) : 0u;
+        // GCG: the home cell is part of the runs (the full neighbourhood) -- no half scan
+        const unsigned home_len = (valid && !GCG) ? home_count(m, rr) : 0u;
         const unsigned total = valid ? rem + home_len : 0u;
         unsigned seg_base = 0, seg_len = 0;
         bool home = false;
@@ -255,6 +265,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         const unsigned my_iters = (total + (unsigned)K - 1u - t) / (unsigned)K;
         const unsigned iters = __reduce_max_sync(kFull, my_iters);  // warp-uniform trip count
         ncalcs += my_iters;
+        if (GCG && valid && t == 0 && total) ncalcs -= 1;  // the query itself is skipped
         unsigned gi = t;
         for (unsigned it = 0; it < iters; ++it, gi += K) {
             bool hit = false;
@@ -284,10 +295,11 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                 load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
                 if (EMIT) oc = __ldg(a.orig + cidx);  // issued with the point, not after the test
                 hit = sqdist<DIM>(qp, cp) <= a.e2;
+                if (GCG) hit = hit && cidx != qlid;  // GCG scans its own cell: skip (q, q)
                 i += K;
             }
-            flush_if<EMIT, BufCap<DIM>::value>(buf, nbuf, 32, a, lane);
-            emit<EMIT>(hit, oq, oc, buf, nbuf, nhits, lt);
+            flush_if<EMIT, GCG, BufCap<DIM>::value>(buf, nbuf, 32, a, lane);
+            emit<EMIT, GCG>(hit, oq, oc, buf, nbuf, nhits, lt);
         }
     }
 }
@@ -295,7 +307,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
 // Evaluate one staged tile against every query of the chunk.  HOME: the tile holds home-cell
 // positions tb.. and a (query, slot) pair is inside the query's circulant half scan iff
 // (p - rr - 1) mod m < home_count(m, rr) (reading c8).
-template <int DIM, int K, bool EMIT, bool HOME>
+template <int DIM, int K, bool EMIT, bool GCG, bool HOME>
 __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
                                             WarpSmem<DIM, EMIT> &ws, int b, int &nbuf, unsigned long long &nhits,
                                             int lane, unsigned lt) {
@@ -328,7 +340,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 rr = ws.qrr[qi];
                 hl = home_count(m, rr);
             }
-            flush_if<EMIT, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
+            flush_if<EMIT, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
             // all SPL distances first (independent FP64 chains -> ILP), then the emissions;
             // evaluated unconditionally and masked after (invalid slots may hold stale or
             // uninitialised bits; FP64 arithmetic on them cannot trap)
@@ -338,12 +350,13 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
 #pragma unroll
             for (int s = 0; s < SPL; ++s) {
                 bool ok = qv & cv[s];
+                if (GCG) ok = ok & (co[s] != oq);  // GCG: skip (q, q)
                 if (HOME) {
                     int d = (int)(tb + t + (unsigned)(K * s)) - (int)rr - 1;
                     if (d < 0) d += (int)m;
                     ok = ok & ((unsigned)d < hl);
                 }
-                emit<EMIT>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
+                emit<EMIT, GCG>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
             }
         }
     } else {  // tile slots read from shared memory each step (higher dimensions)
@@ -358,7 +371,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 rr = ws.qrr[qi];
                 hl = home_count(m, rr);
             }
-            flush_if<EMIT, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
+            flush_if<EMIT, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
 #pragma unroll 2
             for (int s = 0; s < SPL; s += 2) {  // two slots per step: two independent FP64 chains
                 const unsigned j0 = t + (unsigned)(K * s), j1 = j0 + (unsigned)K;
@@ -369,6 +382,10 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 const bool close0 = sqdist<DIM>(qq, c0) <= a.e2;
                 const bool close1 = sqdist<DIM>(qq, c1) <= a.e2;
                 bool ok0 = qv & (j0 < nt), ok1 = qv & (s + 1 < SPL) & (j1 < nt);
+                if (GCG) {  // skip (q, q)
+                    ok0 = ok0 & (tile_orig[j0 & 31] != oq);
+                    ok1 = ok1 & (tile_orig[j1 & 31] != oq);
+                }
                 if (HOME) {
                     int d0 = (int)(tb + j0) - (int)rr - 1, d1 = (int)(tb + j1) - (int)rr - 1;
                     if (d0 < 0) d0 += (int)m;
@@ -377,8 +394,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     ok1 = ok1 & ((unsigned)d1 < hl);
                 }
                 const bool hit0 = close0 & ok0, hit1 = close1 & ok1;
-                emit<EMIT>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt);
-                emit<EMIT>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt);
+                emit<EMIT, GCG>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt);
+                emit<EMIT, GCG>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt);
             }
         }
     }
@@ -389,7 +406,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
 // shared memory (points + input ids); lane t of a group holds tile slots t, t+k, ... and
 // evaluates them against one query per round of 32/k queries, so each staged candidate
 // serves the whole chunk.
-template <int DIM, int K, bool EMIT>
+template <int DIM, int K, bool EMIT, bool GCG>
 __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsigned nq, uint2 qm_lane, uint4 ci,
                                             WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
                                             unsigned long long &ncalcs, int lane, unsigned lt) {
@@ -402,7 +419,8 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         ws.qorig[slot] = __ldg(a.orig + qm_lane.x);
         const unsigned rr = qm_lane.x - hb;
         ws.qrr[slot] = rr;
-        ncalcs += (unsigned long long)S + home_count(m, rr);  // this query's distance calculations
+        // this query's distance calculations
+        ncalcs += GCG ? (unsigned long long)S - 1 : (unsigned long long)S + home_count(m, rr);
     }
     // ---- forward runs (LID-UNICOMP): tiles staged with cp.async, double-buffered, so the
     // next tile's global loads overlap this tile's distance calculations
@@ -432,7 +450,7 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, EMIT, false>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, EMIT, GCG, false>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
         __syncwarp();
     }
     // ---- home cell: balanced circulant half scan as a mask over staged home tiles
@@ -444,6 +462,7 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         }
         cp_async_commit();
     };
+    if (GCG) return;  // GCG: the home cell was one of the runs
     stage_home(0, 0);
     it = 0;
     for (unsigned tb = 0; tb < m; tb += 32, ++it) {
@@ -454,12 +473,12 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, EMIT, true>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, EMIT, GCG, true>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
         __syncwarp();
     }
 }
 
-template <int DIM, int K, bool EMIT>
+template <int DIM, int K, bool EMIT, bool GCG>
 __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     static_assert(32 % K == 0, "k must divide 32");
     constexpr int QPW = 32 / K;
@@ -512,13 +531,13 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
                 cs.z = __shfl_sync(kFull, ci.z, s0);
                 cs.w = __shfl_sync(kFull, ci.w, s0);
                 const unsigned n0 = __shfl_sync(kFull, nseg, s0);
-                tiled_chunk<DIM, K, EMIT>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
+                tiled_chunk<DIM, K, EMIT, GCG>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
             }
-            if (gmask) generic_chunk<DIM, K, EMIT>(a, gmask, qm, ci, ws.buf, nbuf, nhits, ncalcs, lane, lt);
+            if (gmask) generic_chunk<DIM, K, EMIT, GCG>(a, gmask, qm, ci, ws.buf, nbuf, nhits, ncalcs, lane, lt);
         }
     }
     if constexpr (EMIT) {
-        if (nbuf > 0) flush(ws.buf, nbuf, a, lane);
+        if (nbuf > 0) flush<GCG>(ws.buf, nbuf, a, lane);
     } else {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) nhits += __shfl_xor_sync(kFull, nhits, o);
@@ -538,46 +557,53 @@ struct KernelInfo {
     size_t smem = 0;
 };
 
-template <int DIM, int K, bool EMIT>
+template <int DIM, int K, bool EMIT, bool GCG>
 KernelInfo info() {
     KernelInfo ki;
-    ki.f = join_kernel<DIM, K, EMIT>;
+    ki.f = join_kernel<DIM, K, EMIT, GCG>;
     ki.smem = sizeof(WarpSmem<DIM, EMIT>) * kWarps;
     return ki;
 }
 
-template <int DIM, bool EMIT>
+// The LID-UNICOMP / UNICOMP kernels exist for every k; the GCG ablation kernels for the
+// k the paper evaluates (1 and 8) and 32.
+template <int DIM, bool EMIT, bool GCG>
 KernelInfo pick_k(int k) {
     switch (k) {
-        case 1: return info<DIM, 1, EMIT>();
-        case 2: return info<DIM, 2, EMIT>();
-        case 4: return info<DIM, 4, EMIT>();
-        case 8: return info<DIM, 8, EMIT>();
-        case 16: return info<DIM, 16, EMIT>();
-        case 32: return info<DIM, 32, EMIT>();
+        case 1: return info<DIM, 1, EMIT, GCG>();
+        case 8: return info<DIM, 8, EMIT, GCG>();
+        case 32: return info<DIM, 32, EMIT, GCG>();
+    }
+    if constexpr (!GCG) {
+        switch (k) {
+            case 2: return info<DIM, 2, EMIT, false>();
+            case 4: return info<DIM, 4, EMIT, false>();
+            case 16: return info<DIM, 16, EMIT, false>();
+        }
     }
     return KernelInfo();
 }
 
-template <bool EMIT>
+template <bool EMIT, bool GCG>
 KernelInfo pick(int dim, int k) {
     switch (dim) {
-        case 1: return pick_k<1, EMIT>(k);
-        case 2: return pick_k<2, EMIT>(k);
-        case 3: return pick_k<3, EMIT>(k);
-        case 4: return pick_k<4, EMIT>(k);
-        case 5: return pick_k<5, EMIT>(k);
-        case 6: return pick_k<6, EMIT>(k);
-        case 7: return pick_k<7, EMIT>(k);
-        case 8: return pick_k<8, EMIT>(k);
+        case 1: return pick_k<1, EMIT, GCG>(k);
+        case 2: return pick_k<2, EMIT, GCG>(k);
+        case 3: return pick_k<3, EMIT, GCG>(k);
+        case 4: return pick_k<4, EMIT, GCG>(k);
+        case 5: return pick_k<5, EMIT, GCG>(k);
+        case 6: return pick_k<6, EMIT, GCG>(k);
+        case 7: return pick_k<7, EMIT, GCG>(k);
+        case 8: return pick_k<8, EMIT, GCG>(k);
     }
     return KernelInfo();
 }
 
-int prepare(int dim, int k, bool emit, KernelInfo *out) {
-    KernelInfo ki = emit ? pick<true>(dim, k) : pick<false>(dim, k);
+int prepare(int dim, int k, bool emit, bool gcg, KernelInfo *out) {
+    KernelInfo ki = gcg ? (emit ? pick<true, true>(dim, k) : pick<false, true>(dim, k))
+                        : (emit ? pick<true, false>(dim, k) : pick<false, false>(dim, k));
     if (!ki.f) {
-        set_error("join: unsupported dim=%d k=%d", dim, k);
+        set_error("join: unsupported dim=%d k=%d%s", dim, k, gcg ? " for the GCG pattern (k in {1, 8, 32})" : "");
         return SJ_EINVAL;
     }
     SJ_CUDA_TRY(cudaFuncSetAttribute(ki.f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ki.smem));
@@ -587,16 +613,16 @@ int prepare(int dim, int k, bool emit, KernelInfo *out) {
 
 }  // namespace
 
-int join_occupancy(int dim, int k, bool emit, int *blocks_per_sm) {
+int join_occupancy(int dim, int k, bool emit, bool gcg, int *blocks_per_sm) {
     KernelInfo ki;
-    SJ_TRY(prepare(dim, k, emit, &ki));
+    SJ_TRY(prepare(dim, k, emit, gcg, &ki));
     SJ_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, ki.f, kJoinThreads, ki.smem));
     return SJ_OK;
 }
 
 int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaStream_t s) {
     KernelInfo ki;
-    SJ_TRY(prepare(dim, k, emit, &ki));
+    SJ_TRY(prepare(dim, k, emit, a.gcg != 0, &ki));
     ki.f<<<blocks, kJoinThreads, ki.smem, s>>>(a);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());

@@ -12,7 +12,7 @@
 #include "../../include/sj.h"
 
 #define SJ_MAX_DIM 8
-#define SJ_MAX_FWD 3280  // (3^8 - 1) / 2
+#define SJ_MAX_FWD 6560  // 3^8 - 1 rows (UNICOMP in 8-D)
 
 // WorkQueue chunk: at most kChunk D' positions; cells with at least kBigCell points get
 // chunks of their own.
@@ -92,6 +92,8 @@ struct Index {
     uint64_t nc[SJ_MAX_DIM] = {0};
     uint64_t stride[SJ_MAX_DIM] = {0};
     int key_bits = 0;
+    int pattern = SJ_PATTERN_LID_UNICOMP;  // cell access pattern (sj_create_ex)
+    int order = SJ_ORDER_WORKLOAD;         // D' order (sj_create_ex)
     uint64_t n_cells = 0;     // M
     uint64_t n_runs = 0;      // E, forward runs over all cells
     uint64_t dist_calcs = 0;  // D_alg
@@ -132,6 +134,7 @@ struct JoinArgs {
     unsigned long long v_begin;   // batch = virtual chunk range [v_begin, v_end) of this slice
     unsigned long long v_end;
     uint32_t grab;                // chunks per dequeue
+    uint32_t gcg;                 // 1: GCG pattern (full neighbourhood, one pair per hit)
     uint32_t rank, world;         // queue slice: virtual chunk v -> chunk v*world + rank
     uint32_t *out;                // interleaved pairs, or nullptr (count-only)
     unsigned long long *emit_ctr; // pairs emitted (may exceed out_cap -> overflow)
@@ -142,7 +145,7 @@ struct JoinArgs {
 // Launch the join kernel for dim/k; emit=false counts pairs only.
 int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaStream_t s);
 // Max resident CTAs per SM of the join kernel configuration.
-int join_occupancy(int dim, int k, bool emit, int *blocks_per_sm);
+int join_occupancy(int dim, int k, bool emit, bool gcg, int *blocks_per_sm);
 constexpr int kJoinThreads = 256;
 
 // --------------------------------------------------------------------------- misc kernels

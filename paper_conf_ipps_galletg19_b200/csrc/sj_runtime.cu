@@ -273,6 +273,7 @@ JoinArgs base_args(const sj_handle *h) {
     a.n_chunks = (uint32_t)h->ix.n_chunks;
     a.e2 = h->ix.e2;
     a.grab = h->grab;
+    a.gcg = h->ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
     a.rank = (uint32_t)h->rank;
     a.world = (uint32_t)h->world;
     return a;
@@ -280,7 +281,7 @@ JoinArgs base_args(const sj_handle *h) {
 
 int join_blocks(const sj_handle *h, bool emit, int *blocks) {
     int occ = 0;
-    SJ_TRY(join_occupancy(h->ix.dim, h->k, emit, &occ));
+    SJ_TRY(join_occupancy(h->ix.dim, h->k, emit, h->ix.pattern == SJ_PATTERN_GCG, &occ));
     if (h->blocks_per_sm > 0 && h->blocks_per_sm < occ) occ = h->blocks_per_sm;
     if (occ < 1) occ = 1;
     *blocks = occ * h->num_sms;
@@ -603,13 +604,21 @@ static void fill_static_stats(sj_handle *h) {
     for (int d = 0; d < SJ_MAX_DIM; ++d) st.nc[d] = d < h->ix.dim ? (uint32_t)h->ix.nc[d] : 0;
     st.n_chunks = h->ix.n_chunks;
     st.tiled_min = kBigCell;
+    st.pattern = (uint32_t)h->ix.pattern;
+    st.order = (uint32_t)h->ix.order;
 }
 
 sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
+    return sj_create_ex(points, n, dim, eps, SJ_PATTERN_LID_UNICOMP, SJ_ORDER_WORKLOAD);
+}
+
+sj_handle *sj_create_ex(const double *points, uint64_t n, int dim, double eps, int pattern, int order) {
     set_error("");
-    if (!points || n == 0 || n >= (1ull << 32) || dim < 1 || dim > SJ_MAX_DIM || !(eps > 0.0) || !std::isfinite(eps)) {
-        set_error("sj_create: invalid argument (points=%p n=%llu dim=%d eps=%g)", (const void *)points,
-                  (unsigned long long)n, dim, eps);
+    if (!points || n == 0 || n >= (1ull << 32) || dim < 1 || dim > SJ_MAX_DIM || !(eps > 0.0) || !std::isfinite(eps) ||
+        pattern < SJ_PATTERN_LID_UNICOMP || pattern > SJ_PATTERN_UNICOMP || order < SJ_ORDER_WORKLOAD ||
+        order > SJ_ORDER_INPUT) {
+        set_error("sj_create: invalid argument (points=%p n=%llu dim=%d eps=%g pattern=%d order=%d)",
+                  (const void *)points, (unsigned long long)n, dim, eps, pattern, order);
         return nullptr;
     }
     int ndev = 0;
@@ -640,6 +649,8 @@ sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
         d_raw = d_copy;
     }
     float ms = 0;
+    h->ix.pattern = pattern;
+    h->ix.order = order;
     debug_mark("create: upload issued");
     if (rc == SJ_OK) rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_a, h->ev_b, &ms);
     debug_mark("create: build_index");
@@ -766,7 +777,7 @@ namespace {
 struct BlobHeader {
     uint64_t magic;  // "SJIDX003"
     uint64_t n;
-    int32_t dim, pad, key_bits, reserved;
+    int32_t dim, pad, key_bits, pattern_order;
     double eps, e2, w;
     double mins[SJ_MAX_DIM];
     uint64_t nc[SJ_MAX_DIM];
@@ -787,6 +798,7 @@ BlobHeader make_header(const Index &ix) {
     b.dim = ix.dim;
     b.pad = ix.pad;
     b.key_bits = ix.key_bits;
+    b.pattern_order = ix.pattern | (ix.order << 8);
     b.eps = ix.eps;
     b.e2 = ix.e2;
     b.w = ix.w;
@@ -861,6 +873,8 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
     ix.dim = b.dim;
     ix.pad = b.pad;
     ix.key_bits = b.key_bits;
+    ix.pattern = b.pattern_order & 0xFF;
+    ix.order = (b.pattern_order >> 8) & 0xFF;
     ix.eps = b.eps;
     ix.e2 = b.e2;
     ix.w = b.w;

@@ -1,0 +1,131 @@
+"""The paper's ablation variants (Table II) on the GPU: cell patterns GCG
+(GPUCALCGLOBAL), UNICOMP ([18], Alg. 2) and LID-UNICOMP, and
+queue orders (SortByWL D', cell order, input order).  Every variant must return the oracle's
+pair set; their distance-calculation counts and per-cell patterns are pinned to the paper:
+  * GCG evaluates the full 3^n neighbourhood: exactly the oracle's full-scan count;
+  * UNICOMP and LID-UNICOMP evaluate each adjacent cell pair once: half of it;
+  * on a dense 2-D grid an inner cell compares to 4 cells under LID-UNICOMP (Fig. 5)
+    and to 0, 2, 6 or 8 cells under UNICOMP by coordinate parity (Alg. 2).
+"""
+import struct
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import oracle  # noqa: E402
+import paper_conf_ipps_galletg19_b200 as sj  # noqa: E402
+import workloads  # noqa: E402
+
+DEV = "cuda:0"
+PATTERNS = ["lid_unicomp", "gcg", "unicomp"]
+ORDERS = ["workload", "cell", "input"]
+
+
+def run(pts, eps, pattern, order, k=8, **opts):
+    with sj.Handle(torch.from_numpy(np.ascontiguousarray(pts)).to(DEV), eps, pattern=pattern, order=order, k=k,
+                   count_calcs=1, **opts) as h:
+        got = sj.self_join_pairs(h, DEV).cpu().numpy().view(np.uint32).reshape(-1, 2)
+        st = h.stats()
+    return got, st
+
+
+@pytest.mark.parametrize("pattern", PATTERNS)
+@pytest.mark.parametrize("order", ORDERS)
+@pytest.mark.parametrize("name,n", [("c2k64", 60_011), ("c3k64", 50_021), ("c4k32", 20_011)])
+def test_variants_match_oracle(pattern, order, name, n):
+    cfg = workloads.get_config(name).scaled(n)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    g = oracle.grid_count(pts, cfg.eps, with_hash=False)
+    for k in (1, 8):
+        got, st = run(pts, cfg.eps, pattern, order, k=k)
+        assert got.shape == want.shape, (pattern, order, k)
+        np.testing.assert_array_equal(oracle.canonical(got), want)
+        if pattern == "gcg":
+            assert st["calcs_measured"] == st["dist_calcs"] == g["calcs"]       # full 3^n scan
+        else:
+            assert st["calcs_measured"] == st["dist_calcs"] == g["calcs"] // 2  # each pair once
+        assert st["pattern"] == sj.PATTERNS[pattern] and st["order"] == sj.ORDERS[order]
+
+
+def test_variants_sw_shaped_staged():
+    cfg = workloads.get_config("c5").scaled(80_000)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    for pattern in PATTERNS:
+        got, _ = run(pts, cfg.eps, pattern, "workload", fast_path=0, batch_pairs=50_000)
+        np.testing.assert_array_equal(oracle.canonical(got), want)
+
+
+# ---------------------------------------------------------------- index blob parsing
+
+_HDR = struct.Struct("<QQiiiiddd8d8Q8QQQQQII7Q7QQ")
+
+
+def parse_blob(blob: np.ndarray):
+    f = _HDR.unpack_from(blob.tobytes()[:_HDR.size])
+    n, dim = f[1], f[2]
+    nc = f[17:25]
+    n_cells, n_runs = f[33], f[34]
+    off, nbytes = f[39:46], f[46:53]
+
+    def arr(i, dtype):
+        return np.frombuffer(blob.tobytes()[off[i]:off[i] + nbytes[i]], dtype=dtype)
+
+    cellq = arr(3, np.uint32).reshape(-1, 4)
+    runs = arr(4, np.uint32).reshape(-1, 2)
+    lids = arr(5, np.uint64)
+    return dict(n=n, dim=dim, nc=nc[:dim], n_cells=n_cells, n_runs=n_runs, cellq=cellq, runs=runs, lids=lids)
+
+
+def runs_per_cell(ix):
+    z = ix["cellq"][:, 2].astype(np.int64)
+    order = np.argsort(z, kind="stable")
+    counts = np.empty_like(z)
+    zs = z[order]
+    nxt = np.append(zs[1:], ix["n_runs"])
+    counts[order] = nxt - zs
+    return counts
+
+
+def dense_grid(g):
+    """One point per cell of a g x g grid (cell centres) + one point at the origin."""
+    c = (np.arange(g, dtype=np.float64) + 0.5)
+    xx, yy = np.meshgrid(c, c, indexing="ij")
+    pts = np.concatenate([np.zeros((1, 2)), np.stack([xx.ravel(), yy.ravel()], 1)])
+    return pts, 1.0
+
+
+@pytest.mark.parametrize("pattern", PATTERNS)
+def test_inner_cell_patterns_fig5_alg2(pattern):
+    pts, eps = dense_grid(24)
+    with sj.Handle(torch.from_numpy(pts).to(DEV), eps, pattern=pattern) as h:
+        nbytes = h.export_index()
+        blob = torch.empty(nbytes, dtype=torch.uint8)
+        h.export_index(blob, nbytes)
+    ix = parse_blob(blob.numpy())
+    nc1 = int(ix["nc"][1])
+    lid = ix["lids"].astype(np.int64)
+    c0, c1 = lid // nc1, lid % nc1
+    # inner cells away from cell (0, 0), which also holds the extra origin point
+    inner = (c0 >= 2) & (c1 >= 2) & (c0 < ix["nc"][0] - 1) & (c1 < nc1 - 1)
+    assert inner.sum() > 100
+    cnt = runs_per_cell(ix)[inner]
+    fwd_points = ix["cellq"][inner, 3]  # one point per inner neighbour cell
+    if pattern == "lid_unicomp":
+        # Fig. 5 / P:174: every inner cell compares to the same 4 neighbour cells (2 runs)
+        assert np.all(fwd_points == 4) and np.all(cnt == 2)
+    elif pattern == "gcg":
+        assert np.all(fwd_points == 9)  # whole 3x3 neighbourhood incl. the home cell
+    else:
+        # P:78 / Alg. 2: (even, even) -> 0, (odd, even) -> 2, (even, odd) -> 6, (odd, odd) -> 8
+        p0, p1 = c0[inner] & 1, c1[inner] & 1
+        want = np.select([(p0 == 0) & (p1 == 0), (p0 == 1) & (p1 == 0), (p0 == 0) & (p1 == 1)], [0, 2, 6], 8)
+        np.testing.assert_array_equal(fwd_points, want)
+        assert set(np.unique(fwd_points).tolist()) == {0, 2, 6, 8}
