@@ -61,6 +61,7 @@ struct WarpSmem {
     unsigned tile_orig[2][32];             // input ids of the staged candidates
     unsigned qorig[32];                 // input ids of the chunk's queries
     unsigned qrr[32];                   // the queries' positions in their (common) cell
+    unsigned char glist[32];            // generic path: lanes of the chunk's remaining queries
     // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
     // and the smaller footprint buys occupancy)
     alignas(16) uint2 buf[EMIT ? (DIM <= 3 ? kBufHits : kBufHits / 2) : 2];
@@ -222,17 +223,25 @@ __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
 // so their loads coincide), then the home half scan -- taking candidates t, t+k, ...
 template <int DIM, int K, bool EMIT, bool GCG>
 __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
-                                              uint2 *buf, int &nbuf, unsigned long long &nhits,
-                                              unsigned long long &ncalcs, int lane, unsigned lt) {
+                                              uint2 *buf, unsigned char *glist, int &nbuf,
+                                              unsigned long long &nhits, unsigned long long &ncalcs, int lane,
+                                              unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
     const unsigned nq = __popc(gmask);  // the chunk's queries handled here: lanes in gmask
+    // compacted list of those lanes (a contiguous prefix in the common all-generic case)
+    const bool prefix = gmask == (nq >= 32u ? 0xffffffffu : ((1u << nq) - 1u));
+    if (!prefix) {
+        __syncwarp();
+        if ((gmask >> lane) & 1u) glist[__popc(gmask & lt)] = (unsigned char)lane;
+        __syncwarp();
+    }
     for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
         const unsigned qi = r0 + grp;
         const bool valid = qi < nq;
-        const int src = valid ? (int)__fns(gmask, 0, (int)qi + 1) : 0;  // lane of the qi-th query
+        const int src = prefix ? (int)(qi & 31u) : (int)glist[qi & 31u];  // lane of the qi-th query
         const unsigned qlid = __shfl_sync(kFull, qm_lane.x, src);
         // the cell record was fetched per lane at chunk start: shuffle, do not reload
         uint4 ci;
@@ -533,7 +542,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
                 const unsigned n0 = __shfl_sync(kFull, nseg, s0);
                 tiled_chunk<DIM, K, EMIT, GCG>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
             }
-            if (gmask) generic_chunk<DIM, K, EMIT, GCG>(a, gmask, qm, ci, ws.buf, nbuf, nhits, ncalcs, lane, lt);
+            if (gmask) generic_chunk<DIM, K, EMIT, GCG>(a, gmask, qm, ci, ws.buf, ws.glist, nbuf, nhits, ncalcs, lane, lt);
         }
     }
     if constexpr (EMIT) {
