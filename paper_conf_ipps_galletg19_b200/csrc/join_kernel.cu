@@ -62,6 +62,9 @@ struct WarpSmem {
     unsigned qorig[32];                 // input ids of the chunk's queries
     unsigned qrr[32];                   // the queries' positions in their (common) cell
     unsigned char glist[32];            // generic path: lanes of the chunk's remaining queries
+    // 4-D..6-D: the segment cell's forward runs (<= 122) staged once, so the per-tile run walk
+    // reads shared memory instead of chasing L2 latency run by run
+    uint2 runs_s[(DIM >= 4 && DIM <= 6) ? 128 : 1];
     // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
     // and the smaller footprint buys occupancy)
     alignas(16) uint2 buf[EMIT ? (DIM <= 3 ? kBufHits : kBufHits / 2) : 2];
@@ -190,11 +193,12 @@ __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs
 // ranked with __ballot_sync/__popc into the warp's shared buffer.  Before each round the
 // caller makes room for the round's maximum number of hits (flush_if) instead of checking
 // after every step.
-template <bool EMIT, bool GCG>
+template <bool EMIT, bool GCG, bool RARE = false>
 __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *buf, int &nbuf,
                                      unsigned long long &nhits, unsigned lt) {
     if constexpr (EMIT) {
         const unsigned hm = __ballot_sync(kFull, hit);
+        if (RARE && hm == 0u) return;  // high dimensions: most steps have no hit in the warp
         if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, oc);
         nbuf += __popc(hm);
     } else {
@@ -308,7 +312,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                 i += K;
             }
             flush_if<EMIT, GCG, BufCap<DIM>::value>(buf, nbuf, 32, a, lane);
-            emit<EMIT, GCG>(hit, oq, oc, buf, nbuf, nhits, lt);
+            emit<EMIT, GCG, (DIM >= 4)>(hit, oq, oc, buf, nbuf, nhits, lt);
         }
     }
 }
@@ -365,7 +369,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     if (d < 0) d += (int)m;
                     ok = ok & ((unsigned)d < hl);
                 }
-                emit<EMIT, GCG>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
+                emit<EMIT, GCG, (DIM >= 4)>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
             }
         }
     } else {  // tile slots read from shared memory each step (higher dimensions)
@@ -403,8 +407,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     ok1 = ok1 & ((unsigned)d1 < hl);
                 }
                 const bool hit0 = close0 & ok0, hit1 = close1 & ok1;
-                emit<EMIT, GCG>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt);
-                emit<EMIT, GCG>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt);
+                emit<EMIT, GCG, (DIM >= 4)>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt);
+                emit<EMIT, GCG, (DIM >= 4)>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt);
             }
         }
     }
@@ -433,12 +437,26 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
     }
     // ---- forward runs (LID-UNICOMP): tiles staged with cp.async, double-buffered, so the
     // next tile's global loads overlap this tile's distance calculations
-    unsigned e = ci.z, seg_base = 0, seg_len = 0, i = (unsigned)lane;
+    const uint2 *runs = a.runs + ci.z;
+    bool runs_smem = false;
+    if constexpr (DIM >= 4 && DIM <= 6) {  // copy the cell's runs until their lengths add up to S
+        unsigned acc = 0;
+        for (unsigned k0 = 0; acc < S && k0 < 128u; k0 += 32) {
+            const unsigned k = k0 + (unsigned)lane;
+            const uint2 f = (ci.z + k < a.n_runs) ? __ldg(a.runs + ci.z + k) : make_uint2(0, 0);
+            ws.runs_s[k] = f;
+            acc += __reduce_add_sync(kFull, f.y);
+        }
+        __syncwarp();
+        runs_smem = acc >= S;  // GCG / UNICOMP lists can exceed 128 runs: keep reading L2 then
+        if (runs_smem) runs = ws.runs_s;
+    }
+    unsigned e = 0, seg_base = 0, seg_len = 0, i = (unsigned)lane;
     auto stage_fwd = [&](int b, unsigned tb) {
         if (tb + (unsigned)lane < S) {
             while (i >= seg_len) {
                 i -= seg_len;
-                const uint2 f = __ldg(a.runs + (e++));
+                const uint2 f = runs_smem ? runs[e++] : __ldg(runs + (e++));
                 seg_base = f.x;
                 seg_len = f.y;
             }

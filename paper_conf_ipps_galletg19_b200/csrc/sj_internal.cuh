@@ -129,6 +129,7 @@ struct JoinArgs {
     const uint2 *runs;
     const uint32_t *chunks;       // WorkQueue chunks of D'
     uint32_t n_chunks;
+    uint64_t n_runs;              // entries of runs (bounds of the staged copies)
     double e2;
     unsigned long long *head;     // WorkQueue counter (chunks taken), zeroed before the launch
     unsigned long long v_begin;   // batch = virtual chunk range [v_begin, v_end) of this slice

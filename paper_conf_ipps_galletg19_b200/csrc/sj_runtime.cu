@@ -316,6 +316,7 @@ JoinArgs base_args(const sj_handle *h) {
     a.runs = h->ix.runs;
     a.chunks = h->ix.chunks;
     a.n_chunks = (uint32_t)h->ix.n_chunks;
+    a.n_runs = h->ix.n_runs;
     a.e2 = h->ix.e2;
     a.grab = h->grab;
     a.gcg = h->ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
