@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define SJ_ABI_VERSION 1
+#define SJ_ABI_VERSION 2
 
 typedef struct sj_handle sj_handle;
 
@@ -57,8 +57,14 @@ enum sj_option {
     SJ_OPT_GRAB = 5,           /* WorkQueue chunks one warp dequeues per atomic (1..1024); default 1     */
     SJ_OPT_COUNT_CALCS = 6,    /* 1 = instrument the join with a distance-calculation counter; default 0 */
     SJ_OPT_BLOCKS_PER_SM = 7,  /* persistent-grid CTAs per SM; 0 = occupancy maximum (default)           */
-    SJ_OPT_FAST_PATH = 8       /* 1 = device output written in place when it fits (default); 0 = always
+    SJ_OPT_FAST_PATH = 8,      /* 1 = device output written in place when it fits (default); 0 = always
                                   stage per batch (the paper's scheme)                             */
+    SJ_OPT_EXACT = 9           /* 1 = exact two-pass sizing: a count pass records every
+                                  WorkQueue chunk's pairs, their scan gives each chunk its output slots,
+                                  batches are cut at exact sizes <= b_s and the fill pass writes each
+                                  chunk at its own offset -- no estimator, no overflow retries, and the
+                                  output ORDER is deterministic.  0 = the paper's 1% estimator (P:71,
+                                  P:200) with atomic placement (default)                                 */
 };
 
 /* Cell access patterns (sj_create_ex).  The paper's variants, Table II:
@@ -141,6 +147,23 @@ sj_handle *sj_create_ex(const double *points, uint64_t n, int dim, double eps, i
  * Errors: SJ_EINVAL (NULL count, out_pairs NULL with cap > 0, misaligned device
  * buffer), SJ_ECUDA, SJ_ENOMEM; after an error the handle answers SJ_ESTATE. */
 int sj_self_join(sj_handle *h, uint32_t *out_pairs, uint64_t cap, uint64_t *count);
+
+/* Device-resident CSR neighbour lists (the clustering consumers of a
+ * self-join): row i holds the input ids j != i with s(i, j) <= fl(eps^2), i.e.
+ * nbrs[row_off[i] .. row_off[i+1]) -- the same pair set as sj_self_join, grouped by i.
+ * Needs a handle created with SJ_PATTERN_GCG (sj_create_ex): with the full 3^n
+ * neighbourhood (Alg. 1) every query point evaluates all of its own candidates,
+ * so it owns its row and the two passes (degrees -> exclusive scan -> fill) need no
+ * atomics; and the whole queue (slice world 1).
+ *   row_off : uint64[n+1] (host or device), or NULL; receives the exclusive scan of the
+ *             degrees, row_off[n] = total.
+ *   nbrs    : uint32[cap] (host or device), or NULL with cap == 0 (offsets only).
+ *   total   : receives the number of ordered pairs (sum of the degrees).
+ * Row contents follow the neighbourhood traversal order (deterministic, not sorted).
+ * Returns SJ_OK; SJ_EINVAL for NULL total, a handle of another pattern or slice, a
+ * join continuation in progress (SJ_MORE pending), or cap < total (row_off and *total
+ * are filled first, nbrs untouched; the handle stays usable); SJ_ECUDA / SJ_ENOMEM. */
+int sj_neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, uint64_t *total);
 
 /* Free every device / pinned resource of the handle.  NULL-safe. */
 void sj_destroy(sj_handle *h);

@@ -16,7 +16,7 @@ SJ_ORDER_WORKLOAD, SJ_ORDER_CELL, SJ_ORDER_INPUT = 0, 1, 2
 PATTERNS = {"lid_unicomp": SJ_PATTERN_LID_UNICOMP, "gcg": SJ_PATTERN_GCG, "unicomp": SJ_PATTERN_UNICOMP}
 ORDERS = {"workload": SJ_ORDER_WORKLOAD, "cell": SJ_ORDER_CELL, "input": SJ_ORDER_INPUT}
 (SJ_OPT_K, SJ_OPT_BATCH_PAIRS, SJ_OPT_STREAMS, SJ_OPT_SAMPLE_PPM, SJ_OPT_GRAB, SJ_OPT_COUNT_CALCS,
- SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH) = range(1, 9)
+ SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH, SJ_OPT_EXACT) = range(1, 10)
 _NAMES = {0: "SJ_OK", 1: "SJ_MORE", -1: "SJ_EINVAL", -2: "SJ_ENOMEM", -3: "SJ_ECUDA", -4: "SJ_EGRID",
           -5: "SJ_ESTATE"}
 
@@ -70,6 +70,7 @@ _sig = {
     "sj_slice_chunks": (_i64, [_u64, _int, _int, _vp, _u64]),
     "sj_measure_fp64": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
     "sj_measure_atomics": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
+    "sj_neighbor_csr": (_int, [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]),
 }
 for _n, (_r, _a) in _sig.items():
     _f = getattr(_lib, _n)
@@ -170,6 +171,14 @@ def sj_self_join(h: int, out, cap: int):
     return rc, int(cnt.value)
 
 
+def sj_neighbor_csr(h: int, row_off, nbrs, cap: int) -> int:
+    """Fills row_off (uint64[n+1]) and, if nbrs is given, nbrs (uint32[cap]); returns the
+    total number of neighbour entries.  Raises SJError on error (incl. cap < total)."""
+    tot = _u64(0)
+    _check(_lib.sj_neighbor_csr(h, _ptr(row_off), _ptr(nbrs), int(cap), ctypes.byref(tot)))
+    return int(tot.value)
+
+
 def sj_destroy(h: int) -> None:
     _lib.sj_destroy(h)
 
@@ -248,7 +257,7 @@ class Handle:
 
     _OPTS = {"k": SJ_OPT_K, "batch_pairs": SJ_OPT_BATCH_PAIRS, "streams": SJ_OPT_STREAMS,
              "sample_ppm": SJ_OPT_SAMPLE_PPM, "grab": SJ_OPT_GRAB, "count_calcs": SJ_OPT_COUNT_CALCS,
-             "blocks_per_sm": SJ_OPT_BLOCKS_PER_SM, "fast_path": SJ_OPT_FAST_PATH}
+             "blocks_per_sm": SJ_OPT_BLOCKS_PER_SM, "fast_path": SJ_OPT_FAST_PATH, "exact": SJ_OPT_EXACT}
 
     def set_option(self, name, value) -> None:
         sj_set_option(self.h, self._OPTS[name] if isinstance(name, str) else name, int(value))
@@ -264,6 +273,21 @@ class Handle:
 
     def stats(self) -> dict:
         return sj_get_stats(self.h)
+
+    def neighbor_csr(self, device: str = "cuda"):
+        """Device-resident CSR (needs pattern="gcg"): (row_off int64 (n+1,), nbrs int32 (total,))
+        torch tensors holding the uint64 offsets / uint32 input ids, on `device` ("cpu":
+        pinned host memory)."""
+        import torch
+
+        n = self.stats()["n"]
+        pin = device == "cpu"
+        kw = dict(pin_memory=True) if pin else dict(device=device)
+        row_off = torch.empty(n + 1, dtype=torch.int64, **kw)
+        total = sj_neighbor_csr(self.h, row_off, None, 0)
+        nbrs = torch.empty(max(total, 1), dtype=torch.int32, **kw)
+        sj_neighbor_csr(self.h, row_off, nbrs, max(total, 1))
+        return row_off, nbrs[:total]
 
     def export_index(self, dst=None, cap: int = 0) -> int:
         return sj_export_index(self.h, dst, cap)

@@ -38,6 +38,12 @@ namespace {
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarps = kJoinThreads / 32;
 constexpr int kBufHits = 512;  // hits buffered per warp ({orig q, orig c}, 8 B -> 4 KB)
+#ifndef SJ_BUF_HI
+#define SJ_BUF_HI 96
+#endif
+// 4..8-D: few hits per calculation; the small buffer keeps a warp's shared memory under
+// 7 KB, so four 256-thread CTAs fit an SM (occupancy of the FP64-bound kernels)
+constexpr int kBufHitsHi = SJ_BUF_HI;
 // A cell segment of >= 2 queries is tiled when its forward list has at least this many
 // candidates (6-D: ~1300 per cell of ~4 points), so staging pays for itself.
 constexpr unsigned kTileMinCand = 128;
@@ -47,13 +53,21 @@ struct PointPad {
     static constexpr int value = DIM == 1 ? 1 : ((DIM + 1) & ~1);
 };
 
+// Compile-time traits of the kernel modes (JoinMode): exact sizing and the per-chunk counts
+// are modes of their own so the default kernels carry none of their code.
+template <int MODE>
+struct Mode {
+    static constexpr bool pairs = MODE == kPairs || MODE == kExact;  // emits the pair list
+    static constexpr bool exact = MODE == kExact;                     // ... at chunk offsets
+};
+
 template <int DIM>
 struct BufCap {
-    static constexpr int value = DIM <= 3 ? kBufHits : kBufHits / 2;
+    static constexpr int value = DIM <= 3 ? kBufHits : kBufHitsHi;
 };
 
 // Per-warp shared memory: emission buffer, the chunk's queries, one candidate tile.
-template <int DIM, bool EMIT>
+template <int DIM, int MODE>
 struct WarpSmem {
     static constexpr int PAD = PointPad<DIM>::value;
     alignas(16) double tile[2][32 * PAD];  // staged candidates (lid order), double-buffered
@@ -67,7 +81,10 @@ struct WarpSmem {
     uint2 runs_s[(DIM >= 4 && DIM <= 6) ? 128 : 1];
     // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
     // and the smaller footprint buys occupancy)
-    alignas(16) uint2 buf[EMIT ? (DIM <= 3 ? kBufHits : kBufHits / 2) : 2];
+    alignas(16) uint2 buf[Mode<MODE>::pairs ? BufCap<DIM>::value : 2];
+    unsigned long long wcur;  // kPairs, exact sizing: next output slot of the current chunk
+    // kRows: the segment's per-query row cursors; kDegree: their running neighbour counts
+    unsigned long long qcur[(MODE == kRows || MODE == kDegree) ? 32 : 1];
 };
 
 template <int DIM>
@@ -155,12 +172,21 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
 // Flush a warp's staged hits: ONE atomicAdd reserves the output slots, then the lanes write
 // coalesced streaming stores: both mirrored pairs of a hit as one 16-B store {q, c, c, q}
 // (half patterns), or the single pair {q, c} (GCG, which meets every pair twice).
-template <bool GCG>
-__device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane) {
+// Exact sizing (kExact): the slots come from the chunk's own cursor instead, so the output
+// order is deterministic; the counter still totals the pairs.
+template <bool GCG, bool EXACT>
+__device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane,
+                                      unsigned long long *wcur) {
     __syncwarp();
     constexpr unsigned long long kPer = GCG ? 1ull : 2ull;  // pairs per buffered hit
     unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)nbuf);
+    if (lane == 0) {
+        base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)nbuf);
+        if (EXACT) {
+            base = *wcur;
+            *wcur = base + kPer * (unsigned long long)nbuf;
+        }
+    }
     base = __shfl_sync(kFull, base, 0);
     uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
     if constexpr (GCG) {
@@ -192,28 +218,46 @@ __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs
 // Warp-aggregated emission of one evaluation step (all 32 lanes call it): the hits are
 // ranked with __ballot_sync/__popc into the warp's shared buffer.  Before each round the
 // caller makes room for the round's maximum number of hits (flush_if) instead of checking
-// after every step.
-template <bool EMIT, bool GCG, bool RARE = false>
+// after every step.  kRows: the hits of a k-lane group (gbits) go straight to the group's
+// query row at its cursor `cur`, in candidate order.
+template <int MODE, bool GCG, bool RARE = false>
 __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *buf, int &nbuf,
-                                     unsigned long long &nhits, unsigned lt) {
-    if constexpr (EMIT) {
+                                     unsigned long long &nhits, unsigned lt, unsigned gbits,
+                                     unsigned long long &cur, const JoinArgs &a) {
+    if constexpr (Mode<MODE>::pairs) {
         const unsigned hm = __ballot_sync(kFull, hit);
         if (RARE && hm == 0u) return;  // high dimensions: most steps have no hit in the warp
         if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, oc);
         nbuf += __popc(hm);
+    } else if constexpr (MODE == kRows) {
+        const unsigned all = __ballot_sync(kFull, hit);
+        if (RARE && all == 0u) return;
+        const unsigned hm = all & gbits;
+        if (hit) a.nbrs[cur + __popc(hm & lt)] = oc;
+        cur += __popc(hm);
+        nhits += hit ? 1ull : 0ull;
     } else {
         nhits += hit ? (GCG ? 1ull : 2ull) : 0ull;
     }
 }
 
-template <bool EMIT, bool GCG, int CAP = kBufHits>
-__device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane) {
-    if constexpr (EMIT) {
+template <int MODE, bool GCG, int CAP = kBufHits>
+__device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane,
+                                         unsigned long long *wcur) {
+    if constexpr (Mode<MODE>::pairs) {
         if (nbuf > CAP - room) {
-            flush<GCG>(buf, nbuf, a, lane);
+            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
             nbuf = 0;
         }
     }
+}
+
+// Sum over the k lanes of a group (groups are aligned runs of K lanes).
+template <int K>
+__device__ __forceinline__ unsigned group_sum(unsigned v) {
+#pragma unroll
+    for (int o = K / 2; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    return v;
 }
 
 // Home cell of one query: the balanced circulant half scan (reading c8) -- position rr
@@ -225,15 +269,17 @@ __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
 // Generic path: rounds of 32/k queries (possibly from different cells); the k lanes of a
 // group walk their query's list -- forward runs first (identical for queries of one cell,
 // so their loads coincide), then the home half scan -- taking candidates t, t+k, ...
-template <int DIM, int K, bool EMIT, bool GCG>
+template <int DIM, int K, int MODE, bool GCG>
 __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
-                                              uint2 *buf, unsigned char *glist, int &nbuf,
-                                              unsigned long long &nhits, unsigned long long &ncalcs, int lane,
-                                              unsigned lt) {
+                                              WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
+                                              unsigned long long &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
+    const unsigned gbits = K == 32 ? kFull : (((1u << K) - 1u) << (lane & ~(K - 1)));
+    uint2 *buf = ws.buf;
+    unsigned char *glist = ws.glist;
     const unsigned nq = __popc(gmask);  // the chunk's queries handled here: lanes in gmask
     // compacted list of those lanes (a contiguous prefix in the common all-generic case)
     const bool prefix = gmask == (nq >= 32u ? 0xffffffffu : ((1u << nq) - 1u));
@@ -257,10 +303,12 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         unsigned oq = 0;
         uint2 nxt = make_uint2(0, 0);
         if (!valid) ci = make_uint4(0, 0, 0, 0);
+        unsigned long long cur = 0;  // kRows: the query's row cursor
         if (valid) {
             load_point<DIM>(a.pts + (size_t)qlid * PAD, qp);
             oq = __ldg(a.orig + qlid);
             if (ci.w) nxt = __ldg(a.runs + ci.z);  // prefetched next run
+            if constexpr (MODE == kRows) cur = __ldg(a.row_off + oq);
         } else {
 #pragma unroll
             for (int d = 0; d < DIM; ++d) qp[d] = 0.0;
@@ -280,6 +328,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         ncalcs += my_iters;
         if (GCG && valid && t == 0 && total) ncalcs -= 1;  // the query itself is skipped
         unsigned gi = t;
+        const unsigned long long nh0 = nhits;
         for (unsigned it = 0; it < iters; ++it, gi += K) {
             bool hit = false;
             unsigned cidx = 0, oc = 0;
@@ -306,13 +355,17 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                 }
                 double cp[DIM];
                 load_point<DIM>(a.pts + (size_t)cidx * PAD, cp);
-                if (EMIT) oc = __ldg(a.orig + cidx);  // issued with the point, not after the test
+                if (Mode<MODE>::pairs || MODE == kRows) oc = __ldg(a.orig + cidx);  // issued with the point, not after the test
                 hit = sqdist<DIM>(qp, cp) <= a.e2;
                 if (GCG) hit = hit && cidx != qlid;  // GCG scans its own cell: skip (q, q)
                 i += K;
             }
-            flush_if<EMIT, GCG, BufCap<DIM>::value>(buf, nbuf, 32, a, lane);
-            emit<EMIT, GCG, (DIM >= 4)>(hit, oq, oc, buf, nbuf, nhits, lt);
+            flush_if<MODE, GCG, BufCap<DIM>::value>(buf, nbuf, 32, a, lane, &ws.wcur);
+            emit<MODE, GCG, (DIM >= 4)>(hit, oq, oc, buf, nbuf, nhits, lt, gbits, cur, a);
+        }
+        if constexpr (MODE == kDegree) {  // the query's degree: its group's hits
+            const unsigned deg = group_sum<K>((unsigned)(nhits - nh0));
+            if (valid && t == 0) a.qdeg[oq] = deg;
         }
     }
 }
@@ -320,9 +373,9 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
 // Evaluate one staged tile against every query of the chunk.  HOME: the tile holds home-cell
 // positions tb.. and a (query, slot) pair is inside the query's circulant half scan iff
 // (p - rr - 1) mod m < home_count(m, rr) (reading c8).
-template <int DIM, int K, bool EMIT, bool GCG, bool HOME>
+template <int DIM, int K, int MODE, bool GCG, bool HOME>
 __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
-                                            WarpSmem<DIM, EMIT> &ws, int b, int &nbuf, unsigned long long &nhits,
+                                            WarpSmem<DIM, MODE> &ws, int b, int &nbuf, unsigned long long &nhits,
                                             int lane, unsigned lt) {
     const double *tile = ws.tile[b];
     const unsigned *tile_orig = ws.tile_orig[b];
@@ -331,6 +384,16 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
     constexpr int SPL = 32 / K;  // tile slots per lane
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
+    const unsigned gbits = K == 32 ? kFull : (((1u << K) - 1u) << (lane & ~(K - 1)));
+    // kRows / kDegree: the round's query cursor (count) lives in ws.qcur between rounds
+    auto round_end = [&](unsigned qi, bool qv, unsigned long long cur, unsigned long long nh0) {
+        if constexpr (MODE == kRows) {
+            if (t == 0 && qv) ws.qcur[qi] = cur;
+        } else if constexpr (MODE == kDegree) {
+            const unsigned d = group_sum<K>((unsigned)(nhits - nh0));
+            if (t == 0 && qv) ws.qcur[qi] += d;
+        }
+    };
     if constexpr (SPL <= 4 && DIM <= 3) {  // tile slots in registers (register budget)
         double cp[SPL][DIM];
         unsigned co[SPL];
@@ -353,7 +416,9 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 rr = ws.qrr[qi];
                 hl = home_count(m, rr);
             }
-            flush_if<EMIT, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
+            unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
+            const unsigned long long nh0 = nhits;
+            flush_if<MODE, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.wcur);
             // all SPL distances first (independent FP64 chains -> ILP), then the emissions;
             // evaluated unconditionally and masked after (invalid slots may hold stale or
             // uninitialised bits; FP64 arithmetic on them cannot trap)
@@ -369,10 +434,69 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     if (d < 0) d += (int)m;
                     ok = ok & ((unsigned)d < hl);
                 }
-                emit<EMIT, GCG, (DIM >= 4)>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt);
+                emit<MODE, GCG, (DIM >= 4)>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt, gbits, cur, a);
+            }
+            round_end(qi, qv, cur, nh0);
+        }
+    } else if constexpr (DIM >= 4) {
+        // Higher dimensions: a lane keeps ONE tile slot (its candidate, 2*DIM registers) for the
+        // whole tile and the warp walks the segment's queries two at a time; the query reads are
+        // shared-memory broadcasts, so each staged coordinate is read once per lane per tile
+        // instead of once per round (the k-lane split of the rounds above is a register-budget
+        // device of the low-dimensional path; all 32 lanes serve one query here).
+        const bool cv = (unsigned)lane < nt;
+        double cp[DIM];
+        load_smem_point<DIM>(tile + lane * PAD, cp);
+        const unsigned co = tile_orig[lane];
+        int dh = (int)(tb + (unsigned)lane) - 1;  // HOME: slot position - 1, minus rr below
+        for (unsigned q0 = 0; q0 < nq; q0 += 2) {
+            const unsigned q1 = q0 + 1;
+            const bool v1 = q1 < nq;
+            double qa[DIM], qb[DIM];
+            load_smem_point<DIM>(ws.qry + q0 * PAD, qa);
+            load_smem_point<DIM>(ws.qry + (q1 & 31) * PAD, qb);
+            const bool ca = sqdist<DIM>(qa, cp) <= a.e2;  // two independent FP64 chains
+            const bool cb = sqdist<DIM>(qb, cp) <= a.e2;
+            const unsigned oqa = ws.qorig[q0], oqb = ws.qorig[q1 & 31];
+            bool oka = cv, okb = cv & v1;
+            if (GCG) {  // skip (q, q)
+                oka = oka & (co != oqa);
+                okb = okb & (co != oqb);
+            }
+            if (HOME) {
+                const unsigned rra = ws.qrr[q0], rrb = ws.qrr[q1 & 31];
+                int da = dh - (int)rra, db = dh - (int)rrb;
+                if (da < 0) da += (int)m;
+                if (db < 0) db += (int)m;
+                oka = oka & ((unsigned)da < home_count(m, rra));
+                okb = okb & ((unsigned)db < home_count(m, rrb));
+            }
+            const bool ha = ca & oka, hb = cb & okb;
+            flush_if<MODE, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
+            unsigned long long cura = 0, curb = 0;
+            if constexpr (MODE == kRows) {
+                cura = ws.qcur[q0];
+                curb = ws.qcur[q1 & 31];
+            }
+            emit<MODE, GCG, true>(ha, oqa, co, ws.buf, nbuf, nhits, lt, kFull, cura, a);
+            emit<MODE, GCG, true>(hb, oqb, co, ws.buf, nbuf, nhits, lt, kFull, curb, a);
+            if constexpr (MODE == kRows) {
+                __syncwarp();
+                if (lane == 0) {
+                    ws.qcur[q0] = cura;
+                    if (v1) ws.qcur[q1] = curb;
+                }
+                __syncwarp();
+            } else if constexpr (MODE == kDegree) {
+                const unsigned na = __popc(__ballot_sync(kFull, ha)), nb = __popc(__ballot_sync(kFull, hb));
+                if (lane == 0) {
+                    ws.qcur[q0] += na;
+                    if (v1) ws.qcur[q1] += nb;
+                }
+                __syncwarp();
             }
         }
-    } else {  // tile slots read from shared memory each step (higher dimensions)
+    } else {  // tile slots read from shared memory each step (low dimensions, k < 8)
         for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
             const unsigned qi = (r0 + grp) & 31;
             const bool qv = r0 + grp < nq;
@@ -384,9 +508,11 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 rr = ws.qrr[qi];
                 hl = home_count(m, rr);
             }
-            flush_if<EMIT, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane);
+            unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
+            const unsigned long long nh0 = nhits;
 #pragma unroll 2
             for (int s = 0; s < SPL; s += 2) {  // two slots per step: two independent FP64 chains
+                flush_if<MODE, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
                 const unsigned j0 = t + (unsigned)(K * s), j1 = j0 + (unsigned)K;
                 double c0[DIM], c1[DIM];
                 load_smem_point<DIM>(tile + (j0 & 31) * PAD, c0);
@@ -407,9 +533,12 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     ok1 = ok1 & ((unsigned)d1 < hl);
                 }
                 const bool hit0 = close0 & ok0, hit1 = close1 & ok1;
-                emit<EMIT, GCG, (DIM >= 4)>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt);
-                emit<EMIT, GCG, (DIM >= 4)>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt);
+                emit<MODE, GCG, (DIM >= 4)>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
+                                            cur, a);
+                emit<MODE, GCG, (DIM >= 4)>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
+                                            cur, a);
             }
+            round_end(qi, qv, cur, nh0);
         }
     }
 }
@@ -419,9 +548,9 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
 // shared memory (points + input ids); lane t of a group holds tile slots t, t+k, ... and
 // evaluates them against one query per round of 32/k queries, so each staged candidate
 // serves the whole chunk.
-template <int DIM, int K, bool EMIT, bool GCG>
+template <int DIM, int K, int MODE, bool GCG>
 __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsigned nq, uint2 qm_lane, uint4 ci,
-                                            WarpSmem<DIM, EMIT> &ws, int &nbuf, unsigned long long &nhits,
+                                            WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
                                             unsigned long long &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     const unsigned hb = ci.x, m = ci.y, S = ci.w;
@@ -429,7 +558,10 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
     const unsigned slot = (unsigned)lane - s0;  // the segment's queries are lanes s0 .. s0+nq-1
     if (slot < nq) {
         copy_point_to_smem<DIM>(a.pts + (size_t)qm_lane.x * PAD, ws.qry + slot * PAD);
-        ws.qorig[slot] = __ldg(a.orig + qm_lane.x);
+        const unsigned oq = __ldg(a.orig + qm_lane.x);
+        ws.qorig[slot] = oq;
+        if constexpr (MODE == kRows) ws.qcur[slot] = __ldg(a.row_off + oq);
+        if constexpr (MODE == kDegree) ws.qcur[slot] = 0;
         const unsigned rr = qm_lane.x - hb;
         ws.qrr[slot] = rr;
         // this query's distance calculations
@@ -477,7 +609,7 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, EMIT, GCG, false>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, MODE, GCG, false>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
         __syncwarp();
     }
     // ---- home cell: balanced circulant half scan as a mask over staged home tiles
@@ -489,7 +621,13 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         }
         cp_async_commit();
     };
-    if (GCG) return;  // GCG: the home cell was one of the runs
+    if constexpr (GCG) {  // GCG: the home cell was one of the runs
+        if constexpr (MODE == kDegree) {
+            if (slot < nq) a.qdeg[ws.qorig[slot]] = (unsigned)ws.qcur[slot];
+            __syncwarp();
+        }
+        return;
+    }
     stage_home(0, 0);
     it = 0;
     for (unsigned tb = 0; tb < m; tb += 32, ++it) {
@@ -500,12 +638,12 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, EMIT, GCG, true>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, MODE, GCG, true>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
         __syncwarp();
     }
 }
 
-template <int DIM, int K, bool EMIT, bool GCG>
+template <int DIM, int K, int MODE, bool GCG>
 __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     static_assert(32 % K == 0, "k must divide 32");
     constexpr int QPW = 32 / K;
@@ -513,7 +651,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
-    WarpSmem<DIM, EMIT> &ws = reinterpret_cast<WarpSmem<DIM, EMIT> *>(smem_raw)[warp];
+    WarpSmem<DIM, MODE> &ws = reinterpret_cast<WarpSmem<DIM, MODE> *>(smem_raw)[warp];
     int nbuf = 0;
     unsigned long long nhits = 0;
     unsigned long long ncalcs = 0;
@@ -528,6 +666,11 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         for (unsigned long long v = vb; v < vend; ++v) {
             const unsigned long long c = v * a.world + a.rank;  // queue slice (multi-GPU)
             if (c >= a.n_chunks) break;
+            if constexpr (MODE == kExact) {  // exact sizing: the chunk's pairs start at voff[v]
+                if (lane == 0) ws.wcur = __ldg(a.voff + v) - a.out_base;
+                __syncwarp();
+            }
+            const unsigned long long nh0 = nhits;
             const unsigned qs = __ldg(a.chunks + c), qe = __ldg(a.chunks + c + 1);
             const unsigned nq = qe - qs;  // 1..32 D' positions
             const bool lv = (unsigned)lane < nq;
@@ -558,13 +701,25 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
                 cs.z = __shfl_sync(kFull, ci.z, s0);
                 cs.w = __shfl_sync(kFull, ci.w, s0);
                 const unsigned n0 = __shfl_sync(kFull, nseg, s0);
-                tiled_chunk<DIM, K, EMIT, GCG>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
+                tiled_chunk<DIM, K, MODE, GCG>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
             }
-            if (gmask) generic_chunk<DIM, K, EMIT, GCG>(a, gmask, qm, ci, ws.buf, ws.glist, nbuf, nhits, ncalcs, lane, lt);
+            if (gmask) generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
+            if constexpr (MODE == kExact) {  // exact sizing: a chunk's pairs never share a flush
+                if (nbuf > 0) {
+                    flush<GCG, true>(ws.buf, nbuf, a, lane, &ws.wcur);
+                    nbuf = 0;
+                }
+            } else if constexpr (MODE == kChunkCount) {  // exact sizing, pass 1: pairs per chunk
+                unsigned long long d = nhits - nh0;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(kFull, d, o);
+                if (lane == 0) a.vcount[v] = d;
+            }
+            (void)nh0;
         }
     }
-    if constexpr (EMIT) {
-        if (nbuf > 0) flush<GCG>(ws.buf, nbuf, a, lane);
+    if constexpr (Mode<MODE>::pairs) {
+        if (nbuf > 0) flush<GCG, Mode<MODE>::exact>(ws.buf, nbuf, a, lane, &ws.wcur);
     } else {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) nhits += __shfl_xor_sync(kFull, nhits, o);
@@ -584,53 +739,74 @@ struct KernelInfo {
     size_t smem = 0;
 };
 
-template <int DIM, int K, bool EMIT, bool GCG>
+template <int DIM, int K, int MODE, bool GCG>
 KernelInfo info() {
     KernelInfo ki;
-    ki.f = join_kernel<DIM, K, EMIT, GCG>;
-    ki.smem = sizeof(WarpSmem<DIM, EMIT>) * kWarps;
+    ki.f = join_kernel<DIM, K, MODE, GCG>;
+    ki.smem = sizeof(WarpSmem<DIM, MODE>) * kWarps;
     return ki;
 }
 
-// The LID-UNICOMP / UNICOMP kernels exist for every k; the GCG ablation kernels for the
-// k the paper evaluates (1 and 8) and 32.
-template <int DIM, bool EMIT, bool GCG>
+// The LID-UNICOMP / UNICOMP kernels exist for every k; the GCG kernels (ablation, and the
+// row-owner CSR modes) for the k the paper evaluates (1 and 8) and 32.
+template <int DIM, int MODE, bool GCG>
 KernelInfo pick_k(int k) {
+#ifdef SJ_QUICK  // register / SASS experiments: one k only
+    return k == 8 ? info<DIM, 8, MODE, GCG>() : KernelInfo();
+#else
     switch (k) {
-        case 1: return info<DIM, 1, EMIT, GCG>();
-        case 8: return info<DIM, 8, EMIT, GCG>();
-        case 32: return info<DIM, 32, EMIT, GCG>();
+        case 1: return info<DIM, 1, MODE, GCG>();
+        case 8: return info<DIM, 8, MODE, GCG>();
+        case 32: return info<DIM, 32, MODE, GCG>();
     }
     if constexpr (!GCG) {
         switch (k) {
-            case 2: return info<DIM, 2, EMIT, false>();
-            case 4: return info<DIM, 4, EMIT, false>();
-            case 16: return info<DIM, 16, EMIT, false>();
+            case 2: return info<DIM, 2, MODE, false>();
+            case 4: return info<DIM, 4, MODE, false>();
+            case 16: return info<DIM, 16, MODE, false>();
         }
     }
     return KernelInfo();
+#endif
 }
 
-template <bool EMIT, bool GCG>
+template <int MODE, bool GCG>
 KernelInfo pick(int dim, int k) {
+#ifdef SJ_QUICK
     switch (dim) {
-        case 1: return pick_k<1, EMIT, GCG>(k);
-        case 2: return pick_k<2, EMIT, GCG>(k);
-        case 3: return pick_k<3, EMIT, GCG>(k);
-        case 4: return pick_k<4, EMIT, GCG>(k);
-        case 5: return pick_k<5, EMIT, GCG>(k);
-        case 6: return pick_k<6, EMIT, GCG>(k);
-        case 7: return pick_k<7, EMIT, GCG>(k);
-        case 8: return pick_k<8, EMIT, GCG>(k);
+        case 2: return pick_k<2, MODE, GCG>(k);
+        case 3: return pick_k<3, MODE, GCG>(k);
+        case 6: return pick_k<6, MODE, GCG>(k);
     }
     return KernelInfo();
+#else
+    switch (dim) {
+        case 1: return pick_k<1, MODE, GCG>(k);
+        case 2: return pick_k<2, MODE, GCG>(k);
+        case 3: return pick_k<3, MODE, GCG>(k);
+        case 4: return pick_k<4, MODE, GCG>(k);
+        case 5: return pick_k<5, MODE, GCG>(k);
+        case 6: return pick_k<6, MODE, GCG>(k);
+        case 7: return pick_k<7, MODE, GCG>(k);
+        case 8: return pick_k<8, MODE, GCG>(k);
+    }
+    return KernelInfo();
+#endif
 }
 
-int prepare(int dim, int k, bool emit, bool gcg, KernelInfo *out) {
-    KernelInfo ki = gcg ? (emit ? pick<true, true>(dim, k) : pick<false, true>(dim, k))
-                        : (emit ? pick<true, false>(dim, k) : pick<false, false>(dim, k));
+int prepare(int dim, int k, int mode, bool gcg, KernelInfo *out) {
+    KernelInfo ki;
+    switch (mode) {
+        case kCount: ki = gcg ? pick<kCount, true>(dim, k) : pick<kCount, false>(dim, k); break;
+        case kPairs: ki = gcg ? pick<kPairs, true>(dim, k) : pick<kPairs, false>(dim, k); break;
+        case kChunkCount: ki = gcg ? pick<kChunkCount, true>(dim, k) : pick<kChunkCount, false>(dim, k); break;
+        case kExact: ki = gcg ? pick<kExact, true>(dim, k) : pick<kExact, false>(dim, k); break;
+        case kRows: if (gcg) ki = pick<kRows, true>(dim, k); break;
+        case kDegree: if (gcg) ki = pick<kDegree, true>(dim, k); break;
+    }
     if (!ki.f) {
-        set_error("join: unsupported dim=%d k=%d%s", dim, k, gcg ? " for the GCG pattern (k in {1, 8, 32})" : "");
+        set_error("join: unsupported dim=%d k=%d mode=%d%s", dim, k, mode,
+                  gcg ? " for the GCG pattern (k in {1, 8, 32})" : " (CSR modes need the GCG pattern)");
         return SJ_EINVAL;
     }
     SJ_CUDA_TRY(cudaFuncSetAttribute(ki.f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ki.smem));
@@ -640,16 +816,16 @@ int prepare(int dim, int k, bool emit, bool gcg, KernelInfo *out) {
 
 }  // namespace
 
-int join_occupancy(int dim, int k, bool emit, bool gcg, int *blocks_per_sm) {
+int join_occupancy(int dim, int k, int mode, bool gcg, int *blocks_per_sm) {
     KernelInfo ki;
-    SJ_TRY(prepare(dim, k, emit, gcg, &ki));
+    SJ_TRY(prepare(dim, k, mode, gcg, &ki));
     SJ_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, ki.f, kJoinThreads, ki.smem));
     return SJ_OK;
 }
 
-int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaStream_t s) {
+int launch_join(const JoinArgs &a, int dim, int k, int mode, int blocks, cudaStream_t s) {
     KernelInfo ki;
-    SJ_TRY(prepare(dim, k, emit, a.gcg != 0, &ki));
+    SJ_TRY(prepare(dim, k, mode, a.gcg != 0, &ki));
     ki.f<<<blocks, kJoinThreads, ki.smem, s>>>(a);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());

@@ -217,6 +217,40 @@ int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *
     }
     return scan_fused(n, LoadArr{in}, StoreArr{out}, s, DoneTotal{d_total});
 }
+namespace {
+template <class In>
+struct LoadArr64 {
+    const In *in;
+    __device__ unsigned long long operator()(uint64_t i) const { return (unsigned long long)in[i]; }
+};
+struct StoreArr64 {
+    uint64_t *out;
+    __device__ void operator()(uint64_t i, unsigned long long ex, unsigned long long) const { out[i] = ex; }
+};
+struct DoneTotal64 {
+    uint64_t *total;
+    __device__ void operator()(unsigned long long t) const {
+        if (total) *total = t;
+    }
+};
+}  // namespace
+
+int scan_exclusive_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s) {
+    if (n == 0) {
+        if (d_total) SJ_CUDA_TRY(cudaMemsetAsync(d_total, 0, sizeof(uint64_t), s));
+        return SJ_OK;
+    }
+    return scan_fused<unsigned long long>(n, LoadArr64<uint64_t>{in}, StoreArr64{out}, s, DoneTotal64{d_total});
+}
+
+int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s) {
+    if (n == 0) {
+        if (d_total) SJ_CUDA_TRY(cudaMemsetAsync(d_total, 0, sizeof(uint64_t), s));
+        return SJ_OK;
+    }
+    return scan_fused<unsigned long long>(n, LoadArr64<uint32_t>{in}, StoreArr64{out}, s, DoneTotal64{d_total});
+}
+
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
                    uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s) {
     return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s);

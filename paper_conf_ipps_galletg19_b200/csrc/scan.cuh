@@ -12,35 +12,38 @@ constexpr int kThreads = 256;
 constexpr int kItems = 8;
 constexpr int kTile = kThreads * kItems;
 // tile status word: [63:62] flag (0 = not ready, 1 = tile aggregate, 2 = inclusive prefix),
-// [31:0] value
+// [61:0] value (u32 scans, and u64 scans of totals below 2^62)
 constexpr unsigned long long kFlagA = 1ull << 62;
 constexpr unsigned long long kFlagP = 2ull << 62;
+constexpr unsigned long long kValMask = (1ull << 62) - 1ull;
 
-__device__ __forceinline__ unsigned warp_incl(unsigned x) {
+template <class T>
+__device__ __forceinline__ T warp_incl(T x) {
     const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        unsigned y = __shfl_up_sync(0xffffffffu, x, o);
+        T y = __shfl_up_sync(0xffffffffu, x, o);
         if (lane >= o) x += y;
     }
     return x;
 }
 
-__device__ __forceinline__ unsigned block_excl(unsigned v, unsigned *total, unsigned *ws) {
+template <class T>
+__device__ __forceinline__ T block_excl(T v, T *total, T *ws) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr int nw = kThreads / 32;
-    unsigned x = warp_incl(v);
+    T x = warp_incl(v);
     __syncthreads();
     if (lane == 31) ws[wid] = x;
     __syncthreads();
     if (wid == 0) {
-        unsigned w = lane < nw ? ws[lane] : 0u;
+        T w = lane < nw ? ws[lane] : T(0);
         w = warp_incl(w);
         if (lane < nw) ws[lane] = w;
     }
     __syncthreads();
     *total = ws[nw - 1];
-    return (wid > 0 ? ws[wid - 1] : 0u) + x - v;
+    return (wid > 0 ? ws[wid - 1] : T(0)) + x - v;
 }
 
 __device__ __forceinline__ void publish(unsigned long long *status, unsigned tile, unsigned long long word) {
@@ -50,14 +53,15 @@ __device__ __forceinline__ void publish(unsigned long long *status, unsigned til
 // Returns the exclusive prefix of `tile` (sum of all earlier tiles).  Called by the whole
 // first warp; the look-back inspects 32 predecessors per step (decoupled look-back with a
 // warp-wide window), so the dependency chain is ~32x shorter than a one-tile walk.
-__device__ __forceinline__ unsigned look_back_warp(unsigned long long *status, unsigned tile, unsigned agg) {
+template <class T>
+__device__ __forceinline__ T look_back_warp(unsigned long long *status, unsigned tile, T agg) {
     const int lane = threadIdx.x & 31;
     if (tile == 0) {
-        if (lane == 0) publish(status, 0, kFlagP | agg);
-        return 0;
+        if (lane == 0) publish(status, 0, kFlagP | (unsigned long long)agg);
+        return T(0);
     }
-    if (lane == 0) publish(status, tile, kFlagA | agg);
-    unsigned prefix = 0;
+    if (lane == 0) publish(status, tile, kFlagA | (unsigned long long)agg);
+    T prefix = 0;
     int j = (int)tile - 1;  // newest predecessor of the window
     for (;;) {
         const int idx = j - lane;
@@ -69,25 +73,26 @@ __device__ __forceinline__ unsigned look_back_warp(unsigned long long *status, u
         }
         const unsigned pmask = __ballot_sync(0xffffffffu, (st & (3ull << 62)) == kFlagP);
         const int first_p = pmask ? __ffs(pmask) - 1 : 32;  // nearest inclusive prefix
-        unsigned v = lane <= first_p ? (unsigned)st : 0u;
+        T v = lane <= first_p ? (T)(st & kValMask) : T(0);
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
         prefix += v;
         if (pmask) break;
         j -= 32;
     }
-    if (lane == 0) publish(status, tile, kFlagP | (unsigned)(prefix + agg));
+    if (lane == 0) publish(status, tile, kFlagP | ((unsigned long long)(prefix + agg) & kValMask));
     return prefix;
 }
 
 // load(i) -> unsigned value of item i (< n); store(i, excl, value) consumes the exclusive
 // prefix; done(total) runs once, in the last tile, after every earlier prefix is known.
-template <class Load, class Store, class Done>
+template <class T, class Load, class Store, class Done>
 __global__ void __launch_bounds__(kThreads) scan_kernel(uint64_t n, Load load, Store store, Done done,
                                                         unsigned long long *status, unsigned *tile_ctr) {
-    __shared__ unsigned s_tile, s_prefix;
-    __shared__ unsigned ws[32];
-    __shared__ unsigned vals[kTile];
+    __shared__ unsigned s_tile;
+    __shared__ T s_prefix;
+    __shared__ T ws[32];
+    __shared__ T vals[kTile];
     if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);  // dynamic tile order
     __syncthreads();
     const unsigned tile = s_tile;
@@ -95,26 +100,26 @@ __global__ void __launch_bounds__(kThreads) scan_kernel(uint64_t n, Load load, S
 #pragma unroll
     for (int it = 0; it < kItems; ++it) {
         const uint64_t i = base + (uint64_t)it * kThreads + threadIdx.x;
-        vals[it * kThreads + threadIdx.x] = i < n ? load(i) : 0u;
+        vals[it * kThreads + threadIdx.x] = i < n ? (T)load(i) : T(0);
     }
     __syncthreads();
-    unsigned v[kItems], s = 0;
+    T v[kItems], s = 0;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
         v[j] = vals[threadIdx.x * kItems + j];
         s += v[j];
     }
-    unsigned agg;
-    unsigned ex = block_excl(s, &agg, ws);
+    T agg;
+    T ex = block_excl<T>(s, &agg, ws);
     if (threadIdx.x < 32) {
-        const unsigned pre = look_back_warp(status, tile, agg);
+        const T pre = look_back_warp<T>(status, tile, agg);
         if (threadIdx.x == 0) s_prefix = pre;
     }
     __syncthreads();
     ex += s_prefix;
     // per-item exclusive prefixes back to shared memory (blocked), then the stores run in the
     // same striped (coalesced) order as the loads
-    __shared__ unsigned exs[kTile];
+    __shared__ T exs[kTile];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
         exs[threadIdx.x * kItems + j] = ex;
@@ -133,11 +138,13 @@ __global__ void __launch_bounds__(kThreads) scan_kernel(uint64_t n, Load load, S
 }  // namespace scan_detail
 
 struct NoDone {
-    __device__ void operator()(unsigned) const {}
+    template <class T>
+    __device__ void operator()(T) const {}
 };
 
-// Exclusive scan of load(0..n-1) in one launch.  Temporaries from the stream-ordered pool.
-template <class Load, class Store, class Done = NoDone>
+// Exclusive scan of load(0..n-1) in one launch (value type T: unsigned, or unsigned long
+// long for totals below 2^62).  Temporaries from the stream-ordered pool.
+template <class T = unsigned, class Load, class Store, class Done = NoDone>
 int scan_fused(uint64_t n, Load load, Store store, cudaStream_t s, Done done = Done()) {
     using namespace scan_detail;
     if (n == 0) return SJ_OK;
@@ -146,7 +153,7 @@ int scan_fused(uint64_t n, Load load, Store store, cudaStream_t s, Done done = D
     SJ_TRY(dev_alloc(reinterpret_cast<void **>(&status), nt * sizeof(unsigned long long) + 64, s));
     unsigned *ctr = reinterpret_cast<unsigned *>(status + nt);
     SJ_CUDA_TRY(cudaMemsetAsync(status, 0, nt * sizeof(unsigned long long) + 64, s));
-    scan_kernel<<<(unsigned)nt, kThreads, 0, s>>>(n, load, store, done, status, ctr);
+    scan_kernel<T><<<(unsigned)nt, kThreads, 0, s>>>(n, load, store, done, status, ctr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     dev_free(status, s);

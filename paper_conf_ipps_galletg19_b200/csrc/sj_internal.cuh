@@ -70,6 +70,12 @@ void pinned_release(void *p);
 // Exclusive scan of u32 (out may alias in).  total (device, optional) receives the sum.
 int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s);
 
+// Exclusive scans with 64-bit sums (pair counts, CSR row offsets; totals < 2^62).  out may
+// alias in; d_total (device, optional) receives the sum, e.g. out + n for an (n+1)-entry
+// offset array.
+int scan_exclusive_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s);
+int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uint64_t *d_total, cudaStream_t s);
+
 // Stable LSD radix sort of (key, value) pairs on the low `bits` bits of the keys.
 // Hand-written: per 8-bit pass a tile histogram, a digit-major scan and a stable
 // scatter through shared memory (DESIGN.md §4 a4).  Buffers are ping-ponged; the
@@ -141,12 +147,24 @@ struct JoinArgs {
     unsigned long long *emit_ctr; // pairs emitted (may exceed out_cap -> overflow)
     unsigned long long out_cap;   // capacity of out in pairs
     unsigned long long *calcs;    // instrumented distance calculations, or nullptr
+    // exact two-pass sizing
+    unsigned long long *vcount;       // kChunkCount: pairs of virtual chunk v (written per chunk)
+    const unsigned long long *voff;   // kExact: pair offset of virtual chunk v (exclusive scan of vcount);
+    unsigned long long out_base;      //   out holds pairs [out_base, ..)
+    // device CSR (GCG pattern: every query owns its row)
+    uint32_t *qdeg;                   // kDegree: degree by input id
+    const unsigned long long *row_off; // kRows: row start by input id
+    uint32_t *nbrs;                   // kRows: neighbour ids
 };
 
-// Launch the join kernel for dim/k; emit=false counts pairs only.
-int launch_join(const JoinArgs &a, int dim, int k, bool emit, int blocks, cudaStream_t s);
+// Join kernel modes: count pairs; emit the pair list; fill CSR rows; count CSR degrees;
+// count pairs per WorkQueue chunk (exact sizing pass 1); emit at chunk offsets (pass 2).
+enum JoinMode : int { kCount = 0, kPairs = 1, kRows = 2, kDegree = 3, kChunkCount = 4, kExact = 5 };
+
+// Launch the join kernel for dim/k/mode (kRows / kDegree need the GCG pattern).
+int launch_join(const JoinArgs &a, int dim, int k, int mode, int blocks, cudaStream_t s);
 // Max resident CTAs per SM of the join kernel configuration.
-int join_occupancy(int dim, int k, bool emit, bool gcg, int *blocks_per_sm);
+int join_occupancy(int dim, int k, int mode, bool gcg, int *blocks_per_sm);
 constexpr int kJoinThreads = 256;
 
 // --------------------------------------------------------------------------- misc kernels

@@ -113,6 +113,8 @@ constexpr int kMaxStreams = 8;
 
 struct Job {
     uint64_t v0, v1;  // virtual WorkQueue chunk range [v0, v1) of this handle's slice
+    uint64_t base = 0;               // exact sizing: pair offset of chunk v0 in the whole join
+    uint64_t expect = UINT64_MAX;    // exact sizing: the batch's pairs (UINT64_MAX: estimated)
     int slot = -1;
     bool launched = false, complete = false;
     uint64_t cnt = 0, consumed = 0;
@@ -147,7 +149,11 @@ struct sj_handle {
     int count_calcs = 0;
     int blocks_per_sm = 0;
     int fast_path = 1;
+    int exact = 0;
     int rank = 0, world = 1;
+
+    uint64_t *d_voff = nullptr;  // exact sizing: per-chunk pairs -> offsets, [V+1]
+    uint64_t voff_cap = 0;
 
     unsigned long long *d_ctr = nullptr;  // [0]=emit [1]=head [2]=calcs [3..] spare
     uint64_t *mail = nullptr;             // pinned host mailbox [64]
@@ -325,17 +331,19 @@ JoinArgs base_args(const sj_handle *h) {
     return a;
 }
 
-int join_blocks(const sj_handle *h, bool emit, int *blocks) {
+int join_blocks(const sj_handle *h, int mode, int *blocks) {
     int occ = 0;
-    SJ_TRY(join_occupancy(h->ix.dim, h->k, emit, h->ix.pattern == SJ_PATTERN_GCG, &occ));
+    SJ_TRY(join_occupancy(h->ix.dim, h->k, mode, h->ix.pattern == SJ_PATTERN_GCG, &occ));
     if (h->blocks_per_sm > 0 && h->blocks_per_sm < occ) occ = h->blocks_per_sm;
     if (occ < 1) occ = 1;
     *blocks = occ * h->num_sms;
     return SJ_OK;
 }
 
-// Count-only join over virtual range [v0, v1) on the main stream.  Synchronous.
-int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms) {
+// Count-only join over virtual range [v0, v1) on the main stream.  Synchronous.  With
+// vcount, every chunk's pairs are recorded and scanned in place into chunk offsets
+// (exact sizing, pass 1): vcount[V] receives the total.
+int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms, uint64_t *vcount = nullptr) {
     cudaStream_t s = h->s_main;
     SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
     JoinArgs a = base_args(h);
@@ -346,10 +354,13 @@ int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *
     a.emit_ctr = h->d_ctr;
     a.out_cap = 0;
     a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+    a.vcount = reinterpret_cast<unsigned long long *>(vcount);
+    const int mode = vcount ? kChunkCount : kCount;
     int blocks;
-    SJ_TRY(join_blocks(h, false, &blocks));
+    SJ_TRY(join_blocks(h, mode, &blocks));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
-    if (v1 > v0) SJ_TRY(launch_join(a, h->ix.dim, h->k, false, blocks, s));
+    if (v1 > v0) SJ_TRY(launch_join(a, h->ix.dim, h->k, mode, blocks, s));
+    if (vcount) SJ_TRY(scan_exclusive_u64(vcount + v0, vcount + v0, v1 - v0, vcount + v1, s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
     SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
@@ -362,7 +373,7 @@ int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *
 // ------------------------------------------------------------------ staged batches
 int launch_job(sj_handle *h, Job &j, int slot_idx) {
     Slot &s = h->slots[slot_idx];
-    SJ_TRY(slot_buffer(h, s, h->batch_pairs));
+    SJ_TRY(slot_buffer(h, s, j.expect != UINT64_MAX ? std::max<uint64_t>(h->batch_pairs, j.expect) : h->batch_pairs));
     SJ_CUDA_TRY(cudaMemsetAsync(s.d_ctr, 0, 4 * sizeof(unsigned long long), s.stream));
     JoinArgs a = base_args(h);
     a.head = s.d_ctr + 1;  // zeroed above
@@ -372,10 +383,15 @@ int launch_job(sj_handle *h, Job &j, int slot_idx) {
     a.emit_ctr = s.d_ctr;
     a.out_cap = s.cap;
     a.calcs = h->count_calcs ? s.d_ctr + 2 : nullptr;
+    const bool exact = j.expect != UINT64_MAX;
+    if (exact) {  // exact sizing: every chunk writes at its own offset
+        a.voff = reinterpret_cast<const unsigned long long *>(h->d_voff);
+        a.out_base = j.base;
+    }
     int blocks;
-    SJ_TRY(join_blocks(h, true, &blocks));
+    SJ_TRY(join_blocks(h, exact ? kExact : kPairs, &blocks));
     SJ_CUDA_TRY(cudaEventRecord(s.ev_start, s.stream));
-    SJ_TRY(launch_join(a, h->ix.dim, h->k, true, blocks, s.stream));
+    SJ_TRY(launch_join(a, h->ix.dim, h->k, exact ? kExact : kPairs, blocks, s.stream));
     SJ_CUDA_TRY(cudaEventRecord(s.ev_stop, s.stream));
     SJ_CUDA_TRY(cudaMemcpyAsync(h->mail + 8 + 4 * slot_idx, s.d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost,
                                 s.stream));
@@ -422,6 +438,12 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
                 fprintf(stderr, "[sj] batch chunks [%llu, %llu) pairs %llu  %.3f ms  %.1f GB/s\n",
                         (unsigned long long)j.v0, (unsigned long long)j.v1, (unsigned long long)j.cnt, ms,
                         j.cnt * 8.0 / (ms * 1e6));
+            if (j.expect != UINT64_MAX && j.cnt != j.expect) {
+                set_error("sj_self_join: exact sizing mismatch in chunks [%llu, %llu): counted %llu, emitted %llu",
+                          (unsigned long long)j.v0, (unsigned long long)j.v1, (unsigned long long)j.expect,
+                          (unsigned long long)j.cnt);
+                return SJ_ECUDA;
+            }
             if (j.cnt > s.cap) {
                 // overflow (estimate too low): split the range, or grow the buffer if it is one chunk
                 h->st.retries++;
@@ -483,6 +505,120 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
     return SJ_MORE;
 }
 
+// One persistent launch over the slice's chunks [v0, v1) writing the caller's device buffer in
+// place (no staging, no D2D copy).  *emitted = the pairs the kernel produced (> cap: overflow,
+// only the first cap were written).  exact: chunk offsets from h->d_voff.
+int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_t v1, bool exact,
+                 uint64_t *emitted) {
+    cudaStream_t s = h->s_main;
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    JoinArgs a = base_args(h);
+    a.head = h->d_ctr + 1;  // zeroed above
+    a.v_begin = v0;
+    a.v_end = v1;
+    a.out = out;
+    a.emit_ctr = h->d_ctr;
+    a.out_cap = cap;
+    a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+    if (exact) {
+        a.voff = reinterpret_cast<const unsigned long long *>(h->d_voff);
+        a.out_base = 0;
+    }
+    const int mode = exact ? kExact : kPairs;
+    int blocks;
+    SJ_TRY(join_blocks(h, mode, &blocks));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
+    if (v1 > v0) SJ_TRY(launch_join(a, h->ix.dim, h->k, mode, blocks, s));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    float ms = 0;
+    SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
+    h->st.join_launches = 1;
+    h->st.batches = 1;
+    h->st.ms_join = h->st.ms_join_sum = ms;
+    *emitted = h->mail[0];
+    return SJ_OK;
+}
+
+int finish_in_place(sj_handle *h, uint64_t total, uint64_t *count) {
+    if (h->count_calcs) h->st.calcs_measured = h->mail[2];
+    h->st.pairs = total;
+    h->st.fast_path = 1;
+    *count = total;
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_b, h->s_main));
+    SJ_CUDA_TRY(cudaEventSynchronize(h->ev_b));
+    float tot = 0;
+    SJ_CUDA_TRY(cudaEventElapsedTime(&tot, h->ev_a, h->ev_b));
+    h->st.ms_total = tot;
+    h->state = 0;
+    return SJ_OK;
+}
+
+// Staged path: the queued jobs run round-robin over `streams` streams, each into its
+// own b_s buffer, and are copied out in batch order.
+int start_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
+    for (int i = 0; i < h->streams; ++i) SJ_TRY(slot_init(h, i));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_c, h->s_main));
+    for (int i = 0; i < h->streams; ++i) SJ_CUDA_TRY(cudaStreamWaitEvent(h->slots[i].stream, h->ev_c, 0));
+    h->st.batches = (uint32_t)h->jobs.size();
+    h->state = 1;
+    return continue_staged(h, out, cap, count);
+}
+
+// Exact two-pass sizing (SJ_OPT_EXACT): pass 1 counts every
+// chunk's pairs and scans them into chunk offsets; batches are cut at exact sizes <= b_s
+// (a single chunk larger than b_s gets a batch -- and buffer -- of its own); pass 2 writes
+// each chunk at its offset.  No estimator, no overflow retry, deterministic output order.
+int start_exact(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count, bool dev_out) {
+    const uint64_t V = slice_chunks(h);
+    if (h->voff_cap < V + 1) {
+        dev_free(h->d_voff, h->s_main);
+        h->d_voff = nullptr;
+        h->voff_cap = 0;
+        SJ_TRY(dev_alloc_t(&h->d_voff, V + 1, h->s_main));
+        h->voff_cap = V + 1;
+    }
+    uint64_t total = 0;
+    float ms = 0;
+    SJ_TRY(count_range(h, 0, V, &total, &ms, h->d_voff));
+    h->st.ms_estimate = ms;
+    h->st.est_pairs = total;
+    h->st.calcs_measured = 0;
+    if (dev_out && h->fast_path && total <= cap) {
+        uint64_t emitted = 0;
+        SJ_TRY(run_in_place(h, out, cap, 0, V, true, &emitted));
+        if (emitted != total) {
+            set_error("sj_self_join: exact sizing mismatch: counted %llu pairs, emitted %llu",
+                      (unsigned long long)total, (unsigned long long)emitted);
+            return SJ_ECUDA;
+        }
+        return finish_in_place(h, total, count);
+    }
+    std::vector<uint64_t> off(V + 1);
+    SJ_CUDA_TRY(cudaMemcpyAsync(off.data(), h->d_voff, (V + 1) * sizeof(uint64_t), cudaMemcpyDeviceToHost,
+                                h->s_main));
+    SJ_CUDA_TRY(cudaStreamSynchronize(h->s_main));
+    if (off[V] != total) {
+        set_error("sj_self_join: exact sizing: scan total %llu != counter %llu", (unsigned long long)off[V],
+                  (unsigned long long)total);
+        return SJ_ECUDA;
+    }
+    for (uint64_t v = 0; v < V;) {  // greedy: the longest run of chunks with <= b_s pairs
+        uint64_t e = (uint64_t)(std::upper_bound(off.begin() + (long)v + 1, off.end(), off[v] + h->batch_pairs) -
+                                off.begin()) - 1;
+        if (e <= v) e = v + 1;
+        Job j;
+        j.v0 = v;
+        j.v1 = e;
+        j.base = off[v];
+        j.expect = off[e] - off[v];
+        h->jobs.push_back(j);
+        v = e;
+    }
+    return start_staged(h, out, cap, count);
+}
+
 int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     SJ_TRY(ensure_device(h));
     // a new join: reset per-join statistics
@@ -519,6 +655,13 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         return SJ_OK;
     }
 
+    const bool dev_out = is_device_ptr(out, h->device);
+    if (dev_out && (reinterpret_cast<uintptr_t>(out) & 15u)) {
+        set_error("sj_self_join: device out_pairs must be 16-byte aligned");
+        return SJ_EINVAL;
+    }
+    if (h->exact) return start_exact(h, out, cap, count, dev_out);
+
     // a9: batch estimator -- count-only join over the first sample_ppm of D'
     uint64_t sch = (nch * (uint64_t)h->sample_ppm + 999999ull) / 1000000ull;
     if (sch < 1) sch = 1;
@@ -536,79 +679,170 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     if (nb < 1) nb = 1;
     if (nb > nch && nch) nb = nch;
 
-    const bool dev_out = is_device_ptr(out, h->device);
-    if (dev_out && (reinterpret_cast<uintptr_t>(out) & 15u)) {
-        set_error("sj_self_join: device out_pairs must be 16-byte aligned");
-        return SJ_EINVAL;
-    }
     // The sample's own pairs are part of the result, so spairs is a strict lower bound of the
     // total; the extrapolated estimate is NOT (the first 1% of D' is the heaviest part)
     // and is only used to size the staged batches.
     if (dev_out && h->fast_path && spairs <= cap) {
-        // Fast path: the caller's HBM buffer is the result buffer; one persistent launch
-        // over the whole slice writes it in place (no staging, no D2D copy).  Overflow is
-        // detected from the counter and falls back to the staged path.
-        cudaStream_t s = h->s_main;
+        // Fast path: the caller's HBM buffer is the result buffer.  Overflow is detected from
+        // the counter and falls back to the staged path.
         unsigned long long dv0 = 0, dv1 = V;
         if (const char *r = getenv("SJ_DEBUG_VRANGE")) {  // diagnostics: join a sub-range only
             sscanf(r, "%llu,%llu", &dv0, &dv1);
             dv1 = std::min<unsigned long long>(dv1, V);
         }
-        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
-        JoinArgs a = base_args(h);
-        a.head = h->d_ctr + 1;  // zeroed above
-        a.v_begin = dv0;
-        a.v_end = dv1;
-        a.out = out;
-        a.emit_ctr = h->d_ctr;
-        a.out_cap = cap;
-        a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
-        int blocks;
-        SJ_TRY(join_blocks(h, true, &blocks));
-        SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
-        if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, true, blocks, s));
-        SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
-        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
-        SJ_CUDA_TRY(cudaStreamSynchronize(s));
-        float ms = 0;
-        SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
-        h->st.join_launches = 1;
-        h->st.batches = 1;
-        h->st.ms_join = h->st.ms_join_sum = ms;
-        const uint64_t total = h->mail[0];
+        uint64_t total = 0;
+        SJ_TRY(run_in_place(h, out, cap, dv0, dv1, false, &total));
         debug_mark("join: fast path");
-        if (total <= cap) {
-            if (h->count_calcs) h->st.calcs_measured = h->mail[2];
-            h->st.pairs = total;
-            h->st.fast_path = 1;
-            *count = total;
-            SJ_CUDA_TRY(cudaEventRecord(h->ev_b, s));
-            SJ_CUDA_TRY(cudaEventSynchronize(h->ev_b));
-            float tot = 0;
-            SJ_CUDA_TRY(cudaEventElapsedTime(&tot, h->ev_a, h->ev_b));
-            h->st.ms_total = tot;
-            h->state = 0;
-            return SJ_OK;
-        }
+        if (total <= cap) return finish_in_place(h, total, count);
         h->st.retries++;  // did not fit: fall through to the staged path
         h->st.ms_join = h->st.ms_join_sum = 0;
         h->st.join_launches = 0;
     }
 
-    // Staged path: nb batches = contiguous ranges of D' (reading c14), round-robin
-    // over `streams` streams, each into its own b_s buffer, copied out in batch order.
-    for (int i = 0; i < h->streams; ++i) SJ_TRY(slot_init(h, i));
-    SJ_CUDA_TRY(cudaEventRecord(h->ev_c, h->s_main));
-    for (int i = 0; i < h->streams; ++i) SJ_CUDA_TRY(cudaStreamWaitEvent(h->slots[i].stream, h->ev_c, 0));
+    // Staged path: nb batches = contiguous ranges of D' (reading c14).
     for (uint64_t b = 0; b < nb; ++b) {
         Job j;
         j.v0 = nch * b / nb;
         j.v1 = nch * (b + 1) / nb;
         if (j.v1 > j.v0) h->jobs.push_back(j);
     }
-    h->st.batches = (uint32_t)h->jobs.size();
-    h->state = 1;
-    return continue_staged(h, out, cap, count);
+    return start_staged(h, out, cap, count);
+}
+
+// Device CSR (sj_neighbor_csr): degrees (GCG row owners, no atomics) -> exclusive scan ->
+// row fill.  Temporaries come from the stream-ordered pool.
+int neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, uint64_t *total) {
+    if (h->ix.pattern != SJ_PATTERN_GCG) {
+        set_error("sj_neighbor_csr: needs a handle created with SJ_PATTERN_GCG (every query owns its row)");
+        return SJ_EINVAL;
+    }
+    if (h->world != 1) {
+        set_error("sj_neighbor_csr: needs the whole queue (sj_set_slice world 1)");
+        return SJ_EINVAL;
+    }
+    if (h->state == 1) {
+        set_error("sj_neighbor_csr: a staged sj_self_join is pending (SJ_MORE); finish it first");
+        return SJ_EINVAL;
+    }
+    SJ_TRY(ensure_device(h));
+    cudaStream_t s = h->s_main;
+    const uint64_t n = h->ix.n, V = slice_chunks(h);
+    h->st.pairs = 0;
+    h->st.calcs_measured = 0;
+    h->st.batches = 1;
+    h->st.retries = 0;
+    h->st.join_launches = 0;
+    h->st.ms_join = h->st.ms_join_sum = h->st.ms_estimate = h->st.ms_transfer = h->st.ms_total = 0;
+    h->st.fast_path = 0;
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_a, s));
+    const bool off_dev = row_off && is_device_ptr(row_off, h->device) && !(reinterpret_cast<uintptr_t>(row_off) & 7u);
+    uint64_t *d_off = off_dev ? row_off : nullptr;
+    uint32_t *d_deg = nullptr, *d_nbrs = nullptr;
+    int blocks;
+    SJ_TRY(join_blocks(h, kDegree, &blocks));
+    auto cleanup = [&]() {
+        dev_free(d_deg, s);
+        if (!off_dev) dev_free(d_off, s);
+        if (d_nbrs != nbrs) dev_free(d_nbrs, s);
+    };
+    int rc = dev_alloc_t(&d_deg, n, s);
+    if (rc == SJ_OK && !off_dev) rc = dev_alloc_t(&d_off, n + 1, s);
+    if (rc < 0) {
+        cleanup();
+        return rc;
+    }
+    // pass 1: degrees
+    JoinArgs a = base_args(h);
+    a.head = h->d_ctr + 1;
+    a.emit_ctr = h->d_ctr;
+    a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+    a.v_begin = 0;
+    a.v_end = V;
+    a.qdeg = d_deg;
+    rc = [&]() -> int {
+        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
+        if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, kDegree, blocks, s));
+        SJ_TRY(scan_exclusive_u32_to_u64(d_deg, d_off, n, d_off + n, s));
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, d_off + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail + 1, h->d_ctr, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        if (row_off && !off_dev)
+            SJ_CUDA_TRY(cudaMemcpyAsync(row_off, d_off, (n + 1) * sizeof(uint64_t), cudaMemcpyDefault, s));
+        SJ_CUDA_TRY(cudaStreamSynchronize(s));
+        float ms = 0;
+        SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
+        h->st.ms_estimate = ms;
+        h->st.join_launches = 1;
+        *total = h->mail[0];
+        h->st.est_pairs = h->mail[0];
+        if (h->mail[0] != h->mail[1]) {
+            set_error("sj_neighbor_csr: degree sum %llu != counter %llu", (unsigned long long)h->mail[0],
+                      (unsigned long long)h->mail[1]);
+            return SJ_ECUDA;
+        }
+        return SJ_OK;
+    }();
+    if (rc < 0 || !nbrs) {
+        cleanup();
+        return rc;
+    }
+    const uint64_t tot = *total;
+    if (cap < tot) {
+        cleanup();
+        set_error("sj_neighbor_csr: cap %llu < %llu neighbour entries", (unsigned long long)cap,
+                  (unsigned long long)tot);
+        return SJ_EINVAL;
+    }
+    // pass 2: row fill
+    const bool nb_dev = is_device_ptr(nbrs, h->device) && !(reinterpret_cast<uintptr_t>(nbrs) & 3u);
+    d_nbrs = nb_dev ? nbrs : nullptr;
+    if (!nb_dev) {
+        rc = dev_alloc_t(&d_nbrs, tot, s);
+        if (rc < 0) {
+            cleanup();
+            return rc;
+        }
+    }
+    rc = [&]() -> int {
+        JoinArgs b = base_args(h);
+        b.head = h->d_ctr + 1;
+        b.emit_ctr = h->d_ctr;
+        b.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+        b.v_begin = 0;
+        b.v_end = V;
+        b.row_off = reinterpret_cast<const unsigned long long *>(d_off);
+        b.nbrs = d_nbrs;
+        int fb;
+        SJ_TRY(join_blocks(h, kRows, &fb));
+        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
+        if (V) SJ_TRY(launch_join(b, h->ix.dim, h->k, kRows, fb, s));
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        if (!nb_dev && tot)
+            SJ_CUDA_TRY(cudaMemcpyAsync(nbrs, d_nbrs, tot * sizeof(uint32_t), cudaMemcpyDefault, s));
+        SJ_CUDA_TRY(cudaStreamSynchronize(s));
+        float ms = 0;
+        SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
+        h->st.ms_join = h->st.ms_join_sum = ms;
+        h->st.join_launches = 2;
+        if (h->count_calcs) h->st.calcs_measured = h->mail[2];
+        if (h->mail[0] != tot) {
+            set_error("sj_neighbor_csr: filled %llu entries, counted %llu", (unsigned long long)h->mail[0],
+                      (unsigned long long)tot);
+            return SJ_ECUDA;
+        }
+        h->st.pairs = tot;
+        SJ_CUDA_TRY(cudaEventRecord(h->ev_b, s));
+        SJ_CUDA_TRY(cudaEventSynchronize(h->ev_b));
+        float all = 0;
+        SJ_CUDA_TRY(cudaEventElapsedTime(&all, h->ev_a, h->ev_b));
+        h->st.ms_total = all;
+        return SJ_OK;
+    }();
+    cleanup();
+    return rc;
 }
 
 }  // namespace
@@ -740,11 +974,26 @@ int sj_self_join(sj_handle *h, uint32_t *out_pairs, uint64_t cap, uint64_t *coun
     return fail(h, rc);
 }
 
+int sj_neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, uint64_t *total) {
+    if (!h || !total || ((nbrs == nullptr) != (cap == 0))) {
+        set_error("sj_neighbor_csr: NULL handle/total, or nbrs and cap not both set / both NULL-0");
+        return SJ_EINVAL;
+    }
+    *total = 0;
+    if (h->state < 0) {
+        set_error("sj_neighbor_csr: handle is in the error state");
+        return SJ_ESTATE;
+    }
+    const int rc = neighbor_csr(h, row_off, nbrs, cap, total);
+    return rc == SJ_EINVAL ? rc : fail(h, rc);
+}
+
 void sj_destroy(sj_handle *h) {
     if (!h) return;
     debug_mark("destroy: enter");
     cudaSetDevice(h->device);
     slots_release(h);
+    if (h->s_main) dev_free(h->d_voff, h->s_main);
     if (h->s_main && h->owns_index) free_index(h->ix, h->s_main);  // stream-ordered frees
     if (!core_release(h)) {
         if (h->s_main) {
@@ -796,6 +1045,9 @@ int sj_set_option(sj_handle *h, int opt, int64_t v) {
             return SJ_OK;
         case SJ_OPT_FAST_PATH:
             h->fast_path = v ? 1 : 0;
+            return SJ_OK;
+        case SJ_OPT_EXACT:
+            h->exact = v ? 1 : 0;
             return SJ_OK;
 
     }
