@@ -285,7 +285,7 @@ static uint64_t grid_query(const grid_t *g, uint64_t i, uint32_t *cols, uint64_t
     const int dim = g->dim;
     const int64_t *ci = g->coord + i * dim;
     const double *pi = g->pts + i * dim;
-    int64_t nb[8];
+    int64_t nb[8] = {0};
     int off[8];
     for (int d = 0; d < dim; ++d) off[d] = -1;
     uint64_t c = 0, ev = 0;
