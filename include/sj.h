@@ -59,12 +59,20 @@ enum sj_option {
     SJ_OPT_BLOCKS_PER_SM = 7,  /* persistent-grid CTAs per SM; 0 = occupancy maximum (default)           */
     SJ_OPT_FAST_PATH = 8,      /* 1 = device output written in place when it fits (default); 0 = always
                                   stage per batch (the paper's scheme)                             */
-    SJ_OPT_EXACT = 9           /* 1 = exact two-pass sizing: a count pass records every
+    SJ_OPT_EXACT = 9,          /* 1 = exact two-pass sizing: a count pass records every
                                   WorkQueue chunk's pairs, their scan gives each chunk its output slots,
                                   batches are cut at exact sizes <= b_s and the fill pass writes each
                                   chunk at its own offset -- no estimator, no overflow retries, and the
                                   output ORDER is deterministic.  0 = the paper's 1% estimator (P:71,
                                   P:200) with atomic placement (default)                                 */
+    SJ_OPT_QUEUE = 10          /* 1 = WorkQueue: warps dequeue D' chunks with an atomic
+                                  counter, batches are contiguous ranges of D', the estimator samples
+                                  the first 1% of D' (default).  0 = SortByWL only
+                                  (P:187-192): warp w statically takes chunks w, w + #warps, ... of D'
+                                  (no atomics), staged batches are the strided D'_l = {chunk v :
+                                  v mod nbBatches = l} (Fig. 1) and the estimator samples
+                                  every (1/1%)-th chunk of the whole queue.  The pair set is
+                                  the same either way                                                    */
 };
 
 /* Cell access patterns (sj_create_ex).  The paper's variants, Table II:
@@ -213,6 +221,15 @@ int sj_forward_offsets(int dim, int8_t *out, uint64_t cap);
  * writes them ascending into out (if out != NULL and cap is large enough) and
  * returns their number, or a negative sj_status. */
 int64_t sj_slice_chunks(uint64_t n_chunks, int rank, int world, uint32_t *out, uint64_t cap);
+
+/* Virtual WorkQueue chunks of staged batch `batch` out of `n_batches` over a slice of
+ * n_chunks chunks: queue = 1 (WorkQueue) -> the contiguous range
+ * [n_chunks*batch/n_batches, n_chunks*(batch+1)/n_batches) (reading c14); queue = 0
+ * (SortByWL only) -> the strided D'_l: batch, batch + n_batches, ... (Fig. 1).  Writes them
+ * ascending into out (if out != NULL and cap is large enough) and returns their number, or
+ * SJ_EINVAL.  sj_self_join cuts its estimated batches with exactly this rule. */
+int64_t sj_batch_chunks(uint64_t n_chunks, uint64_t n_batches, uint64_t batch, int queue, uint32_t *out,
+                        uint64_t cap);
 
 /* ---- diagnostics (GPU microbenchmarks for the roofline denominators) ------ */
 

@@ -16,7 +16,7 @@ SJ_ORDER_WORKLOAD, SJ_ORDER_CELL, SJ_ORDER_INPUT = 0, 1, 2
 PATTERNS = {"lid_unicomp": SJ_PATTERN_LID_UNICOMP, "gcg": SJ_PATTERN_GCG, "unicomp": SJ_PATTERN_UNICOMP}
 ORDERS = {"workload": SJ_ORDER_WORKLOAD, "cell": SJ_ORDER_CELL, "input": SJ_ORDER_INPUT}
 (SJ_OPT_K, SJ_OPT_BATCH_PAIRS, SJ_OPT_STREAMS, SJ_OPT_SAMPLE_PPM, SJ_OPT_GRAB, SJ_OPT_COUNT_CALCS,
- SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH, SJ_OPT_EXACT) = range(1, 10)
+ SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH, SJ_OPT_EXACT, SJ_OPT_QUEUE) = range(1, 11)
 _NAMES = {0: "SJ_OK", 1: "SJ_MORE", -1: "SJ_EINVAL", -2: "SJ_ENOMEM", -3: "SJ_ECUDA", -4: "SJ_EGRID",
           -5: "SJ_ESTATE"}
 
@@ -68,6 +68,7 @@ _sig = {
     "sj_create_from_index": (_vp, [_vp, _u64]),
     "sj_forward_offsets": (_int, [_int, _vp, _u64]),
     "sj_slice_chunks": (_i64, [_u64, _int, _int, _vp, _u64]),
+    "sj_batch_chunks": (_i64, [_u64, _u64, _u64, _int, _vp, _u64]),
     "sj_measure_fp64": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
     "sj_measure_atomics": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
     "sj_neighbor_csr": (_int, [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]),
@@ -221,6 +222,15 @@ def sj_slice_chunks(n_chunks: int, rank: int, world: int):
     return out[:cnt]
 
 
+def sj_batch_chunks(n_chunks: int, n_batches: int, batch: int, queue: int = 1):
+    import numpy as np
+
+    cnt = _check(_lib.sj_batch_chunks(int(n_chunks), int(n_batches), int(batch), int(queue), None, 0))
+    out = np.zeros(max(cnt, 1), dtype=np.uint32)
+    _check(_lib.sj_batch_chunks(int(n_chunks), int(n_batches), int(batch), int(queue), out.ctypes.data, out.size))
+    return out[:cnt]
+
+
 def sj_measure_fp64():
     r, ms = _dbl(0), _dbl(0)
     _check(_lib.sj_measure_fp64(ctypes.byref(r), ctypes.byref(ms)))
@@ -257,7 +267,8 @@ class Handle:
 
     _OPTS = {"k": SJ_OPT_K, "batch_pairs": SJ_OPT_BATCH_PAIRS, "streams": SJ_OPT_STREAMS,
              "sample_ppm": SJ_OPT_SAMPLE_PPM, "grab": SJ_OPT_GRAB, "count_calcs": SJ_OPT_COUNT_CALCS,
-             "blocks_per_sm": SJ_OPT_BLOCKS_PER_SM, "fast_path": SJ_OPT_FAST_PATH, "exact": SJ_OPT_EXACT}
+             "blocks_per_sm": SJ_OPT_BLOCKS_PER_SM, "fast_path": SJ_OPT_FAST_PATH, "exact": SJ_OPT_EXACT,
+             "queue": SJ_OPT_QUEUE}
 
     def set_option(self, name, value) -> None:
         sj_set_option(self.h, self._OPTS[name] if isinstance(name, str) else name, int(value))

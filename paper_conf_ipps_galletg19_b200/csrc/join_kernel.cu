@@ -47,6 +47,14 @@ constexpr int kBufHitsHi = SJ_BUF_HI;
 // A cell segment of >= 2 queries is tiled when its forward list has at least this many
 // candidates (6-D: ~1300 per cell of ~4 points), so staging pays for itself.
 constexpr unsigned kTileMinCand = 128;
+// Column emission buffers (1-D..3-D pair modes, see flush_cols): kColRows hits per lane,
+// rows kColPitch = 33 entries apart so that reading one column down its rows (the flush)
+// walks the shared-memory banks instead of hitting one bank pair 32 times.
+constexpr int kColRows = 16;
+constexpr int kColPitch = 33;
+#ifndef SJ_COLS
+#define SJ_COLS 0  // measured slower than the ballot-ranked buffer on B200 (C5 join +40 %)
+#endif
 
 template <int DIM>
 struct PointPad {
@@ -81,8 +89,11 @@ struct WarpSmem {
     uint2 runs_s[(DIM >= 4 && DIM <= 6) ? 128 : 1];
     // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
     // and the smaller footprint buys occupancy)
-    alignas(16) uint2 buf[Mode<MODE>::pairs ? BufCap<DIM>::value : 2];
-    unsigned long long wcur;  // kPairs, exact sizing: next output slot of the current chunk
+    alignas(16) uint2 buf[Mode<MODE>::pairs ? ((SJ_COLS && DIM <= 3) ? kColRows * kColPitch : BufCap<DIM>::value) : 2];
+    // kExact: next output slot of the current chunk; kPairs: nonzero once a flush of this warp
+    // found the output full (the warp stops dequeuing: the caller re-runs the join staged)
+    unsigned long long wcur;
+    unsigned snext;  // SortByWL only (static assignment): this warp's next chunk index
     // kRows: the segment's per-query row cursors; kDegree: their running neighbour counts
     unsigned long long qcur[(MODE == kRows || MODE == kDegree) ? 32 : 1];
 };
@@ -185,6 +196,8 @@ __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs
         if (EXACT) {
             base = *wcur;
             *wcur = base + kPer * (unsigned long long)nbuf;
+        } else if (base + kPer * (unsigned long long)nbuf > a.out_cap) {
+            *wcur = 1;  // overflow: stop dequeuing
         }
     }
     base = __shfl_sync(kFull, base, 0);
@@ -215,16 +228,102 @@ __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs
     __syncwarp();
 }
 
+// 1-D..3-D pair modes: COLUMN buffers.  Lane l appends its own hits to column l of the warp's
+// buffer (hit r of lane l at buf[r*kColPitch + l]) with one predicated shared store, so an evaluation
+// step costs no warp vote; a flush ranks the columns with one warp scan, reserves the output
+// slots with ONE atomicAdd and writes coalesced 16-byte streaming stores -- output position o
+// finds its column by a 5-step binary search over the columns' exclusive offsets.  (In 4-D+
+// hits are rare (~2 % of the calculations) and the ballot-ranked buffer below skips hit-free
+// steps with one vote; there the column fill would force frequent flushes.)
+template <int DIM, int MODE>
+struct Cols {
+    static constexpr bool value = SJ_COLS && Mode<MODE>::pairs && DIM <= 3;
+};
+
+//
+// In the column modes the per-lane `nbuf` is the shared-memory ADDRESS of the lane's next
+// column slot (column base + kColPitch * 8 B per buffered hit), so appending a hit is one predicated
+// st.shared plus one add.
+__device__ __forceinline__ unsigned col_base(const uint2 *buf, int lane) {
+    return (unsigned)__cvta_generic_to_shared(buf) + 8u * (unsigned)lane;
+}
+
+template <bool GCG, bool EXACT>
+__device__ __forceinline__ void flush_cols(const uint2 *buf, int &nbuf, const JoinArgs &a, int lane,
+                                           unsigned long long *wcur) {
+    __syncwarp();
+    const unsigned col0 = col_base(buf, lane);
+    const int cnt = (int)(((unsigned)nbuf - col0) / (8u * kColPitch));
+    int incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += v;
+    }
+    const int excl = incl - cnt;
+    const unsigned total = (unsigned)__shfl_sync(kFull, incl, 31);
+    constexpr unsigned long long kPer = GCG ? 1ull : 2ull;  // pairs per buffered hit
+    unsigned long long base = 0;
+    if (lane == 0) {
+        base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)total);
+        if (EXACT) {
+            base = *wcur;
+            *wcur = base + kPer * (unsigned long long)total;
+        } else if (base + kPer * (unsigned long long)total > a.out_cap) {
+            *wcur = 1;  // overflow: stop dequeuing
+        }
+    }
+    base = __shfl_sync(kFull, base, 0);
+    const bool fits = base + kPer * (unsigned long long)total <= a.out_cap;
+    uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
+    uint4 *out4 = reinterpret_cast<uint4 *>(a.out) + (base >> 1);  // base is even (mirrored modes)
+    for (unsigned o0 = 0; o0 < total; o0 += 32) {
+        const int o = (int)o0 + lane;
+        int l = 0, el = 0;  // the last column whose exclusive offset is <= o
+#pragma unroll
+        for (int st = 16; st > 0; st >>= 1) {
+            const int e = __shfl_sync(kFull, excl, l + st);
+            if (e <= o) {
+                l += st;
+                el = e;
+            }
+        }
+        if ((unsigned)o < total) {
+            uint2 v;  // {orig q, orig c}; volatile asm: ordered after the column stores
+            asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n"
+                         : "=r"(v.x), "=r"(v.y)
+                         : "r"((unsigned)__cvta_generic_to_shared(buf + (o - el) * kColPitch + l)));
+            if constexpr (GCG) {
+                if (fits || base + (unsigned long long)o < a.out_cap) __stcs(out2 + base + o, v);
+            } else {
+                const unsigned long long slot = base + 2ull * (unsigned long long)o;
+                if (fits || slot + 2 <= a.out_cap)
+                    __stcs(out4 + o, make_uint4(v.x, v.y, v.y, v.x));  // (q,c) and (c,q)
+                else if (slot < a.out_cap)
+                    __stcs(out2 + slot, make_uint2(v.x, v.y));
+            }
+        }
+    }
+    nbuf = (int)col0;
+    __syncwarp();
+}
+
 // Warp-aggregated emission of one evaluation step (all 32 lanes call it): the hits are
 // ranked with __ballot_sync/__popc into the warp's shared buffer.  Before each round the
 // caller makes room for the round's maximum number of hits (flush_if) instead of checking
 // after every step.  kRows: the hits of a k-lane group (gbits) go straight to the group's
 // query row at its cursor `cur`, in candidate order.
-template <int MODE, bool GCG, bool RARE = false>
+template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *buf, int &nbuf,
                                      unsigned long long &nhits, unsigned lt, unsigned gbits,
-                                     unsigned long long &cur, const JoinArgs &a) {
-    if constexpr (Mode<MODE>::pairs) {
+                                     unsigned long long &cur, const JoinArgs &a, int lane) {
+    constexpr bool RARE = DIM >= 4;
+    if constexpr (Cols<DIM, MODE>::value) {  // nbuf: shared address of this lane's next column slot
+        if (hit) {
+            asm volatile("st.shared.v2.u32 [%0], {%1, %2};\n" ::"r"(nbuf), "r"(oq), "r"(oc));
+            nbuf += 8 * kColPitch;
+        }
+    } else if constexpr (Mode<MODE>::pairs) {
         const unsigned hm = __ballot_sync(kFull, hit);
         if (RARE && hm == 0u) return;  // high dimensions: most steps have no hit in the warp
         if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, oc);
@@ -241,11 +340,32 @@ __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *
     }
 }
 
-template <int MODE, bool GCG, int CAP = kBufHits>
+// Make room before a round: `room` = the most hits the round can add to the warp (a multiple
+// of 32; a column gains at most room/32).
+template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane,
                                          unsigned long long *wcur) {
-    if constexpr (Mode<MODE>::pairs) {
+    constexpr int CAP = BufCap<DIM>::value;
+    if constexpr (Cols<DIM, MODE>::value) {
+        const unsigned lim = col_base(buf, lane) + 8u * kColPitch * (unsigned)(kColRows - room / 32);
+        if (__any_sync(kFull, (unsigned)nbuf > lim)) flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+    } else if constexpr (Mode<MODE>::pairs) {
         if (nbuf > CAP - room) {
+            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+            nbuf = 0;
+        }
+    }
+}
+
+// Flush whatever is buffered (end of an exact-sizing chunk, end of the kernel).
+template <int DIM, int MODE, bool GCG>
+__device__ __forceinline__ void flush_all(uint2 *buf, int &nbuf, const JoinArgs &a, int lane,
+                                          unsigned long long *wcur) {
+    if constexpr (Cols<DIM, MODE>::value) {
+        if (__any_sync(kFull, (unsigned)nbuf != col_base(buf, lane)))
+            flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+    } else if constexpr (Mode<MODE>::pairs) {
+        if (nbuf > 0) {
             flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
             nbuf = 0;
         }
@@ -360,8 +480,8 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                 if (GCG) hit = hit && cidx != qlid;  // GCG scans its own cell: skip (q, q)
                 i += K;
             }
-            flush_if<MODE, GCG, BufCap<DIM>::value>(buf, nbuf, 32, a, lane, &ws.wcur);
-            emit<MODE, GCG, (DIM >= 4)>(hit, oq, oc, buf, nbuf, nhits, lt, gbits, cur, a);
+            flush_if<DIM, MODE, GCG>(buf, nbuf, 32, a, lane, &ws.wcur);
+            emit<DIM, MODE, GCG>(hit, oq, oc, buf, nbuf, nhits, lt, gbits, cur, a, lane);
         }
         if constexpr (MODE == kDegree) {  // the query's degree: its group's hits
             const unsigned deg = group_sum<K>((unsigned)(nhits - nh0));
@@ -418,7 +538,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             }
             unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
             const unsigned long long nh0 = nhits;
-            flush_if<MODE, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.wcur);
+            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.wcur);
             // all SPL distances first (independent FP64 chains -> ILP), then the emissions;
             // evaluated unconditionally and masked after (invalid slots may hold stale or
             // uninitialised bits; FP64 arithmetic on them cannot trap)
@@ -434,7 +554,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     if (d < 0) d += (int)m;
                     ok = ok & ((unsigned)d < hl);
                 }
-                emit<MODE, GCG, (DIM >= 4)>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt, gbits, cur, a);
+                emit<DIM, MODE, GCG>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt, gbits, cur, a, lane);
             }
             round_end(qi, qv, cur, nh0);
         }
@@ -472,14 +592,14 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 okb = okb & ((unsigned)db < home_count(m, rrb));
             }
             const bool ha = ca & oka, hb = cb & okb;
-            flush_if<MODE, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
+            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
             unsigned long long cura = 0, curb = 0;
             if constexpr (MODE == kRows) {
                 cura = ws.qcur[q0];
                 curb = ws.qcur[q1 & 31];
             }
-            emit<MODE, GCG, true>(ha, oqa, co, ws.buf, nbuf, nhits, lt, kFull, cura, a);
-            emit<MODE, GCG, true>(hb, oqb, co, ws.buf, nbuf, nhits, lt, kFull, curb, a);
+            emit<DIM, MODE, GCG>(ha, oqa, co, ws.buf, nbuf, nhits, lt, kFull, cura, a, lane);
+            emit<DIM, MODE, GCG>(hb, oqb, co, ws.buf, nbuf, nhits, lt, kFull, curb, a, lane);
             if constexpr (MODE == kRows) {
                 __syncwarp();
                 if (lane == 0) {
@@ -512,7 +632,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             const unsigned long long nh0 = nhits;
 #pragma unroll 2
             for (int s = 0; s < SPL; s += 2) {  // two slots per step: two independent FP64 chains
-                flush_if<MODE, GCG, BufCap<DIM>::value>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
+                flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
                 const unsigned j0 = t + (unsigned)(K * s), j1 = j0 + (unsigned)K;
                 double c0[DIM], c1[DIM];
                 load_smem_point<DIM>(tile + (j0 & 31) * PAD, c0);
@@ -533,10 +653,10 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     ok1 = ok1 & ((unsigned)d1 < hl);
                 }
                 const bool hit0 = close0 & ok0, hit1 = close1 & ok1;
-                emit<MODE, GCG, (DIM >= 4)>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
-                                            cur, a);
-                emit<MODE, GCG, (DIM >= 4)>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
-                                            cur, a);
+                emit<DIM, MODE, GCG>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
+                                            cur, a, lane);
+                emit<DIM, MODE, GCG>(hit1, oq, hit1 ? tile_orig[j1 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
+                                            cur, a, lane);
             }
             round_end(qi, qv, cur, nh0);
         }
@@ -652,18 +772,39 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     const int warp = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     WarpSmem<DIM, MODE> &ws = reinterpret_cast<WarpSmem<DIM, MODE> *>(smem_raw)[warp];
-    int nbuf = 0;
+    int nbuf = Cols<DIM, MODE>::value ? (int)col_base(ws.buf, lane) : 0;  // column modes: see flush_cols
     unsigned long long nhits = 0;
     unsigned long long ncalcs = 0;
+    if constexpr (MODE == kPairs) {
+        if (lane == 0) ws.wcur = 0;
+        __syncwarp();
+    }
 
+    // The batch: virtual chunks v_begin, v_begin + v_stride, ... < v_end (contiguous, or the
+    // strided D'_l of the SortByWL-only batches); i indexes them.
+    const unsigned vcount = a.v_count;
+    if (lane == 0) ws.snext = (blockIdx.x * (unsigned)kWarps + (unsigned)warp) * a.grab;  // static assignment
     for (;;) {
-        // WorkQueue dequeue: one atomic per warp, result shuffled
-        unsigned long long vb = 0;
-        if (lane == 0) vb = atomicAdd(a.head, (unsigned long long)a.grab);
-        vb = __shfl_sync(kFull, vb, 0) + a.v_begin;
-        if (vb >= a.v_end) break;
-        const unsigned long long vend = min(vb + a.grab, a.v_end);
-        for (unsigned long long v = vb; v < vend; ++v) {
+        // WorkQueue dequeue: one atomic per warp, result shuffled.  SortByWL only
+        // (static_q): warp w takes w, w + #warps, ... in D' order, no atomics (the
+        // cursor lives in shared memory, not in a register of the hot loops).
+        // kPairs: a warp whose flush found the output full stops (the caller re-runs staged).
+        unsigned ib = 0;
+        if (lane == 0) {
+            if (MODE == kPairs && ws.wcur) {
+                ib = vcount;
+            } else if (a.static_q) {
+                ib = ws.snext;
+                ws.snext = ib + gridDim.x * (unsigned)kWarps * a.grab;
+            } else {
+                ib = (unsigned)atomicAdd(a.head, (unsigned long long)a.grab);
+            }
+        }
+        ib = __shfl_sync(kFull, ib, 0);
+        if (ib >= vcount) break;
+        const unsigned iend = min(ib + a.grab, vcount);
+        for (unsigned i = ib; i < iend; ++i) {
+            const unsigned long long v = a.v_begin + (unsigned long long)i * a.v_stride;
             const unsigned long long c = v * a.world + a.rank;  // queue slice (multi-GPU)
             if (c >= a.n_chunks) break;
             if constexpr (MODE == kExact) {  // exact sizing: the chunk's pairs start at voff[v]
@@ -705,10 +846,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
             }
             if (gmask) generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
             if constexpr (MODE == kExact) {  // exact sizing: a chunk's pairs never share a flush
-                if (nbuf > 0) {
-                    flush<GCG, true>(ws.buf, nbuf, a, lane, &ws.wcur);
-                    nbuf = 0;
-                }
+                flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.wcur);
             } else if constexpr (MODE == kChunkCount) {  // exact sizing, pass 1: pairs per chunk
                 unsigned long long d = nhits - nh0;
 #pragma unroll
@@ -719,7 +857,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         }
     }
     if constexpr (Mode<MODE>::pairs) {
-        if (nbuf > 0) flush<GCG, Mode<MODE>::exact>(ws.buf, nbuf, a, lane, &ws.wcur);
+        flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.wcur);
     } else {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) nhits += __shfl_xor_sync(kFull, nhits, o);
@@ -823,9 +961,13 @@ int join_occupancy(int dim, int k, int mode, bool gcg, int *blocks_per_sm) {
     return SJ_OK;
 }
 
-int launch_join(const JoinArgs &a, int dim, int k, int mode, int blocks, cudaStream_t s) {
+int launch_join(const JoinArgs &a0, int dim, int k, int mode, int blocks, cudaStream_t s) {
     KernelInfo ki;
-    SJ_TRY(prepare(dim, k, mode, a.gcg != 0, &ki));
+    SJ_TRY(prepare(dim, k, mode, a0.gcg != 0, &ki));
+    JoinArgs a = a0;
+    const uint64_t st = a.v_stride ? a.v_stride : 1;
+    a.v_stride = (uint32_t)st;
+    a.v_count = a.v_end > a.v_begin ? (uint32_t)((a.v_end - a.v_begin + st - 1) / st) : 0u;
     ki.f<<<blocks, kJoinThreads, ki.smem, s>>>(a);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());

@@ -138,8 +138,11 @@ struct JoinArgs {
     uint64_t n_runs;              // entries of runs (bounds of the staged copies)
     double e2;
     unsigned long long *head;     // WorkQueue counter (chunks taken), zeroed before the launch
-    unsigned long long v_begin;   // batch = virtual chunk range [v_begin, v_end) of this slice
-    unsigned long long v_end;
+    unsigned long long v_begin;   // batch = virtual chunks v_begin, v_begin + v_stride, ... < v_end
+    unsigned long long v_end;     //   of this slice (v_stride 1: a contiguous range)
+    uint32_t v_stride;
+    uint32_t v_count;             // the batch's chunks (set by launch_join)
+    uint32_t static_q;            // 1: static warp -> chunk assignment (SortByWL only), 0: WorkQueue
     uint32_t grab;                // chunks per dequeue
     uint32_t gcg;                 // 1: GCG pattern (full neighbourhood, one pair per hit)
     uint32_t rank, world;         // queue slice: virtual chunk v -> chunk v*world + rank

@@ -112,7 +112,8 @@ namespace {
 constexpr int kMaxStreams = 8;
 
 struct Job {
-    uint64_t v0, v1;  // virtual WorkQueue chunk range [v0, v1) of this handle's slice
+    uint64_t v0, v1;  // virtual chunks v0, v0 + stride, ... < v1 of this handle's slice
+    uint64_t stride = 1;             // 1: contiguous (WorkQueue); nbBatches: strided D'_l
     uint64_t base = 0;               // exact sizing: pair offset of chunk v0 in the whole join
     uint64_t expect = UINT64_MAX;    // exact sizing: the batch's pairs (UINT64_MAX: estimated)
     int slot = -1;
@@ -135,7 +136,8 @@ struct sj_handle {
     int device = 0;
     int state = 0;  // 0 ready, 1 continuing (staged path), -1 error
     cudaStream_t s_main = nullptr;
-    cudaEvent_t ev_a = nullptr, ev_b = nullptr, ev_c = nullptr, ev_d = nullptr;
+    cudaStream_t s_side = nullptr;  // fast path: the estimator, concurrent with the join
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr, ev_c = nullptr, ev_d = nullptr, ev_e = nullptr;
     sj::Index ix;
     bool owns_index = true;
     int num_sms = 148;
@@ -150,6 +152,7 @@ struct sj_handle {
     int blocks_per_sm = 0;
     int fast_path = 1;
     int exact = 0;
+    int queue = 1;  // 1: WorkQueue; 0: SortByWL only (static assignment, strided batches)
     int rank = 0, world = 1;
 
     uint64_t *d_voff = nullptr;  // exact sizing: per-chunk pairs -> offsets, [V+1]
@@ -186,14 +189,14 @@ bool is_device_ptr(const void *p, int dev) {
     return false;
 }
 
-// Per-handle CUDA objects (main stream, 4 timing events, device counters, pinned mailbox)
+// Per-handle CUDA objects (main stream, 5 timing events, device counters, pinned mailbox)
 // are recycled process-wide per device: creating and destroying them costs ~0.1 ms per
 // handle, a visible fraction of a millisecond-scale join.
 struct Core {
     int device;
     int num_sms;
-    cudaStream_t s;
-    cudaEvent_t ev[4];
+    cudaStream_t s, s2;
+    cudaEvent_t ev[5];
     unsigned long long *d_ctr;
     uint64_t *mail;
 };
@@ -210,10 +213,12 @@ int handle_init_common(sj_handle *h) {
                 g_core_cache.erase(g_core_cache.begin() + (long)k);
                 h->num_sms = c.num_sms;
                 h->s_main = c.s;
+                h->s_side = c.s2;
                 h->ev_a = c.ev[0];
                 h->ev_b = c.ev[1];
                 h->ev_c = c.ev[2];
                 h->ev_d = c.ev[3];
+                h->ev_e = c.ev[4];
                 h->d_ctr = c.d_ctr;
                 h->mail = c.mail;
                 return SJ_OK;
@@ -222,10 +227,12 @@ int handle_init_common(sj_handle *h) {
     pool_setup(h->device);
     SJ_CUDA_TRY(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device));
     SJ_CUDA_TRY(cudaStreamCreateWithFlags(&h->s_main, cudaStreamNonBlocking));
+    SJ_CUDA_TRY(cudaStreamCreateWithFlags(&h->s_side, cudaStreamNonBlocking));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_a));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_b));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_c));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_d));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_e));
     h->mail = static_cast<uint64_t *>(pinned_acquire());
     if (!h->mail) return SJ_ENOMEM;
     SJ_TRY(dev_alloc_t(&h->d_ctr, 8, h->s_main));
@@ -234,14 +241,14 @@ int handle_init_common(sj_handle *h) {
 
 // Returns the handle's core to the cache (stream drained first); false if it must be freed.
 bool core_release(sj_handle *h) {
-    if (!h->s_main || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->d_ctr || !h->mail) return false;
+    if (!h->s_main || !h->s_side || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->ev_e || !h->d_ctr || !h->mail) return false;
     if (cudaStreamSynchronize(h->s_main) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
     std::lock_guard<std::mutex> lk(g_core_mu);
     if (g_core_cache.size() >= 64) return false;
-    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d}, h->d_ctr,
+    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, h->s_side, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e}, h->d_ctr,
                                 h->mail});
     return true;
 }
@@ -307,6 +314,22 @@ void slots_release(sj_handle *h) {
 }
 
 // number of WorkQueue chunks of this handle's slice (chunk c belongs to rank c mod world)
+// Batch l of nb over the nch virtual chunks of a slice: WorkQueue batches are
+// contiguous ranges of D' (reading c14); SortByWL-only batches are the strided D'_l =
+// {v : v mod nb = l} of Fig. 1.  Returned as {v0, v1, stride}: chunks v0, v0 + stride, ... < v1.
+Job batch_job(uint64_t nch, uint64_t nb, uint64_t l, bool queue) {
+    Job j;
+    if (queue) {
+        j.v0 = nch * l / nb;
+        j.v1 = nch * (l + 1) / nb;
+    } else {
+        j.v0 = l;
+        j.v1 = nch;
+        j.stride = nb;
+    }
+    return j;
+}
+
 uint64_t slice_chunks(const sj_handle *h) {
     const uint64_t nchunks = h->ix.n_chunks;
     if (nchunks <= (uint64_t)h->rank) return 0;
@@ -325,6 +348,8 @@ JoinArgs base_args(const sj_handle *h) {
     a.n_runs = h->ix.n_runs;
     a.e2 = h->ix.e2;
     a.grab = h->grab;
+    a.v_stride = 1;
+    a.static_q = h->queue ? 0u : 1u;
     a.gcg = h->ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
     a.rank = (uint32_t)h->rank;
     a.world = (uint32_t)h->world;
@@ -343,13 +368,15 @@ int join_blocks(const sj_handle *h, int mode, int *blocks) {
 // Count-only join over virtual range [v0, v1) on the main stream.  Synchronous.  With
 // vcount, every chunk's pairs are recorded and scanned in place into chunk offsets
 // (exact sizing, pass 1): vcount[V] receives the total.
-int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms, uint64_t *vcount = nullptr) {
+int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms, uint64_t *vcount = nullptr,
+                uint64_t stride = 1) {
     cudaStream_t s = h->s_main;
     SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
     JoinArgs a = base_args(h);
     a.head = h->d_ctr + 1;  // zeroed above
     a.v_begin = v0;
     a.v_end = v1;
+    a.v_stride = (uint32_t)stride;
     a.out = nullptr;
     a.emit_ctr = h->d_ctr;
     a.out_cap = 0;
@@ -379,6 +406,7 @@ int launch_job(sj_handle *h, Job &j, int slot_idx) {
     a.head = s.d_ctr + 1;  // zeroed above
     a.v_begin = j.v0;
     a.v_end = j.v1;
+    a.v_stride = (uint32_t)j.stride;
     a.out = s.buf;
     a.emit_ctr = s.d_ctr;
     a.out_cap = s.cap;
@@ -449,7 +477,7 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
                 h->st.retries++;
                 if (h->count_calcs) h->st.calcs_measured -= m[2];
                 const Job old = j;
-                const uint64_t chunks = old.v1 - old.v0;
+                const uint64_t chunks = (old.v1 - old.v0 + old.stride - 1) / old.stride;
                 h->jobs.pop_front();
                 s.busy = false;
                 if (chunks <= 1) {
@@ -457,14 +485,21 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
                     Job again;
                     again.v0 = old.v0;
                     again.v1 = old.v1;
+                    again.stride = old.stride;
                     h->jobs.push_front(again);
                     SJ_TRY(launch_job(h, h->jobs.front(), old.slot));
                 } else {
                     const uint64_t parts = std::min<uint64_t>(chunks, old.cnt / s.cap + 2);
                     for (uint64_t p = parts; p-- > 0;) {
                         Job nj;
-                        nj.v0 = old.v0 + chunks * p / parts;
-                        nj.v1 = old.v0 + chunks * (p + 1) / parts;
+                        if (old.stride == 1) {  // WorkQueue batches stay contiguous ranges of D' (c14)
+                            nj.v0 = old.v0 + chunks * p / parts;
+                            nj.v1 = old.v0 + chunks * (p + 1) / parts;
+                        } else {  // strided batches split into interleaved sub-batches
+                            nj.v0 = old.v0 + p * old.stride;
+                            nj.v1 = old.v1;
+                            nj.stride = old.stride * parts;
+                        }
                         if (nj.v1 > nj.v0) h->jobs.push_front(nj);
                     }
                     h->st.batches += (uint32_t)(parts - 1);
@@ -538,6 +573,59 @@ int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_
     h->st.batches = 1;
     h->st.ms_join = h->st.ms_join_sum = ms;
     *emitted = h->mail[0];
+    return SJ_OK;
+}
+
+// Fast path (caller's HBM buffer, in place): the estimator (a9) -- a count-only join of
+// the first sch chunks of D' -- runs on a side stream CONCURRENTLY with the join, which writes
+// the whole queue [0, V) into the caller's buffer and does not wait for the estimate (in place
+// there are no batches to size; the estimate is reported, and sizes the staged fallback if the
+// buffer overflows).  The estimator gets only the CTAs its chunks can use, so it shares the
+// GPU with the join instead of running ahead of it.  *spairs = the sample's pairs, *total =
+// all pairs emitted (> cap: overflow, only the first cap were written).
+int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, uint64_t sv1, uint64_t sstride,
+                     uint64_t V, uint64_t *spairs, uint64_t *total) {
+    cudaStream_t s = h->s_main;
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
+    SJ_CUDA_TRY(cudaStreamWaitEvent(h->s_side, h->ev_c, 0));
+    JoinArgs e = base_args(h);
+    e.head = h->d_ctr + 5;
+    e.emit_ctr = h->d_ctr + 4;
+    e.v_begin = 0;
+    e.v_end = sv1;  // the sample: chunks 0, sstride, ... < sv1 (sch of them)
+    e.v_stride = (uint32_t)sstride;
+    int blocks_e;
+    SJ_TRY(join_blocks(h, kCount, &blocks_e));
+    const uint64_t warps = (sch + h->grab - 1) / h->grab;  // one dequeue per warp
+    const uint64_t need = (warps + kJoinThreads / 32 - 1) / (kJoinThreads / 32);
+    blocks_e = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)blocks_e, need));
+    if (sch) SJ_TRY(launch_join(e, h->ix.dim, h->k, kCount, blocks_e, h->s_side));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_e, h->s_side));
+    JoinArgs a = base_args(h);
+    a.out = out;
+    a.emit_ctr = h->d_ctr;
+    a.out_cap = cap;
+    a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+    a.head = h->d_ctr + 1;
+    a.v_begin = 0;
+    a.v_end = V;
+    int blocks;
+    SJ_TRY(join_blocks(h, kPairs, &blocks));
+    if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, kPairs, blocks, s));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+    SJ_CUDA_TRY(cudaStreamWaitEvent(s, h->ev_e, 0));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 5 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    float ms_est = 0, ms = 0;
+    SJ_CUDA_TRY(cudaEventElapsedTime(&ms_est, h->ev_c, h->ev_e));
+    SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
+    h->st.join_launches = V ? 1u : 0u;
+    h->st.batches = 1;
+    h->st.ms_estimate = ms_est;              // the estimator (concurrent with the join)
+    h->st.ms_join = h->st.ms_join_sum = ms;  // the join launch (with the estimator alongside)
+    *spairs = h->mail[4];
+    *total = h->mail[0];
     return SJ_OK;
 }
 
@@ -662,14 +750,37 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     }
     if (h->exact) return start_exact(h, out, cap, count, dev_out);
 
-    // a9: batch estimator -- count-only join over the first sample_ppm of D'
+    // a9: batch estimator -- join over the first sample_ppm of D' (WorkQueue), or over a
+    // strided sample of the whole dataset (SortByWL only: "samples a percentage of the
+    // dataset"; P:200 contrasts the two)
     uint64_t sch = (nch * (uint64_t)h->sample_ppm + 999999ull) / 1000000ull;
     if (sch < 1) sch = 1;
     if (sch > nch) sch = nch;
+    uint64_t sstride = 1, sv1 = sch;
+    if (!h->queue && nch) {
+        sstride = (nch + sch - 1) / sch;
+        sv1 = nch;
+        sch = (nch + sstride - 1) / sstride;  // chunks 0, sstride, 2 sstride, ...
+    }
     uint64_t spairs = 0;
     float ms_est = 0;
     debug_mark("join: enter");
-    if (nch) SJ_TRY(count_range(h, 0, sch, &spairs, &ms_est));
+    if (dev_out && h->fast_path && !getenv("SJ_DEBUG_VRANGE")) {
+        // Fast path: the caller's HBM buffer is the result buffer; the estimator runs alongside
+        // the join.  Overflow is detected from the counter (the join stops early) and falls back
+        // to the staged path below, whose batches are sized by the estimate.
+        uint64_t total = 0;
+        SJ_TRY(run_in_place_est(h, out, cap, sch, sv1, sstride, V, &spairs, &total));
+        debug_mark("join: fast path");
+        h->st.est_pairs = nch ? (uint64_t)((double)spairs * (double)nch / (double)sch) : 0;
+        if (total <= cap) return finish_in_place(h, total, count);
+        ms_est = (float)h->st.ms_estimate;
+        h->st.retries++;  // did not fit: fall through to the staged path
+        h->st.ms_join = h->st.ms_join_sum = 0;
+        h->st.join_launches = 0;
+    } else if (nch) {
+        SJ_TRY(count_range(h, 0, sv1, &spairs, &ms_est, nullptr, sstride));
+    }
     debug_mark("join: estimator");
     h->st.ms_estimate = ms_est;
     h->st.calcs_measured = 0;
@@ -682,9 +793,8 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     // The sample's own pairs are part of the result, so spairs is a strict lower bound of the
     // total; the extrapolated estimate is NOT (the first 1% of D' is the heaviest part)
     // and is only used to size the staged batches.
-    if (dev_out && h->fast_path && spairs <= cap) {
-        // Fast path: the caller's HBM buffer is the result buffer.  Overflow is detected from
-        // the counter and falls back to the staged path.
+    if (dev_out && h->fast_path && spairs <= cap && getenv("SJ_DEBUG_VRANGE")) {
+        // diagnostics: the in-place join of a sub-range only
         unsigned long long dv0 = 0, dv1 = V;
         if (const char *r = getenv("SJ_DEBUG_VRANGE")) {  // diagnostics: join a sub-range only
             sscanf(r, "%llu,%llu", &dv0, &dv1);
@@ -699,11 +809,10 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         h->st.join_launches = 0;
     }
 
-    // Staged path: nb batches = contiguous ranges of D' (reading c14).
+    // Staged path: nb batches = contiguous ranges of D' (WorkQueue, reading c14), or the
+    // strided D'_l = {chunk v : v mod nb = l} of SortByWL only (Fig. 1).
     for (uint64_t b = 0; b < nb; ++b) {
-        Job j;
-        j.v0 = nch * b / nb;
-        j.v1 = nch * (b + 1) / nb;
+        const Job j = batch_job(nch, nb, b, h->queue != 0);
         if (j.v1 > j.v0) h->jobs.push_back(j);
     }
     return start_staged(h, out, cap, count);
@@ -1001,11 +1110,13 @@ void sj_destroy(sj_handle *h) {
             dev_free(h->d_ctr, h->s_main);
             cudaStreamSynchronize(h->s_main);
             cudaStreamDestroy(h->s_main);
+            if (h->s_side) cudaStreamDestroy(h->s_side);
         }
         if (h->ev_a) cudaEventDestroy(h->ev_a);
         if (h->ev_b) cudaEventDestroy(h->ev_b);
         if (h->ev_c) cudaEventDestroy(h->ev_c);
         if (h->ev_d) cudaEventDestroy(h->ev_d);
+        if (h->ev_e) cudaEventDestroy(h->ev_e);
         pinned_release(h->mail);
     }
     delete h;
@@ -1048,6 +1159,10 @@ int sj_set_option(sj_handle *h, int opt, int64_t v) {
             return SJ_OK;
         case SJ_OPT_EXACT:
             h->exact = v ? 1 : 0;
+            return SJ_OK;
+        case SJ_OPT_QUEUE:
+            if (v != 0 && v != 1) break;
+            h->queue = (int)v;
             return SJ_OK;
 
     }
@@ -1222,6 +1337,22 @@ int64_t sj_slice_chunks(uint64_t n_chunks, int rank, int world, uint32_t *out, u
         if (out) {
             if ((uint64_t)cnt >= cap) return SJ_EINVAL;
             out[cnt] = (uint32_t)c;
+        }
+        ++cnt;
+    }
+    return cnt;
+}
+
+int64_t sj_batch_chunks(uint64_t n_chunks, uint64_t n_batches, uint64_t batch, int queue, uint32_t *out,
+                        uint64_t cap) {
+    if (n_batches < 1 || batch >= n_batches || n_chunks >= (1ull << 32) || (queue != 0 && queue != 1))
+        return SJ_EINVAL;
+    const Job j = batch_job(n_chunks, n_batches, batch, queue != 0);
+    int64_t cnt = 0;
+    for (uint64_t v = j.v0; v < j.v1; v += j.stride) {
+        if (out) {
+            if ((uint64_t)cnt >= cap) return SJ_EINVAL;
+            out[cnt] = (uint32_t)v;
         }
         ++cnt;
     }

@@ -73,6 +73,37 @@ def test_slice_chunks_disjoint_cover(nch, world):
     assert max(sizes) - min(sizes) <= 1
 
 
+def test_batch_chunks_fig1_strided():
+    """P:73, Fig. 1: 12 points, nbBatches = 3, each batch 4 points strided across the dataset --
+    query q_i (1-based) goes to batch (i - 1) mod 3.  With one point per chunk, the SortByWL-only
+    rule (queue = 0) must reproduce exactly that assignment."""
+    for l in range(3):
+        got = sj.sj_batch_chunks(12, 3, l, queue=0)
+        want = [i - 1 for i in range(1, 13) if (i - 1) % 3 == l]
+        assert got.tolist() == want and len(got) == 4
+
+
+@pytest.mark.parametrize("nch,nb", [(12, 3), (1000, 7), (5, 5), (240173, 5), (1, 1), (10, 4)])
+@pytest.mark.parametrize("queue", [0, 1])
+def test_batch_chunks_partition(nch, nb, queue):
+    """Every chunk lands in exactly one batch; WorkQueue batches are contiguous ascending ranges
+    of D' (reading c14), SortByWL-only batches are residue classes mod nbBatches."""
+    parts = [sj.sj_batch_chunks(nch, nb, l, queue) for l in range(nb)]
+    cat = np.concatenate(parts)
+    assert np.array_equal(np.sort(cat), np.arange(nch, dtype=np.uint32))
+    for l, p in enumerate(parts):
+        if queue:
+            assert len(p) == 0 or np.array_equal(p, np.arange(p[0], p[0] + len(p), dtype=np.uint32))
+            if l and len(p) and len(parts[l - 1]):
+                assert p[0] == parts[l - 1][-1] + 1
+        else:
+            assert np.all(p % nb == l)
+    sizes = [len(p) for p in parts]
+    assert max(sizes) - min(sizes) <= 1
+    with pytest.raises(sj.SJError):
+        sj.sj_batch_chunks(nch, nb, nb, queue)
+
+
 def test_fails_loudly_without_gpu():
     import torch
 

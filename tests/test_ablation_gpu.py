@@ -129,3 +129,51 @@ def test_inner_cell_patterns_fig5_alg2(pattern):
         want = np.select([(p0 == 0) & (p1 == 0), (p0 == 1) & (p1 == 0), (p0 == 0) & (p1 == 1)], [0, 2, 6], 8)
         np.testing.assert_array_equal(fwd_points, want)
         assert set(np.unique(fwd_points).tolist()) == {0, 2, 6, 8}
+
+
+# ---------------------------------------------------------------- SortByWL only
+
+@pytest.mark.parametrize("pattern", ["lid_unicomp", "gcg"])
+@pytest.mark.parametrize("name,n", [("c2k64", 60_011), ("c3k64", 50_021), ("c4k32", 20_011), ("c5", 80_000)])
+def test_sortbywl_only_matches_oracle(pattern, name, n):
+    """SJ_OPT_QUEUE = 0: static warp -> chunk assignment over D', no WorkQueue atomics.
+    Same pair set and the same distance calculations as the WorkQueue (P:196 changes only who
+    takes which query, not what is computed), in place and through strided staged batches."""
+    cfg = workloads.get_config(name).scaled(n)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    for k in (1, 8):
+        got, st = run(pts, cfg.eps, pattern, "workload", k=k, queue=0)
+        np.testing.assert_array_equal(oracle.canonical(got), want)
+        ref = st["dist_calcs"]
+        assert st["calcs_measured"] == ref and st["fast_path"] == 1
+    # staged: the strided D'_l batches (P:71-73), several of them, with overflow re-runs
+    bp = max(2_000, want.shape[0] // 6)
+    got, st = run(pts, cfg.eps, pattern, "workload", queue=0, fast_path=0, batch_pairs=bp)
+    np.testing.assert_array_equal(oracle.canonical(got), want)
+    assert st["batches"] >= 2 and st["calcs_measured"] == st["dist_calcs"]
+
+
+def test_sortbywl_only_host_more_and_exact():
+    """Strided batches delivered into a small pageable host buffer (SJ_MORE continuation), and
+    exact two-pass sizing with the static assignment (deterministic order across runs)."""
+    cfg = workloads.get_config("c3k64").scaled(40_009)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    d = torch.from_numpy(pts).to(DEV)
+    with sj.Handle(d, cfg.eps, queue=0, fast_path=0, batch_pairs=20_000) as h:
+        total = h.count()
+        cap = total // 5 + 3
+        buf = np.zeros((cap, 2), dtype=np.uint32)
+        parts, rc = [], sj.SJ_MORE
+        while rc == sj.SJ_MORE:
+            rc, c = h.self_join(buf, cap)
+            parts.append(buf[:c].copy())
+        got = np.concatenate(parts)
+    np.testing.assert_array_equal(oracle.canonical(got), want)
+    orders = []
+    for _ in range(2):
+        with sj.Handle(d, cfg.eps, queue=0, exact=1) as h:
+            orders.append(sj.self_join_pairs(h, DEV).cpu().numpy().view(np.uint32).reshape(-1, 2))
+    np.testing.assert_array_equal(orders[0], orders[1])
+    np.testing.assert_array_equal(oracle.canonical(orders[0]), want)

@@ -11,7 +11,7 @@ def main(path, steps):
     ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
     agg = collections.OrderedDict()
     for r in rows[hi + 1:]:
-        name = r[ki].split("(")[0].replace("void ", "").replace("sj::<unnamed>::", "")[:48]
+        name = r[ki].split("(")[0].replace("void ", "").replace("sj::<unnamed>::", "").replace("sj::", "")[:int(__import__("os").environ.get("LS_W", "48"))]
         v = float(r[vi].replace(",", ""))
         u = r[ui]
         v = v / 1e3 if u in ("ns", "nsecond") else v * 1e3 if u in ("ms", "msecond") else v
