@@ -498,6 +498,40 @@ struct ChunkLoad {
         return f ? 1u : 0u;
     }
 };
+// The same boundaries counted and written per queue CELL (cells are contiguous in D' in the
+// SortByWL and cell orders): a scan over the M cells instead of a gather per D' position.
+// Cell i = [beg, beg + m): a big cell has a boundary every kChunk positions from beg; a small
+// one at its kChunk-aligned positions, plus beg itself when the previous cell was big.
+struct CellChunkLoad {
+    const uint4 *cellq;
+    const uint32_t *qb;
+    uint32_t big_min;
+    __device__ unsigned operator()(uint64_t i) const {
+        const uint32_t beg = qb[i], m = cellq[i].y;
+        if (m >= big_min) return (m + kChunk - 1) / kChunk;
+        unsigned c = (beg + m + kChunk - 1) / kChunk - (beg + kChunk - 1) / kChunk;
+        if (beg % kChunk != 0 && i > 0 && cellq[i - 1].y >= big_min) ++c;
+        return c;
+    }
+};
+struct CellChunkStore {
+    const uint4 *cellq;
+    const uint32_t *qb;
+    uint32_t big_min;
+    uint32_t *chunks;
+    __device__ void operator()(uint64_t i, unsigned ex, unsigned cnt) const {
+        if (!cnt) return;
+        const uint32_t beg = qb[i], m = cellq[i].y;
+        if (m >= big_min) {
+            for (unsigned j = 0; j < cnt; ++j) chunks[ex + j] = beg + j * kChunk;
+            return;
+        }
+        unsigned o = ex;
+        if (beg % kChunk != 0 && i > 0 && cellq[i - 1].y >= big_min) chunks[o++] = beg;
+        for (uint32_t p = (beg + kChunk - 1) / kChunk * kChunk; p < beg + m; p += kChunk) chunks[o++] = p;
+    }
+};
+
 struct ChunkStore {
     uint32_t *chunks;
     __device__ void operator()(uint64_t p, unsigned ex, unsigned flag) const {
@@ -765,7 +799,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     const unsigned long long ncells_total = (unsigned long long)total;
     ix.key_bits = bits_for(ncells_total - 1);
 
-    // ---- a3 + a4: cell ids and radix sort
+    // ---- a3 + a4 + a5: cell ids, point -> cell sort, compaction of the non-empty cells
     uint32_t *idx_sorted = nullptr;
     uint32_t *cellof;
     unsigned long long *cell_lid;
@@ -775,6 +809,9 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&cell_lid, n));
     SJ_TRY(tmp.alloc(&cell_start, n + 1));
     SJ_TRY(tmp.alloc(&d_M, 1));
+    // lid -> rank lookup: a dense table when prod(nc) is small, else a hash table
+    Lookup L{};
+    const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
     if (ix.key_bits <= 32) {
         uint32_t *ks;
         SJ_TRY(sort_points<uint32_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
@@ -784,10 +821,6 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         SJ_TRY(sort_points<uint64_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
         SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s));
     }
-
-    // ---- lid -> rank lookup: dense table when prod(nc) is small, else a hash table
-    Lookup L{};
-    const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
     if (dense) {
         uint32_t *tab;
         SJ_TRY(tmp.alloc(&tab, ncells_total));
@@ -918,8 +951,12 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(dev_alloc_t(&ix.chunks, n + 1, s));
     // in input order a cell's points are scattered: no chunk may claim a cell
     const uint32_t big_min = ix.order == SJ_ORDER_INPUT ? 0xFFFFFFFFu : kBigCell;
-    SJ_TRY(scan_fused(n, ChunkLoad{ix.qmap, ix.cellq, qb, big_min}, ChunkStore{ix.chunks}, s,
-                      ChunkDone{n, ix.chunks, d_nc}));
+    if (ix.order == SJ_ORDER_INPUT)
+        SJ_TRY(scan_fused(n, ChunkLoad{ix.qmap, ix.cellq, qb, big_min}, ChunkStore{ix.chunks}, s,
+                          ChunkDone{n, ix.chunks, d_nc}));
+    else
+        SJ_TRY(scan_fused(M, CellChunkLoad{ix.cellq, qb, big_min}, CellChunkStore{ix.cellq, qb, big_min, ix.chunks}, s,
+                          ChunkDone{n, ix.chunks, d_nc}));
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
     debug_mark("build: tail issued");

@@ -5,9 +5,9 @@
         -k regex:join_kernel --csv python tools/ablation.py --one c3k64 gcg input 1   # WEE of one variant
 
 Variants (Table II): GPUCALCGLOBAL (full 3^n pattern, input order, k=1), UNICOMP,
-LID-UNICOMP, k=8, SortByWL (workload-sorted order) and the combination (LID-UNICOMP +
-WorkQueue over the workload-sorted D' + k=8).  Every variant runs through the same chunked
-dequeue; "input" order is the paper's unsorted D.
+LID-UNICOMP, k=8, SortByWL (workload-sorted D', static thread assignment), WorkQueue (the
+same D' handed out by an atomic counter) and the combination (LID-UNICOMP + WorkQueue + k=8).
+"input" order is the paper's unsorted D.
 """
 import json
 import sys
@@ -18,25 +18,26 @@ sys.path.insert(0, ".")
 import paper_conf_ipps_galletg19_b200 as sj  # noqa: E402
 import workloads  # noqa: E402
 
-VARIANTS = [
-    ("GPUCALCGLOBAL", "gcg", "input", 1),
-    ("UNICOMP", "unicomp", "input", 1),
-    ("LID-UNICOMP", "lid_unicomp", "input", 1),
-    ("GPUCALCGLOBAL k=8", "gcg", "input", 8),
-    ("SORTBYWL (cell order)", "gcg", "cell", 1),
-    ("WORKQUEUE (sorted D')", "gcg", "workload", 1),
-    ("WORKQUEUE k=8", "gcg", "workload", 8),
-    ("WQ + LID-UNICOMP + k=8", "lid_unicomp", "workload", 8),
+VARIANTS = [  # (label, pattern, order, k, queue): queue 0 = static thread assignment, 1 = WorkQueue
+    ("GPUCALCGLOBAL", "gcg", "input", 1, 0),
+    ("UNICOMP", "unicomp", "input", 1, 0),
+    ("LID-UNICOMP", "lid_unicomp", "input", 1, 0),
+    ("GPUCALCGLOBAL k=8", "gcg", "input", 8, 0),
+    ("SORTBYWL", "gcg", "workload", 1, 0),
+    ("SORTBYWL k=8", "gcg", "workload", 8, 0),
+    ("WORKQUEUE", "gcg", "workload", 1, 1),
+    ("WORKQUEUE k=8", "gcg", "workload", 8, 1),
+    ("WQ + LID-UNICOMP + k=8", "lid_unicomp", "workload", 8, 1),
 ]
 
 
-def measure(cfg, d, pattern, order, k, reps=3):
-    with sj.Handle(d, cfg.eps, pattern=pattern, order=order, k=k) as h:
+def measure(cfg, d, pattern, order, k, queue, reps=3):
+    with sj.Handle(d, cfg.eps, pattern=pattern, order=order, k=k, queue=queue) as h:
         n = h.count()
     out = torch.empty((max(n, 1), 2), dtype=torch.int32, device="cuda")
     ts = []
     for _ in range(reps):
-        with sj.Handle(d, cfg.eps, pattern=pattern, order=order, k=k) as h:
+        with sj.Handle(d, cfg.eps, pattern=pattern, order=order, k=k, queue=queue) as h:
             rc, c = h.self_join(out, n)
             assert rc == sj.SJ_OK and c == n
             st = h.stats()
@@ -47,18 +48,21 @@ def measure(cfg, d, pattern, order, k, reps=3):
 def main():
     if len(sys.argv) > 1 and sys.argv[1] == "--one":
         name, pattern, order, k = sys.argv[2], sys.argv[3], sys.argv[4], int(sys.argv[5])
+        queue = int(sys.argv[6]) if len(sys.argv) > 6 else 1
         cfg = workloads.get_config(name)
         d = torch.from_numpy(cfg.points()).cuda()
-        ms, st, n = measure(cfg, d, pattern, order, k, reps=1)
-        print(json.dumps({"config": name, "pattern": pattern, "order": order, "k": k, "join_ms": ms}))
+        ms, st, n = measure(cfg, d, pattern, order, k, queue, reps=1)
+        print(json.dumps({"config": name, "pattern": pattern, "order": order, "k": k, "queue": queue,
+                          "join_ms": ms}))
         return
     names = sys.argv[1:] or ["c2k64", "c3k64", "c4k32", "c5"]
     for name in names:
         cfg = workloads.get_config(name)
         d = torch.from_numpy(cfg.points()).cuda()
-        for label, pattern, order, k in VARIANTS:
-            ms, st, n = measure(cfg, d, pattern, order, k)
+        for label, pattern, order, k, queue in VARIANTS:
+            ms, st, n = measure(cfg, d, pattern, order, k, queue)
             print(json.dumps({"config": name, "variant": label, "pattern": pattern, "order": order, "k": k,
+                              "queue": queue,
                               "join_ms": round(ms, 4), "dist_calcs": st["dist_calcs"], "pairs": n}), flush=True)
 
 
