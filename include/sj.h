@@ -141,6 +141,25 @@ sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps);
  * SJ_EINVAL for an unknown pattern or order. */
 sj_handle *sj_create_ex(const double *points, uint64_t n, int dim, double eps, int pattern, int order);
 
+/* A spatial PARTITION of a larger self-join (data beyond one GPU's memory, or
+ * several GPUs without replication).  The caller cuts the global grid (cell side
+ * w = eps(1+2^-20), origin = the global per-dimension minimum) into slabs of whole cell columns
+ * along dimension 0 and gives each partition
+ *   points[0 .. n_query)  : its own points -- the QUERIES of this handle,
+ *   points[n_query .. n)  : its halo -- the points of the FIRST cell column of the next slab,
+ *                           candidates only (the LID-UNICOMP forward cells of a cell, P:174,
+ *                           Alg. 3, never lie more than one column ahead in dimension 0);
+ *   ids                   : the global id of every point (uint32[n], host or device), written
+ *                           into the output instead of input positions; NULL = positions;
+ *   origin                : host double[dim], the global grid origin (every coordinate must be
+ *                           >= it, else SJ_EINVAL), so all partitions' cells align.
+ * sj_self_join on the handle returns exactly the ordered pairs of the global join that this
+ * partition's queries own (both directions): the partitions' results are disjoint and
+ * their union is the global result.  Pattern LID-UNICOMP, order SortByWL.  A cell holding both
+ * query and halo points (a cut through a cell column) is rejected with SJ_EINVAL.  NULL on error. */
+sj_handle *sj_create_part(const double *points, const uint32_t *ids, uint64_t n, uint64_t n_query, int dim,
+                          double eps, const double *origin);
+
 /* Run (or continue) the self-join.
  *   out_pairs : caller-owned uint32[2*cap], interleaved (i, j) of 0-based input ids,
  *               host (pinned or pageable) or device memory; a device buffer must be

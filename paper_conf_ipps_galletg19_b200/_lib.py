@@ -66,6 +66,7 @@ _sig = {
     "sj_get_stats": (_int, [_vp, ctypes.POINTER(SJStats)]),
     "sj_export_index": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
     "sj_create_from_index": (_vp, [_vp, _u64]),
+    "sj_create_part": (_vp, [_vp, _vp, _u64, _u64, _int, _dbl, _vp]),
     "sj_forward_offsets": (_int, [_int, _vp, _u64]),
     "sj_slice_chunks": (_i64, [_u64, _int, _int, _vp, _u64]),
     "sj_batch_chunks": (_i64, [_u64, _u64, _u64, _int, _vp, _u64]),
@@ -74,6 +75,8 @@ _sig = {
     "sj_neighbor_csr": (_int, [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]),
 }
 for _n, (_r, _a) in _sig.items():
+    if os.environ.get("SJ_LIB_PATH") and not hasattr(_lib, _n):
+        continue  # an older experimental build (SJ_LIB_PATH) may lack newer entry points
     _f = getattr(_lib, _n)
     _f.restype = _r
     _f.argtypes = _a
@@ -152,6 +155,21 @@ def sj_create_ex(points, n=None, dim=None, eps=None, pattern: int = 0, order: in
     """sj_create_ex(points, eps, pattern=, order=) or (ptr, n, dim, eps, pattern, order)."""
     n, dim, eps = _shape(points, n, dim, eps)
     h = _lib.sj_create_ex(_ptr(points), int(n), int(dim), float(eps), int(pattern), int(order))
+    if not h:
+        raise SJError(SJ_EINVAL, sj_last_error())
+    return h
+
+
+def sj_create_part(points, ids, n_query: int, eps: float, origin) -> int:
+    """sj_create_part(points (n, dim) float64, ids (n,) uint32 or None, n_query, eps, origin (dim,)):
+    a partition of a larger join -- the first n_query rows are its queries, the rest its halo."""
+    import numpy as np
+
+    n, dim, eps = _shape(points, eps, None, None)
+    org = np.ascontiguousarray(np.asarray(origin, dtype=np.float64).reshape(-1))
+    if org.shape[0] != dim:
+        raise SJError(SJ_EINVAL, f"origin needs {dim} values")
+    h = _lib.sj_create_part(_ptr(points), _ptr(ids), int(n), int(n_query), int(dim), float(eps), org.ctypes.data)
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
     return h
@@ -249,9 +267,12 @@ class Handle:
     """Owning wrapper of an sj_handle*."""
 
     def __init__(self, points=None, eps: float | None = None, *, raw: int | None = None, pattern=None, order=None,
-                 **options):
+                 part=None, **options):
         if raw is not None:
             self.h = raw
+        elif part is not None:  # (ids, n_query, origin): a partition (sj_create_part)
+            ids, n_query, origin = part
+            self.h = sj_create_part(points, ids, n_query, eps, origin)
         elif pattern is None and order is None:
             self.h = sj_create(points, eps)
         else:

@@ -228,6 +228,11 @@ struct FwdGeom {
     int rows;   // rows of the cell pattern (see pattern_rows())
     int small;  // prod(nc) < 2^32: 32-bit lid arithmetic
     int full;   // GCG: the rows cover the whole 3^n neighbourhood incl. the home cell
+    // partitioned index (sj_create_part): a cell is a query cell iff its first member (lowest
+    // input id, the sort is stable) is < nq; halo cells get no runs and no workload
+    const uint32_t *idx;  // sorted position -> input id, or null (every cell is a query cell)
+    uint32_t nq;
+    unsigned int *mixed;  // set if a cell holds both query and halo points
 };
 
 struct BuildTotals {
@@ -350,17 +355,22 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
     if (LPC == 1 ? valid : __any_sync(0xffffffffu, valid)) {
         long long c[SJ_MAX_DIM];
         uint32_t m = 0, out = 0;
+        bool qcell = valid;
         if (valid) {
             decode_lid(cell_lid[r], g, c);
             m = cell_start[r + 1] - cell_start[r];
             if (FILL) out = rbegin[r];
+            if (g.idx) {
+                qcell = g.idx[cell_start[r]] < g.nq;
+                if (!FILL && sub == 0 && qcell != (g.idx[cell_start[r + 1] - 1] < g.nq)) atomicOr(g.mixed, 1u);
+            }
         }
         uint32_t cnt = 0;
         unsigned long long summ = 0;
         for (int jb = 0; jb < g.rows; jb += LPC) {
             const int j = jb + (int)sub;
             uint32_t b = 0, len = 0;
-            const bool found = valid && j < g.rows && eval_row(j, c, g, L, cell_start, b, len);
+            const bool found = qcell && j < g.rows && eval_row(j, c, g, L, cell_start, b, len);
             if (FILL) {
                 if (LPC == 1) {
                     if (found) runs[out++] = make_uint2(b, len);
@@ -384,7 +394,10 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
             }
             if (valid && sub == 0) {
                 rcnt[r] = cnt;
-                if (g.full) {  // GCG: every candidate of the 3^n neighbourhood but the query itself
+                if (!qcell) {  // halo cell (partitioned index): candidates only
+                    w = 0;
+                    calcs = 0;
+                } else if (g.full) {  // GCG: every candidate of the 3^n neighbourhood but the query itself
                     w = (uint32_t)(summ - 1);
                     calcs = (unsigned long long)m * (summ - 1);
                 } else {       // half patterns: ceil((m-1)/2) = floor(m/2) home + the forward runs
@@ -420,11 +433,14 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
 }
 
 // a8 (SortByWL): key = max_w - W so an ascending stable sort gives non-increasing W
+// (partitioned index: halo cells get max_w + 1, so they sort after every query cell and the
+// queries occupy D' positions [0, nq))
 __global__ void __launch_bounds__(kThreads) wl_keys_kernel(const uint32_t *wload, uint64_t M, uint32_t max_w,
-                                                           uint32_t *keys, uint32_t *vals) {
+                                                           uint32_t *keys, uint32_t *vals, const uint32_t *cell_start,
+                                                           const uint32_t *idx, uint32_t nq) {
     uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= M) return;
-    keys[r] = max_w - wload[r];
+    keys[r] = (idx && idx[cell_start[r]] >= nq) ? max_w + 1u : max_w - wload[r];
     vals[r] = (uint32_t)r;
 }
 
@@ -441,11 +457,18 @@ __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t
                                                                   const uint32_t *wload,
                                                                   const unsigned long long *cell_lid, uint64_t M,
                                                                   int full, uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
-                                                                  uint64_t *lid_q) {
+                                                                  uint64_t *lid_q, const uint32_t *idx, uint32_t nq) {
     uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= M) return;
     uint32_t r = qorder[i];
     uint32_t m = cell_start[r + 1] - cell_start[r];
+    if (idx && idx[cell_start[r]] >= nq) {  // halo cell: never queued (m = 0 in its record)
+        cellq[i] = make_uint4(cell_start[r], 0u, rbegin[r], 0u);
+        r2q[r] = (uint32_t)i;
+        qbr[r] = qb[i];
+        lid_q[i] = cell_lid[r];
+        return;
+    }
     // {begin in the lid-ordered storage, m, first run, S = sum of the runs' lengths}
     // (half patterns: W = floor(m/2) + S; GCG: W = S - 1, the query itself excluded)
     cellq[i] = make_uint4(cell_start[r], m, rbegin[r], full ? wload[r] + 1 : wload[r] - m / 2);
@@ -461,7 +484,7 @@ __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, ui
                                                            const uint32_t *idx_sorted, const uint32_t *cellof,
                                                            const uint32_t *cell_start, const uint32_t *qbr,
                                                            const uint32_t *r2q, double *pts, uint32_t *orig,
-                                                           uint2 *qmap, int input_order) {
+                                                           uint2 *qmap, int input_order, const uint32_t *ids) {
     uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
     const uint32_t r = cellof[p];
@@ -471,7 +494,7 @@ __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, ui
     } else {
         for (int d = 0; d < pad; ++d) pts[p * pad + d] = d < dim ? raw[(uint64_t)src * dim + d] : 0.0;
     }
-    orig[p] = src;
+    orig[p] = ids ? ids[src] : src;  // partitioned index: the caller's global ids
     const uint64_t dest = input_order ? (uint64_t)src : (uint64_t)qbr[r] + (p - cell_start[r]);
     qmap[dest] = make_uint2((uint32_t)p, r2q[r]);
 }
@@ -508,6 +531,7 @@ struct CellChunkLoad {
     uint32_t big_min;
     __device__ unsigned operator()(uint64_t i) const {
         const uint32_t beg = qb[i], m = cellq[i].y;
+        if (m == 0) return 0;  // halo cell of a partitioned index: not queued
         if (m >= big_min) return (m + kChunk - 1) / kChunk;
         unsigned c = (beg + m + kChunk - 1) / kChunk - (beg + kChunk - 1) / kChunk;
         if (beg % kChunk != 0 && i > 0 && cellq[i - 1].y >= big_min) ++c;
@@ -726,9 +750,11 @@ static int rle(const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *ce
 }
 
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s, cudaEvent_t ev0,
-                cudaEvent_t ev1, float *ms) {
+                cudaEvent_t ev1, float *ms, const BuildPart *part) {
     Temps tmp(s);
     ix.n = n;
+    const uint64_t nq = part ? part->n_query : n;  // queries: input points [0, nq)
+    ix.n_query = nq;
     ix.dim = dim;
     ix.pad = dim == 1 ? 1 : ((dim + 1) & ~1);
     ix.eps = eps;
@@ -776,6 +802,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     for (int d = 0; d < dim; ++d) {
         double mn = from_ordered_key(bb.mn[d]);
         double mx = from_ordered_key(bb.mx[d]);
+        if (part) {  // partition of a larger grid: its origin, so the cells of all partitions align
+            if (!(part->origin[d] <= mn) || !std::isfinite(part->origin[d])) {
+                set_error("sj_create_part: a coordinate in dimension %d lies below the grid origin", d);
+                return SJ_EINVAL;
+            }
+            mn = part->origin[d];
+        }
         ix.mins[d] = mn;
         geo.mins[d] = mn;
         // nc_d = max c_d + 1; c_d is monotone in x_d so max c_d = c_d(max x_d)
@@ -853,6 +886,14 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     fg.rows = R;
     fg.small = ncells_total <= 0xFFFFFFFFull ? 1 : 0;
     fg.full = ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
+    unsigned int *d_mixed = nullptr;
+    if (part) {
+        SJ_TRY(tmp.alloc(&d_mixed, 1));
+        SJ_CUDA_TRY(cudaMemsetAsync(d_mixed, 0, sizeof(unsigned int), s));
+        fg.idx = idx_sorted;
+        fg.nq = (uint32_t)nq;
+        fg.mixed = d_mixed;
+    }
     for (int d = 0; d < dim; ++d) {
         fg.nc[d] = ix.nc[d];
         fg.stride[d] = ix.stride[d];
@@ -874,30 +915,47 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin;
     SJ_TRY(tmp.alloc(&rbegin, n + 1));
+    // host round trip 2: M, plus the workload totals (max W sizes the SortByWL keys, D_alg)
     SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_M, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 64, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
+    if (d_mixed) SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 128, d_mixed, sizeof(unsigned int), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
     debug_mark("build: sort+rle+runcount sync");
     uint64_t M;
     memcpy(&M, mail, sizeof M);
     ix.n_cells = M;
+    BuildTotals bt;
+    memcpy(&bt, (char *)mail + 64, sizeof bt);
+    if (d_mixed) {
+        unsigned int mixed = 0;
+        memcpy(&mixed, (char *)mail + 128, sizeof mixed);
+        if (mixed) {
+            set_error("sj_create_part: a grid cell holds both query and halo points (partition the data by "
+                      "whole cell columns)");
+            return SJ_EINVAL;
+        }
+    }
+    ix.dist_calcs = bt.dist_calcs;
+    ix.max_w = bt.max_w;
     uint32_t *d_E32;
     SJ_TRY(tmp.alloc(&d_E32, 1));
     SJ_CUDA_TRY(cudaMemsetAsync(rcnt + M, 0, sizeof(uint32_t), s));
     SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, rbegin + M, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    SJ_CUDA_TRY(cudaStreamSynchronize(s));
-    debug_mark("build: scan sync");
-    BuildTotals bt;
-    memcpy(&bt, mail, sizeof bt);
-    uint32_t E32;
-    memcpy(&E32, (char *)mail + 256, sizeof E32);
-    const uint64_t E = E32;
-    ix.n_runs = E;
-    ix.dist_calcs = bt.dist_calcs;
-    ix.max_w = bt.max_w;
-
-    SJ_TRY(dev_alloc_t(&ix.runs, E + 2, s));
+    // The runs array is allocated at its bound M * rows when that is small (every 1-D..4-D
+    // index), so the run total E is read with the final round trip instead of a third one.
+    const uint64_t runs_bound = M * (uint64_t)R + 2;
+    const bool bounded = runs_bound * sizeof(uint2) <= (256ull << 20);
+    uint64_t E = 0;
+    if (!bounded) {
+        SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        SJ_CUDA_TRY(cudaStreamSynchronize(s));
+        debug_mark("build: scan sync");
+        uint32_t E32;
+        memcpy(&E32, (char *)mail + 256, sizeof E32);
+        E = E32;
+        ix.n_runs = E;
+    }
+    SJ_TRY(dev_alloc_t(&ix.runs, bounded ? runs_bound : E + 2, s));
     if (wide)
         runs_kernel<true, 32><<<grid_for(M * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
                                                                     rbegin, ix.runs, nullptr);
@@ -913,10 +971,12 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wv, M));
     SJ_TRY(tmp.alloc(&wk2, M));
     SJ_TRY(tmp.alloc(&wv2, M));
-    wl_keys_kernel<<<grid_for(M), kThreads, 0, s>>>(wload, M, ix.max_w, wk, wv);
+    wl_keys_kernel<<<grid_for(M), kThreads, 0, s>>>(wload, M, ix.max_w, wk, wv, cell_start, part ? idx_sorted : nullptr,
+                                                    (uint32_t)nq);
     note_launch();
     if (ix.order == SJ_ORDER_WORKLOAD) {
-        SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(ix.max_w), &qorder_keys, &qorder, s));
+        SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(part ? ix.max_w + 1ull : ix.max_w), &qorder_keys, &qorder,
+                              s));
     } else {  // ablation orders: cells stay in lid order (no SortByWL)
         qorder_keys = wk;
         qorder = wv;
@@ -938,10 +998,12 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&r2q, M));
     SJ_TRY(tmp.alloc(&qbr, M));
     cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, rbegin, wload, cell_lid, M,
-                                                           fg.full, ix.cellq, r2q, qbr, ix.cell_lid);
+                                                           fg.full, ix.cellq, r2q, qbr, ix.cell_lid,
+                                                           part ? idx_sorted : nullptr, (uint32_t)nq);
     note_launch();
     permute_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, dim, ix.pad, idx_sorted, cellof, cell_start, qbr, r2q,
-                                                    ix.pts, ix.orig, ix.qmap, ix.order == SJ_ORDER_INPUT ? 1 : 0);
+                                                    ix.pts, ix.orig, ix.qmap, ix.order == SJ_ORDER_INPUT ? 1 : 0,
+                                                    part ? part->d_ids : nullptr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
@@ -956,8 +1018,9 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
                           ChunkDone{n, ix.chunks, d_nc}));
     else
         SJ_TRY(scan_fused(M, CellChunkLoad{ix.cellq, qb, big_min}, CellChunkStore{ix.cellq, qb, big_min, ix.chunks}, s,
-                          ChunkDone{n, ix.chunks, d_nc}));
+                          ChunkDone{nq, ix.chunks, d_nc}));
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if (bounded) SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
     debug_mark("build: tail issued");
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
@@ -966,6 +1029,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     uint32_t nchunks;
     memcpy(&nchunks, (char *)mail + 512, sizeof nchunks);
     ix.n_chunks = nchunks;
+    if (bounded) {
+        uint32_t E32;
+        memcpy(&E32, (char *)mail + 256, sizeof E32);
+        ix.n_runs = E32;
+    }
     return SJ_OK;
 }
 

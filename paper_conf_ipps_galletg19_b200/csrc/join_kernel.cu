@@ -663,6 +663,55 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
     }
 }
 
+#ifndef SJ_HOMEWIN
+#define SJ_HOMEWIN 1
+#endif
+// Home cell of at most 32 points (one staged tile, tb = 0): instead of evaluating every
+// (query, slot) pair of the tile and masking half of them out (tile_rounds<HOME>), lane t of
+// a group evaluates only the query's circulant window (reading c8): window offsets i = t,
+// t+k, ... < home_count(m, rr) <= 16, slot (rr + 1 + i) mod m read from shared memory.
+template <int DIM, int K, int MODE, bool GCG>
+__device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned nq, unsigned m, WarpSmem<DIM, MODE> &ws,
+                                                   int b, int &nbuf, unsigned long long &nhits, int lane, unsigned lt) {
+    constexpr int PAD = PointPad<DIM>::value;
+    constexpr int QPW = 32 / K;
+    constexpr int WS = (16 + K - 1) / K;  // window slots per lane
+    const double *tile = ws.tile[b];
+    const unsigned *tile_orig = ws.tile_orig[b];
+    const int grp = lane / K;
+    const unsigned t = (unsigned)(lane % K);
+    const unsigned gbits = K == 32 ? kFull : (((1u << K) - 1u) << (lane & ~(K - 1)));
+    for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+        const unsigned qi = (r0 + grp) & 31;
+        const bool qv = r0 + grp < nq;
+        double qq[DIM];
+        load_smem_point<DIM>(ws.qry + qi * PAD, qq);
+        const unsigned oq = ws.qorig[qi];
+        const unsigned rr = ws.qrr[qi];
+        const unsigned hl = home_count(m, rr);
+        unsigned long long cur = 0;
+        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * WS, a, lane, &ws.wcur);
+        double cp[WS][DIM];
+        unsigned co[WS];
+        bool ok[WS], close[WS];
+#pragma unroll
+        for (int s = 0; s < WS; ++s) {
+            const unsigned i = t + (unsigned)(K * s);
+            ok[s] = qv && i < hl;
+            unsigned p = rr + 1u + i;
+            if (p >= m) p -= m;
+            p &= 31u;
+            load_smem_point<DIM>(tile + p * PAD, cp[s]);
+            co[s] = tile_orig[p];
+        }
+#pragma unroll
+        for (int s = 0; s < WS; ++s) close[s] = sqdist<DIM>(qq, cp[s]) <= a.e2;
+#pragma unroll
+        for (int s = 0; s < WS; ++s)
+            emit<DIM, MODE, GCG>(close[s] & ok[s], oq, co[s], ws.buf, nbuf, nhits, lt, gbits, cur, a, lane);
+    }
+}
+
 // Tiled path: all nq queries of the chunk lie in one cell (hb, m, runs rb.., S forward
 // candidates).  The forward runs, then the home cell, are staged 32 candidates at a time in
 // shared memory (points + input ids); lane t of a group holds tile slots t, t+k, ... and
@@ -749,6 +798,15 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         return;
     }
     stage_home(0, 0);
+    if constexpr (SJ_HOMEWIN && !GCG && DIM <= 3 && K >= 4 && MODE != kRows && MODE != kDegree) {
+        if (m <= 32u) {  // one tile: evaluate the circulant windows only
+            cp_async_wait<0>();
+            __syncwarp();
+            home_window_rounds<DIM, K, MODE, GCG>(a, nq, m, ws, 0, nbuf, nhits, lane, lt);
+            __syncwarp();
+            return;
+        }
+    }
     it = 0;
     for (unsigned tb = 0; tb < m; tb += 32, ++it) {
         const bool more = tb + 32 < m;

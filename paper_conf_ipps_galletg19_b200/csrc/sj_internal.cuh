@@ -113,15 +113,26 @@ struct Index {
     uint64_t *cell_lid = nullptr; // [M]      queue-order cell -> linear id (export / tests)
     uint32_t *chunks = nullptr; // [C+1]      WorkQueue chunk c = D' positions [chunks[c], chunks[c+1])
     uint64_t n_chunks = 0;      // C
+    uint64_t n_query = 0;       // queries: D' positions [0, n_query) (n unless partitioned)
 };
 
 struct BuildTimes {
     float ms = 0;
 };
 
+// Spatial partition of a join (sj_create_part): the grid origin is given (the
+// global per-dimension minimum, so every partition's cells align), only the first n_query
+// points are queries (the rest is the halo: candidates only), and the output carries the
+// caller's global ids.
+struct BuildPart {
+    double origin[SJ_MAX_DIM];
+    const uint32_t *d_ids = nullptr;  // [n] device, or null (ids = input positions)
+    uint64_t n_query = 0;
+};
+
 // Builds the index from device-resident raw points (n x dim AoS).  Returns sj_status.
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s,
-                cudaEvent_t ev0, cudaEvent_t ev1, float *ms);
+                cudaEvent_t ev0, cudaEvent_t ev1, float *ms, const BuildPart *part = nullptr);
 void free_index(Index &ix, cudaStream_t s);
 // LID-UNICOMP forward offsets (host): F = (3^dim - 1)/2 offsets, int8 each dim.
 int forward_offsets_public(int dim, int8_t *out, uint64_t cap);
