@@ -121,7 +121,7 @@ typedef struct sj_stats {
     uint32_t tiled_min;       /* smallest cell (points) that gets shared-memory tiles */
     uint32_t pattern;         /* enum sj_pattern of the index                        */
     uint32_t order;           /* enum sj_order of the index                          */
-    uint32_t reserved;
+    uint32_t est_fused;       /* 1 if the estimator (a9) ran fused into the in-place join */
 } sj_stats;
 
 /* Build the eps-grid index of `n` points of dimension `dim` (row-major AoS,

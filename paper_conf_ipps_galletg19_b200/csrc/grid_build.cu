@@ -42,20 +42,13 @@ __host__ __device__ inline double from_ordered_key(unsigned long long k) {
     return d;
 }
 
+// Zero-initialised (it lives in the build workspace's pre-zeroed region): the minimum is kept
+// as the maximum of the complemented ordered key, so 0 is the neutral element of both.
 struct BBox {
-    unsigned long long mn[SJ_MAX_DIM];
+    unsigned long long mn_c[SJ_MAX_DIM];  // ~ordered_key(min)
     unsigned long long mx[SJ_MAX_DIM];
     unsigned int nonfinite;
 };
-
-__global__ void bbox_init_kernel(BBox *bb) {
-    int t = threadIdx.x;
-    if (t < SJ_MAX_DIM) {
-        bb->mn[t] = ~0ull;
-        bb->mx[t] = 0ull;
-    }
-    if (t == 0) bb->nonfinite = 0;
-}
 
 // a2: exact per-dimension min/max (order-independent) + non-finite check (a1 validation).
 // The coordinates are read as a flat array of double2; the total thread count T is chosen
@@ -83,7 +76,7 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
         const double x = raw[total - 1];
         bad |= !isfinite(x);
         const unsigned long long k = ordered_key(x);
-        atomicMin(&bb->mn[dim - 1], k);
+        atomicMax(&bb->mn_c[dim - 1], ~k);
         atomicMax(&bb->mx[dim - 1], k);
     }
     // block reduction per dimension in shared memory, then ONE atomic per dimension and block
@@ -104,7 +97,7 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
     if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) s_bad = 1;
     __syncthreads();
     if (threadIdx.x < (unsigned)dim) {
-        atomicMin(&bb->mn[threadIdx.x], s_mn[threadIdx.x]);
+        atomicMax(&bb->mn_c[threadIdx.x], ~s_mn[threadIdx.x]);
         atomicMax(&bb->mx[threadIdx.x], s_mx[threadIdx.x]);
     }
     if (threadIdx.x == 0 && s_bad) atomicOr(&bb->nonfinite, 1u);
@@ -352,6 +345,7 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
     unsigned long long calcs = 0;
     uint32_t w = 0;
     const bool valid = r < M;  // uniform across the LPC lanes of a cell
+    if (!FILL && r == M && sub == 0) rcnt[M] = 0;  // the scan runs over M + 1 entries
     if (LPC == 1 ? valid : __any_sync(0xffffffffu, valid)) {
         long long c[SJ_MAX_DIM];
         uint32_t m = 0, out = 0;
@@ -619,6 +613,8 @@ int forward_offsets_public(int dim, int8_t *out, uint64_t cap) {
 }
 
 void free_index(Index &ix, cudaStream_t s) {
+    dev_free(ix.d_meta, s);
+    ix.d_meta = nullptr;
     dev_free(ix.pts, s);
     dev_free(ix.orig, s);
     dev_free(ix.qmap, s);
@@ -705,19 +701,48 @@ static int pattern_rows(int dim, int pattern, std::vector<uint64_t> &rows) {
 }
 
 namespace {
-// RAII list of temporaries freed on the stream at scope exit.
+// The build's temporaries: one stream-ordered block (Workspace: bump region + pre-zeroed
+// region), freed on the stream at scope exit; requests that do not fit fall back to the pool.
 struct Temps {
     cudaStream_t s;
-    std::vector<void *> ptrs;
+    Workspace ws;
+    void *block = nullptr;
+    std::vector<void *> ptrs;  // fallback allocations
     explicit Temps(cudaStream_t st) : s(st) {}
     ~Temps() {
         for (void *p : ptrs) dev_free(p, s);
+        dev_free(block, s);
+    }
+    int reserve(size_t bytes, size_t zbytes) {
+        bytes = Workspace::round(bytes);
+        zbytes = Workspace::round(zbytes);
+        SJ_TRY(dev_alloc(&block, bytes + zbytes, s));
+        ws.base = static_cast<char *>(block);
+        ws.cap = bytes;
+        ws.zbase = ws.base + bytes;
+        ws.zcap = zbytes;
+        SJ_CUDA_TRY(cudaMemsetAsync(ws.zbase, 0, zbytes, s));
+        return SJ_OK;
     }
     template <class T>
     int alloc(T **p, size_t count) {
+        if (void *q = ws.take(count * sizeof(T) + 16)) {
+            *p = static_cast<T *>(q);
+            return SJ_OK;
+        }
         int rc = dev_alloc_t(p, count, s);
         if (rc == SJ_OK) ptrs.push_back(*p);
         return rc;
+    }
+    template <class T>
+    int alloc_zero(T **p, size_t count) {  // zero-filled
+        if (void *q = ws.take_zero(count * sizeof(T))) {
+            *p = static_cast<T *>(q);
+            return SJ_OK;
+        }
+        SJ_TRY(alloc(p, count));
+        SJ_CUDA_TRY(cudaMemsetAsync(*p, 0, count * sizeof(T), s));
+        return SJ_OK;
     }
 };
 }  // namespace
@@ -735,22 +760,21 @@ static int sort_points(Temps &tmp, const double *d_raw, uint64_t n, const GridGe
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     if constexpr (sizeof(K) == 4)
-        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s));
+        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws));
     else
-        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s));
+        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws));
     return SJ_OK;
 }
 
 template <class K>
 static int rle(const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *cell_lid, uint32_t *cell_start,
-               uint64_t *d_M, cudaStream_t s) {
-    SJ_CUDA_TRY(cudaMemsetAsync(d_M, 0, sizeof(uint64_t), s));
+               uint64_t *d_M, cudaStream_t s, Workspace *ws) {  // d_M: zero-filled
     return scan_fused(n, RleLoad<K>{ks}, RleStore<K>{ks, cellof, cell_lid, cell_start}, s,
-                      RleDone{n, cell_start, d_M});
+                      RleDone{n, cell_start, d_M}, ws);
 }
 
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s, cudaEvent_t ev0,
-                cudaEvent_t ev1, float *ms, const BuildPart *part) {
+                cudaEvent_t ev1, float *ms, const BuildPart *part, uint64_t *tail_mail) {
     Temps tmp(s);
     ix.n = n;
     const uint64_t nq = part ? part->n_query : n;  // queries: input points [0, nq)
@@ -771,11 +795,19 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         ~MailFree() { pinned_release(p); }
     } mail_free{mail};
 
+    // One workspace for every temporary (upper bounds from n; M <= n): sort keys/values
+    // (8-byte keys at most), the per-point and per-cell arrays, the radix histograms; the
+    // zeroed region holds the counters and every scan's look-back status words.
+    {
+        const uint64_t tiles = (n + 2047) / 2048 + 1;
+        const size_t bytes = (size_t)n * 84 + (size_t)2 * 256 * 4 * tiles + 64 * 512;
+        const size_t zbytes = (size_t)8 * (12 * tiles + 64) + 48 * 512;
+        SJ_TRY(tmp.reserve(bytes, zbytes));
+    }
+
     // ---- a2: bounding box + non-finite check
     BBox *d_bb;
-    SJ_TRY(tmp.alloc(&d_bb, 1));
-    bbox_init_kernel<<<1, 32, 0, s>>>(d_bb);
-    note_launch();
+    SJ_TRY(tmp.alloc_zero(&d_bb, 1));
     {
         // 2 * threads must be a multiple of dim (see bbox_kernel): blocks a multiple of dim
         const uint64_t pairs = n * (uint64_t)dim / 2;
@@ -800,7 +832,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     geo.w = ix.w;
     unsigned __int128 total = 1;
     for (int d = 0; d < dim; ++d) {
-        double mn = from_ordered_key(bb.mn[d]);
+        double mn = from_ordered_key(~bb.mn_c[d]);
         double mx = from_ordered_key(bb.mx[d]);
         if (part) {  // partition of a larger grid: its origin, so the cells of all partitions align
             if (!(part->origin[d] <= mn) || !std::isfinite(part->origin[d])) {
@@ -841,18 +873,18 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&cellof, n));
     SJ_TRY(tmp.alloc(&cell_lid, n));
     SJ_TRY(tmp.alloc(&cell_start, n + 1));
-    SJ_TRY(tmp.alloc(&d_M, 1));
+    SJ_TRY(tmp.alloc_zero(&d_M, 1));
     // lid -> rank lookup: a dense table when prod(nc) is small, else a hash table
     Lookup L{};
     const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
     if (ix.key_bits <= 32) {
         uint32_t *ks;
         SJ_TRY(sort_points<uint32_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
-        SJ_TRY(rle<uint32_t>(ks, n, cellof, cell_lid, cell_start, d_M, s));
+        SJ_TRY(rle<uint32_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
     } else {
         uint64_t *ks;
         SJ_TRY(sort_points<uint64_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
-        SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s));
+        SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
     }
     if (dense) {
         uint32_t *tab;
@@ -880,7 +912,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // ---- a6 + a7: forward runs, workload, D_alg
     std::vector<uint64_t> rows;
     const int R = pattern_rows(dim, ix.pattern, rows);
-    SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, rows.data(), R * sizeof(uint64_t), 0, cudaMemcpyHostToDevice, s));
+    if (R * sizeof(uint64_t) <= 2048) {  // through the pinned mailbox: a truly asynchronous copy
+        memcpy((char *)mail + 1024, rows.data(), R * sizeof(uint64_t));
+        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, (char *)mail + 1024, R * sizeof(uint64_t), 0,
+                                            cudaMemcpyHostToDevice, s));
+    } else {
+        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, rows.data(), R * sizeof(uint64_t), 0, cudaMemcpyHostToDevice, s));
+    }
     FwdGeom fg{};
     fg.dim = dim;
     fg.rows = R;
@@ -888,8 +926,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     fg.full = ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
     unsigned int *d_mixed = nullptr;
     if (part) {
-        SJ_TRY(tmp.alloc(&d_mixed, 1));
-        SJ_CUDA_TRY(cudaMemsetAsync(d_mixed, 0, sizeof(unsigned int), s));
+        SJ_TRY(tmp.alloc_zero(&d_mixed, 1));
         fg.idx = idx_sorted;
         fg.nq = (uint32_t)nq;
         fg.mixed = d_mixed;
@@ -902,15 +939,15 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     BuildTotals *d_tot;
     SJ_TRY(tmp.alloc(&rcnt, n + 1));
     SJ_TRY(tmp.alloc(&wload, n));
-    SJ_TRY(tmp.alloc(&d_tot, 1));
-    SJ_CUDA_TRY(cudaMemsetAsync(d_tot, 0, sizeof(BuildTotals), s));
+    SJ_TRY(tmp.alloc_zero(&d_tot, 1));
     const bool wide = R >= 16;  // one warp per cell for many rows
+    // (n + 1 cells' worth of threads: the one with r == M zeroes rcnt[M] for the scan below)
     if (wide)
-        runs_kernel<false, 32><<<grid_for(n * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                     nullptr, nullptr, d_tot);
+        runs_kernel<false, 32><<<grid_for((n + 1) * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt,
+                                                                           wload, nullptr, nullptr, d_tot);
     else
-        runs_kernel<false, 1><<<grid_for(n), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload, nullptr,
-                                                               nullptr, d_tot);
+        runs_kernel<false, 1><<<grid_for(n + 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
+                                                                   nullptr, nullptr, d_tot);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin;
@@ -937,10 +974,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     }
     ix.dist_calcs = bt.dist_calcs;
     ix.max_w = bt.max_w;
-    uint32_t *d_E32;
-    SJ_TRY(tmp.alloc(&d_E32, 1));
-    SJ_CUDA_TRY(cudaMemsetAsync(rcnt + M, 0, sizeof(uint32_t), s));
-    SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s));
+    // persistent device words {n_chunks, E}: the join reads the chunk count from here (a
+    // device-sized launch needs no host round trip after the build)
+    SJ_TRY(dev_alloc_t(&ix.d_meta, 4, s));
+    uint32_t *d_E32 = ix.d_meta + 1;
+    SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s, &tmp.ws));
     // The runs array is allocated at its bound M * rows when that is small (every 1-D..4-D
     // index), so the run total E is read with the final round trip instead of a third one.
     const uint64_t runs_bound = M * (uint64_t)R + 2;
@@ -955,7 +993,8 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         E = E32;
         ix.n_runs = E;
     }
-    SJ_TRY(dev_alloc_t(&ix.runs, bounded ? runs_bound : E + 2, s));
+    ix.runs_cap = bounded ? runs_bound : E + 2;
+    SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
     if (wide)
         runs_kernel<true, 32><<<grid_for(M * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
                                                                     rbegin, ix.runs, nullptr);
@@ -976,7 +1015,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     note_launch();
     if (ix.order == SJ_ORDER_WORKLOAD) {
         SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(part ? ix.max_w + 1ull : ix.max_w), &qorder_keys, &qorder,
-                              s));
+                              s, &tmp.ws));
     } else {  // ablation orders: cells stay in lid order (no SortByWL)
         qorder_keys = wk;
         qorder = wv;
@@ -986,7 +1025,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&qb, M));
     queue_m_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, cell_start, M, mq);
     note_launch();
-    SJ_TRY(scan_exclusive_u32(mq, qb, M, nullptr, s));
+    SJ_TRY(scan_exclusive_u32(mq, qb, M, nullptr, s, &tmp.ws));
 
     // ---- final arrays
     SJ_TRY(dev_alloc_t(&ix.cellq, M, s));
@@ -1008,17 +1047,28 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_CUDA_TRY(cudaGetLastError());
 
     // ---- WorkQueue chunks over D'
-    uint32_t *d_nc;
-    SJ_TRY(tmp.alloc(&d_nc, 1));
+    uint32_t *d_nc = ix.d_meta;
     SJ_TRY(dev_alloc_t(&ix.chunks, n + 1, s));
     // in input order a cell's points are scattered: no chunk may claim a cell
     const uint32_t big_min = ix.order == SJ_ORDER_INPUT ? 0xFFFFFFFFu : kBigCell;
     if (ix.order == SJ_ORDER_INPUT)
         SJ_TRY(scan_fused(n, ChunkLoad{ix.qmap, ix.cellq, qb, big_min}, ChunkStore{ix.chunks}, s,
-                          ChunkDone{n, ix.chunks, d_nc}));
+                          ChunkDone{n, ix.chunks, d_nc}, &tmp.ws));
     else
         SJ_TRY(scan_fused(M, CellChunkLoad{ix.cellq, qb, big_min}, CellChunkStore{ix.cellq, qb, big_min, ix.chunks}, s,
-                          ChunkDone{nq, ix.chunks, d_nc}));
+                          ChunkDone{nq, ix.chunks, d_nc}, &tmp.ws));
+    if (tail_mail) {
+        // no final round trip: {n_chunks, E} land in the caller's pinned mailbox, read once the
+        // stream has passed ev1 (the join reads n_chunks on the device meanwhile)
+        tail_mail[0] = tail_mail[1] = 0;
+        SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        if (bounded)
+            SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail + 1, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        else
+            tail_mail[1] = E;
+        if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
+        return SJ_OK;
+    }
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (bounded) SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));

@@ -75,6 +75,20 @@ struct BufCap {
 };
 
 // Per-warp shared memory: emission buffer, the chunk's queries, one candidate tile.
+// Per-warp control words (shared memory, lane 0 writes).
+struct WarpCtl {
+    // kExact: next output slot of the current chunk; kPairs: nonzero once a flush of this warp
+    // found the output full (the warp stops dequeuing: the caller re-runs the join staged)
+    unsigned long long wcur;
+    // kPairs with the fused estimator (a9): hits this warp has flushed so far, and its
+    // hits in the sample chunks, taken when it first dequeues a chunk past the sample (a warp
+    // meets its chunks in increasing order), so no state is live across a chunk
+    unsigned long long wtot, samp;
+    unsigned sclosed;
+    unsigned long long sv1;  // end of the fused estimator's sample (virtual chunks [0, sv1))
+    unsigned vcount;         // the batch's virtual chunks (in shared memory: no register in the loops)
+};
+
 template <int DIM, int MODE>
 struct WarpSmem {
     static constexpr int PAD = PointPad<DIM>::value;
@@ -90,9 +104,7 @@ struct WarpSmem {
     // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
     // and the smaller footprint buys occupancy)
     alignas(16) uint2 buf[Mode<MODE>::pairs ? ((SJ_COLS && DIM <= 3) ? kColRows * kColPitch : BufCap<DIM>::value) : 2];
-    // kExact: next output slot of the current chunk; kPairs: nonzero once a flush of this warp
-    // found the output full (the warp stops dequeuing: the caller re-runs the join staged)
-    unsigned long long wcur;
+    WarpCtl ctl;
     unsigned snext;  // SortByWL only (static assignment): this warp's next chunk index
     // kRows: the segment's per-query row cursors; kDegree: their running neighbour counts
     unsigned long long qcur[(MODE == kRows || MODE == kDegree) ? 32 : 1];
@@ -187,17 +199,18 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
 // order is deterministic; the counter still totals the pairs.
 template <bool GCG, bool EXACT>
 __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane,
-                                      unsigned long long *wcur) {
+                                      WarpCtl *wc) {
     __syncwarp();
     constexpr unsigned long long kPer = GCG ? 1ull : 2ull;  // pairs per buffered hit
     unsigned long long base = 0;
     if (lane == 0) {
         base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)nbuf);
+        wc->wtot += (unsigned long long)nbuf;
         if (EXACT) {
-            base = *wcur;
-            *wcur = base + kPer * (unsigned long long)nbuf;
+            base = wc->wcur;
+            wc->wcur = base + kPer * (unsigned long long)nbuf;
         } else if (base + kPer * (unsigned long long)nbuf > a.out_cap) {
-            *wcur = 1;  // overflow: stop dequeuing
+            wc->wcur = 1;  // overflow: stop dequeuing
         }
     }
     base = __shfl_sync(kFull, base, 0);
@@ -250,7 +263,7 @@ __device__ __forceinline__ unsigned col_base(const uint2 *buf, int lane) {
 
 template <bool GCG, bool EXACT>
 __device__ __forceinline__ void flush_cols(const uint2 *buf, int &nbuf, const JoinArgs &a, int lane,
-                                           unsigned long long *wcur) {
+                                           WarpCtl *wc) {
     __syncwarp();
     const unsigned col0 = col_base(buf, lane);
     const int cnt = (int)(((unsigned)nbuf - col0) / (8u * kColPitch));
@@ -266,11 +279,12 @@ __device__ __forceinline__ void flush_cols(const uint2 *buf, int &nbuf, const Jo
     unsigned long long base = 0;
     if (lane == 0) {
         base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)total);
+        wc->wtot += (unsigned long long)total;
         if (EXACT) {
-            base = *wcur;
-            *wcur = base + kPer * (unsigned long long)total;
+            base = wc->wcur;
+            wc->wcur = base + kPer * (unsigned long long)total;
         } else if (base + kPer * (unsigned long long)total > a.out_cap) {
-            *wcur = 1;  // overflow: stop dequeuing
+            wc->wcur = 1;  // overflow: stop dequeuing
         }
     }
     base = __shfl_sync(kFull, base, 0);
@@ -344,14 +358,14 @@ __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *
 // of 32; a column gains at most room/32).
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane,
-                                         unsigned long long *wcur) {
+                                         WarpCtl *wc) {
     constexpr int CAP = BufCap<DIM>::value;
     if constexpr (Cols<DIM, MODE>::value) {
         const unsigned lim = col_base(buf, lane) + 8u * kColPitch * (unsigned)(kColRows - room / 32);
-        if (__any_sync(kFull, (unsigned)nbuf > lim)) flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+        if (__any_sync(kFull, (unsigned)nbuf > lim)) flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
     } else if constexpr (Mode<MODE>::pairs) {
         if (nbuf > CAP - room) {
-            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
             nbuf = 0;
         }
     }
@@ -360,13 +374,13 @@ __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const 
 // Flush whatever is buffered (end of an exact-sizing chunk, end of the kernel).
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void flush_all(uint2 *buf, int &nbuf, const JoinArgs &a, int lane,
-                                          unsigned long long *wcur) {
+                                          WarpCtl *wc) {
     if constexpr (Cols<DIM, MODE>::value) {
         if (__any_sync(kFull, (unsigned)nbuf != col_base(buf, lane)))
-            flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+            flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
     } else if constexpr (Mode<MODE>::pairs) {
         if (nbuf > 0) {
-            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wcur);
+            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
             nbuf = 0;
         }
     }
@@ -480,7 +494,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                 if (GCG) hit = hit && cidx != qlid;  // GCG scans its own cell: skip (q, q)
                 i += K;
             }
-            flush_if<DIM, MODE, GCG>(buf, nbuf, 32, a, lane, &ws.wcur);
+            flush_if<DIM, MODE, GCG>(buf, nbuf, 32, a, lane, &ws.ctl);
             emit<DIM, MODE, GCG>(hit, oq, oc, buf, nbuf, nhits, lt, gbits, cur, a, lane);
         }
         if constexpr (MODE == kDegree) {  // the query's degree: its group's hits
@@ -538,7 +552,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             }
             unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
             const unsigned long long nh0 = nhits;
-            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.wcur);
+            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.ctl);
             // all SPL distances first (independent FP64 chains -> ILP), then the emissions;
             // evaluated unconditionally and masked after (invalid slots may hold stale or
             // uninitialised bits; FP64 arithmetic on them cannot trap)
@@ -592,7 +606,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 okb = okb & ((unsigned)db < home_count(m, rrb));
             }
             const bool ha = ca & oka, hb = cb & okb;
-            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
+            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.ctl);
             unsigned long long cura = 0, curb = 0;
             if constexpr (MODE == kRows) {
                 cura = ws.qcur[q0];
@@ -632,7 +646,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             const unsigned long long nh0 = nhits;
 #pragma unroll 2
             for (int s = 0; s < SPL; s += 2) {  // two slots per step: two independent FP64 chains
-                flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.wcur);
+                flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.ctl);
                 const unsigned j0 = t + (unsigned)(K * s), j1 = j0 + (unsigned)K;
                 double c0[DIM], c1[DIM];
                 load_smem_point<DIM>(tile + (j0 & 31) * PAD, c0);
@@ -690,7 +704,7 @@ __device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned n
         const unsigned rr = ws.qrr[qi];
         const unsigned hl = home_count(m, rr);
         unsigned long long cur = 0;
-        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * WS, a, lane, &ws.wcur);
+        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * WS, a, lane, &ws.ctl);
         double cp[WS][DIM];
         unsigned co[WS];
         bool ok[WS], close[WS];
@@ -833,13 +847,30 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     int nbuf = Cols<DIM, MODE>::value ? (int)col_base(ws.buf, lane) : 0;  // column modes: see flush_cols
     unsigned long long nhits = 0;
     unsigned long long ncalcs = 0;
-    if constexpr (MODE == kPairs) {
-        if (lane == 0) ws.wcur = 0;
-        __syncwarp();
-    }
-
     // The batch: virtual chunks v_begin, v_begin + v_stride, ... < v_end (contiguous, or the
-    // strided D'_l of the SortByWL-only batches); i indexes them.
+    // strided D'_l of the SortByWL-only batches); i indexes them.  A device-sized
+    // launch reads the build's chunk count here: V = the slice's chunks (rank, world).
+    if (lane == 0) {
+        unsigned vc = a.v_count;
+        unsigned long long sv1 = a.sample_v1;
+        if (a.d_nchunks) {
+            const unsigned nch = *a.d_nchunks;  // 32-bit arithmetic: no division subroutine
+            const unsigned long long V = nch > a.rank ? (nch - a.rank + a.world - 1u) / a.world : 0u;
+            vc = (unsigned)V;
+            if (a.sample_ppm) {  // the estimator's sample: the first ceil(V * ppm / 1e6) chunks
+                sv1 = (V * a.sample_ppm + 999999ull) / 1000000ull;
+                if (sv1 < 1) sv1 = 1;
+                if (sv1 > V) sv1 = V;
+            }
+        }
+        ws.ctl.vcount = vc;
+        ws.ctl.sv1 = sv1;
+        ws.ctl.wcur = ws.ctl.wtot = ws.ctl.samp = 0;
+        ws.ctl.sclosed = 0;
+    }
+    __syncwarp();
+    // a kernel parameter, not a register: the dequeue compares against the constant bank (a
+    // register here costs the 1-D..3-D kernels 16 registers and a quarter of their occupancy)
     const unsigned vcount = a.v_count;
     if (lane == 0) ws.snext = (blockIdx.x * (unsigned)kWarps + (unsigned)warp) * a.grab;  // static assignment
     for (;;) {
@@ -849,13 +880,21 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         // kPairs: a warp whose flush found the output full stops (the caller re-runs staged).
         unsigned ib = 0;
         if (lane == 0) {
-            if (MODE == kPairs && ws.wcur) {
+            if (MODE == kPairs && ws.ctl.wcur) {
                 ib = vcount;
             } else if (a.static_q) {
                 ib = ws.snext;
                 ws.snext = ib + gridDim.x * (unsigned)kWarps * a.grab;
             } else {
                 ib = (unsigned)atomicAdd(a.head, (unsigned long long)a.grab);
+            }
+            // device-sized launch (a.v_count = ~0u): the bound the prologue read (grab 1)
+            if (ib >= ws.ctl.vcount) ib = 0xFFFFFFFFu;
+            // fused estimator (a9; v_begin 0, stride 1, grab 1): on the first dequeue past the
+            // sample, this warp's hits so far all came from sample chunks
+            if (MODE == kPairs && !Cols<DIM, MODE>::value && !ws.ctl.sclosed && ib >= ws.ctl.sv1) {
+                ws.ctl.samp = ws.ctl.wtot + (unsigned long long)nbuf;
+                ws.ctl.sclosed = 1;
             }
         }
         ib = __shfl_sync(kFull, ib, 0);
@@ -866,7 +905,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
             const unsigned long long c = v * a.world + a.rank;  // queue slice (multi-GPU)
             if (c >= a.n_chunks) break;
             if constexpr (MODE == kExact) {  // exact sizing: the chunk's pairs start at voff[v]
-                if (lane == 0) ws.wcur = __ldg(a.voff + v) - a.out_base;
+                if (lane == 0) ws.ctl.wcur = __ldg(a.voff + v) - a.out_base;
                 __syncwarp();
             }
             const unsigned long long nh0 = nhits;
@@ -904,7 +943,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
             }
             if (gmask) generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
             if constexpr (MODE == kExact) {  // exact sizing: a chunk's pairs never share a flush
-                flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.wcur);
+                flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
             } else if constexpr (MODE == kChunkCount) {  // exact sizing, pass 1: pairs per chunk
                 unsigned long long d = nhits - nh0;
 #pragma unroll
@@ -915,7 +954,11 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         }
     }
     if constexpr (Mode<MODE>::pairs) {
-        flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.wcur);
+        flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
+        if (MODE == kPairs && a.sample_ctr && lane == 0) {
+            const unsigned long long sh = ws.ctl.sclosed ? ws.ctl.samp : ws.ctl.wtot;
+            if (sh) atomicAdd(a.sample_ctr, (GCG ? 1ull : 2ull) * sh);
+        }
     } else {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) nhits += __shfl_xor_sync(kFull, nhits, o);

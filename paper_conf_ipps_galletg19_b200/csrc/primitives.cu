@@ -164,7 +164,7 @@ __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *k
 
 template <class K>
 int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_t n, int bits, K **keys_out,
-               uint32_t **vals_out, cudaStream_t s) {
+               uint32_t **vals_out, cudaStream_t s, Workspace *ws) {
     *keys_out = keys;
     *vals_out = vals;
     if (n <= 1 || bits <= 0) return SJ_OK;
@@ -173,21 +173,23 @@ int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_
         return SJ_EINVAL;
     }
     const uint32_t ntiles = (uint32_t)((n + kRadixTile - 1) / kRadixTile);
-    uint32_t *hist = nullptr;
-    SJ_TRY(dev_alloc_t(&hist, (uint64_t)kRadixBins * ntiles, s));
+    const uint64_t hbytes = (uint64_t)kRadixBins * ntiles * sizeof(uint32_t);
+    uint32_t *hist = ws ? static_cast<uint32_t *>(ws->take(hbytes)) : nullptr;
+    const bool own = hist == nullptr;
+    if (own) SJ_TRY(dev_alloc(reinterpret_cast<void **>(&hist), hbytes + 16, s));
     K *ka = keys, *kb = keys_alt;
     uint32_t *va = vals, *vb = vals_alt;
     for (int shift = 0; shift < bits; shift += 8) {
         radix_hist_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, n, shift, hist, ntiles);
         note_launch();
-        SJ_TRY(scan_exclusive_u32(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s));
+        SJ_TRY(scan_exclusive_u32(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s, ws));
         radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, va, kb, vb, n, shift, hist, ntiles);
         note_launch();
         SJ_CUDA_TRY(cudaGetLastError());
         K *tk = ka; ka = kb; kb = tk;
         uint32_t *tv = va; va = vb; vb = tv;
     }
-    dev_free(hist, s);
+    if (own) dev_free(hist, s);
     *keys_out = ka;
     *vals_out = va;
     return SJ_OK;
@@ -210,12 +212,13 @@ struct DoneTotal {
 
 }  // namespace
 
-int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s) {
+int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s,
+                       Workspace *ws) {
     if (n == 0) {
         if (d_total) SJ_CUDA_TRY(cudaMemsetAsync(d_total, 0, sizeof(uint32_t), s));
         return SJ_OK;
     }
-    return scan_fused(n, LoadArr{in}, StoreArr{out}, s, DoneTotal{d_total});
+    return scan_fused(n, LoadArr{in}, StoreArr{out}, s, DoneTotal{d_total}, ws);
 }
 namespace {
 template <class In>
@@ -252,12 +255,12 @@ int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uin
 }
 
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s) {
-    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s);
+                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws) {
+    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws);
 }
 int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s) {
-    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s);
+                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws) {
+    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws);
 }
 
 }  // namespace sj

@@ -144,19 +144,25 @@ struct NoDone {
 
 // Exclusive scan of load(0..n-1) in one launch (value type T: unsigned, or unsigned long
 // long for totals below 2^62).  Temporaries from the stream-ordered pool.
+// With a workspace the tile status words come from its pre-zeroed region (no memset, no
+// allocation); without one, or when that region is exhausted, from the pool.
 template <class T = unsigned, class Load, class Store, class Done = NoDone>
-int scan_fused(uint64_t n, Load load, Store store, cudaStream_t s, Done done = Done()) {
+int scan_fused(uint64_t n, Load load, Store store, cudaStream_t s, Done done = Done(), Workspace *ws = nullptr) {
     using namespace scan_detail;
     if (n == 0) return SJ_OK;
     const uint64_t nt = (n + kTile - 1) / kTile;
-    unsigned long long *status = nullptr;
-    SJ_TRY(dev_alloc(reinterpret_cast<void **>(&status), nt * sizeof(unsigned long long) + 64, s));
+    const size_t bytes = nt * sizeof(unsigned long long) + 64;
+    unsigned long long *status = ws ? static_cast<unsigned long long *>(ws->take_zero(bytes)) : nullptr;
+    const bool own = status == nullptr;
+    if (own) {
+        SJ_TRY(dev_alloc(reinterpret_cast<void **>(&status), bytes, s));
+        SJ_CUDA_TRY(cudaMemsetAsync(status, 0, bytes, s));
+    }
     unsigned *ctr = reinterpret_cast<unsigned *>(status + nt);
-    SJ_CUDA_TRY(cudaMemsetAsync(status, 0, nt * sizeof(unsigned long long) + 64, s));
     scan_kernel<T><<<(unsigned)nt, kThreads, 0, s>>>(n, load, store, done, status, ctr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
-    dev_free(status, s);
+    if (own) dev_free(status, s);
     return SJ_OK;
 }
 

@@ -60,6 +60,34 @@ inline int dev_alloc_t(T **p, size_t count, cudaStream_t s) {
     return dev_alloc(reinterpret_cast<void **>(p), count * sizeof(T) + 16, s);
 }
 
+// Build workspace (one stream-ordered block per sj_create): a bump region for the build's
+// temporaries and a region zeroed ONCE up front for the small counters and the look-back
+// status words of every scan, so the build issues one allocation and one memset instead of
+// one of each per temporary and per scan (the host's API calls, not the GPU, paced the
+// short build kernels).  take*() return nullptr when the region is exhausted; callers then
+// fall back to dev_alloc (+ memset).
+struct Workspace {
+    char *base = nullptr;
+    size_t cap = 0, off = 0;
+    char *zbase = nullptr;
+    size_t zcap = 0, zoff = 0;
+    static size_t round(size_t b) { return (b + 255) & ~(size_t)255; }
+    void *take(size_t bytes) {
+        bytes = round(bytes);
+        if (!base || off + bytes > cap) return nullptr;
+        void *p = base + off;
+        off += bytes;
+        return p;
+    }
+    void *take_zero(size_t bytes) {
+        bytes = round(bytes);
+        if (!zbase || zoff + bytes > zcap) return nullptr;
+        void *p = zbase + zoff;
+        zoff += bytes;
+        return p;
+    }
+};
+
 // Process-wide free list of 4 KiB pinned host blocks ("mailboxes" for small D2H reads);
 // cudaMallocHost costs far more than a whole small join, so blocks are recycled.
 constexpr size_t kMailBytes = 4096;
@@ -68,7 +96,8 @@ void pinned_release(void *p);
 
 // --------------------------------------------------------------------------- primitives
 // Exclusive scan of u32 (out may alias in).  total (device, optional) receives the sum.
-int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s);
+int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s,
+                       Workspace *ws = nullptr);
 
 // Exclusive scans with 64-bit sums (pair counts, CSR row offsets; totals < 2^62).  out may
 // alias in; d_total (device, optional) receives the sum, e.g. out + n for an (n+1)-entry
@@ -82,9 +111,9 @@ int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uin
 // result pointer pair is returned through *keys_out / *vals_out (one of the inputs
 // or the alternates).
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s);
+                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws = nullptr);
 int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s);
+                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws = nullptr);
 
 // --------------------------------------------------------------------------- index
 // The index I in its B200 layout, DESIGN.md §4.  Points are stored in the
@@ -114,6 +143,8 @@ struct Index {
     uint32_t *chunks = nullptr; // [C+1]      WorkQueue chunk c = D' positions [chunks[c], chunks[c+1])
     uint64_t n_chunks = 0;      // C
     uint64_t n_query = 0;       // queries: D' positions [0, n_query) (n unless partitioned)
+    uint32_t *d_meta = nullptr; // [4]        device {n_chunks, E}, written by the build
+    uint64_t runs_cap = 0;      // entries allocated for runs (>= E + 2)
 };
 
 struct BuildTimes {
@@ -132,7 +163,11 @@ struct BuildPart {
 
 // Builds the index from device-resident raw points (n x dim AoS).  Returns sj_status.
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s,
-                cudaEvent_t ev0, cudaEvent_t ev1, float *ms, const BuildPart *part = nullptr);
+                cudaEvent_t ev0, cudaEvent_t ev1, float *ms, const BuildPart *part = nullptr,
+                uint64_t *tail_mail = nullptr);
+// tail_mail (pinned host, 2 words): the build ends without a host round trip; {n_chunks, E}
+// arrive there once the stream passes ev1, and ix.n_chunks / ix.n_runs / *ms stay unset
+// until the caller reads them (sj_runtime.cu: ix_ready).  nullptr: synchronous, all set.
 void free_index(Index &ix, cudaStream_t s);
 // LID-UNICOMP forward offsets (host): F = (3^dim - 1)/2 offsets, int8 each dim.
 int forward_offsets_public(int dim, int8_t *out, uint64_t cap);
@@ -161,6 +196,15 @@ struct JoinArgs {
     unsigned long long *emit_ctr; // pairs emitted (may exceed out_cap -> overflow)
     unsigned long long out_cap;   // capacity of out in pairs
     unsigned long long *calcs;    // instrumented distance calculations, or nullptr
+    // kPairs: the batch estimator fused into the join (a9): pairs of the virtual chunks
+    // [v_begin, sample_v1) are added to *sample_ctr (sample_v1 = 0: off)
+    unsigned long long *sample_ctr;
+    unsigned long long sample_v1;
+    // device-sized launch (the build's chunk count not yet on the host): the slice's virtual
+    // chunk count V is computed from *d_nchunks in the kernel (v_begin 0, stride 1, v_end V),
+    // and with sample_ppm the fused estimator's sample is the first ceil(V * ppm / 1e6) chunks
+    const uint32_t *d_nchunks;
+    uint32_t sample_ppm;
     // exact two-pass sizing
     unsigned long long *vcount;       // kChunkCount: pairs of virtual chunk v (written per chunk)
     const unsigned long long *voff;   // kExact: pair offset of virtual chunk v (exclusive scan of vcount);

@@ -137,6 +137,8 @@ struct sj_handle {
     int state = 0;  // 0 ready, 1 continuing (staged path), -1 error
     cudaStream_t s_main = nullptr;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr, ev_c = nullptr, ev_d = nullptr, ev_e = nullptr;
+    cudaEvent_t ev_ba = nullptr, ev_bb = nullptr;  // build start / end
+    int pending = 0;  // 1: the build's tail {n_chunks, E} and its timing not read yet (ix_ready)
     sj::Index ix;
     bool owns_index = true;
     int num_sms = 148;
@@ -195,7 +197,7 @@ struct Core {
     int device;
     int num_sms;
     cudaStream_t s;
-    cudaEvent_t ev[5];
+    cudaEvent_t ev[7];
     unsigned long long *d_ctr;
     uint64_t *mail;
 };
@@ -217,6 +219,8 @@ int handle_init_common(sj_handle *h) {
                 h->ev_c = c.ev[2];
                 h->ev_d = c.ev[3];
                 h->ev_e = c.ev[4];
+                h->ev_ba = c.ev[5];
+                h->ev_bb = c.ev[6];
                 h->d_ctr = c.d_ctr;
                 h->mail = c.mail;
                 return SJ_OK;
@@ -230,6 +234,8 @@ int handle_init_common(sj_handle *h) {
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_c));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_d));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_e));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_ba));
+    SJ_CUDA_TRY(cudaEventCreate(&h->ev_bb));
     h->mail = static_cast<uint64_t *>(pinned_acquire());
     if (!h->mail) return SJ_ENOMEM;
     SJ_TRY(dev_alloc_t(&h->d_ctr, 8, h->s_main));
@@ -238,14 +244,16 @@ int handle_init_common(sj_handle *h) {
 
 // Returns the handle's core to the cache (stream drained first); false if it must be freed.
 bool core_release(sj_handle *h) {
-    if (!h->s_main || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->ev_e || !h->d_ctr || !h->mail) return false;
+    if (!h->s_main || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->ev_e || !h->ev_ba || !h->ev_bb || !h->d_ctr ||
+        !h->mail)
+        return false;
     if (cudaStreamSynchronize(h->s_main) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
     std::lock_guard<std::mutex> lk(g_core_mu);
     if (g_core_cache.size() >= 64) return false;
-    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e}, h->d_ctr,
+    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e, h->ev_ba, h->ev_bb}, h->d_ctr,
                                 h->mail});
     return true;
 }
@@ -351,6 +359,40 @@ JoinArgs base_args(const sj_handle *h) {
     a.rank = (uint32_t)h->rank;
     a.world = (uint32_t)h->world;
     return a;
+}
+
+void fill_static_stats(sj_handle *h) {
+    sj_stats &st = h->st;
+    st.n = h->ix.n;
+    st.dim = (uint32_t)h->ix.dim;
+    st.key_bits = (uint32_t)h->ix.key_bits;
+    st.n_cells = h->ix.n_cells;
+    st.fwd_runs = h->ix.n_runs;
+    st.dist_calcs = h->ix.dist_calcs;
+    st.max_cell_load = h->ix.max_w;
+    st.k = (uint32_t)h->k;
+    for (int d = 0; d < SJ_MAX_DIM; ++d) st.nc[d] = d < h->ix.dim ? (uint32_t)h->ix.nc[d] : 0;
+    st.n_chunks = h->ix.n_chunks;
+    st.tiled_min = kBigCell;
+    st.pattern = (uint32_t)h->ix.pattern;
+    st.order = (uint32_t)h->ix.order;
+}
+
+// The build's tail (sj_create returns without a final round trip): {n_chunks, E} from the
+// handle's mailbox once the stream passed the build's end event, the build time, the static
+// statistics.  Every host path that needs them calls this first; the in-place fast path does
+// so only after its join (the kernel reads n_chunks on the device).
+int ix_ready(sj_handle *h) {
+    if (!h->pending) return SJ_OK;
+    SJ_CUDA_TRY(cudaEventSynchronize(h->ev_bb));
+    h->ix.n_chunks = h->mail[48];
+    h->ix.n_runs = h->mail[49];
+    float ms = 0;
+    SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_ba, h->ev_bb));
+    h->pending = 0;
+    fill_static_stats(h);
+    h->st.ms_build = ms;
+    return SJ_OK;
 }
 
 int join_blocks(const sj_handle *h, int mode, int *blocks) {
@@ -573,28 +615,38 @@ int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_
     return SJ_OK;
 }
 
-// Fast path (caller's HBM buffer, in place): the estimator (a9) -- a count-only join of
-// the sample chunks -- then the join of the whole queue [0, V) into the caller's buffer, back
-// to back on the main stream: in place there are no batches to size, so the join does not wait
-// for the estimate on the host (it is reported, and sizes the staged fallback if the buffer
-// overflows).  (Running the estimator concurrently on a side stream was measured: it wins
-// ~0.04 ms on C5 but loses 3 ms on C5 eps=0.2, where estimator and join fight over the same
-// heaviest head of D'.)  *spairs = the sample's pairs, *total = all pairs emitted (> cap:
-// overflow, only the first cap were written).
+// Fast path (caller's HBM buffer, in place): the estimator (a9) and the join of the
+// whole queue [0, V) into the caller's buffer.  In place there are no batches to size, so the
+// join never waits for the estimate; it is reported, and sizes the staged fallback if the
+// buffer overflows.  WorkQueue: the estimator is FUSED into the join -- the sample is the first
+// sch chunks of D', which are exactly the first chunks the queue hands out, so the join
+// adds the pairs of chunks [0, sv1) to a counter of their own: the same number a separate
+// count-only launch over [0, sv1) returns, without evaluating the heaviest 1 % twice (a
+// separate launch of it cannot fill the GPU: 84 us on C5).  Every dequeued chunk is finished,
+// so the sample is complete whenever the queue head passed sv1 -- always, unless the output
+// overflowed early; then the separate estimator runs.  SortByWL only (strided sample, static
+// assignment): the separate count-only launch first, back to back on the main stream.
+// (Running it concurrently on a side stream was measured: it wins ~0.04 ms on C5 but loses
+// 3 ms on C5 eps=0.2, where estimator and join fight over the same heaviest head of D'.)
+// *spairs = the sample's pairs, *total = all pairs emitted (> cap: overflow, only the first
+// cap were written).
 int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, uint64_t sv1, uint64_t sstride,
                      uint64_t V, uint64_t *spairs, uint64_t *total) {
     cudaStream_t s = h->s_main;
+    const bool fused = sstride == 1 && h->queue && h->grab == 1 && sch && !getenv("SJ_SEPARATE_EST");
     SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
-    JoinArgs e = base_args(h);
-    e.head = h->d_ctr + 5;
-    e.emit_ctr = h->d_ctr + 4;
-    e.v_begin = 0;
-    e.v_end = sv1;  // the sample: chunks 0, sstride, ... < sv1 (sch of them)
-    e.v_stride = (uint32_t)sstride;
-    int blocks_e;
-    SJ_TRY(join_blocks(h, kCount, &blocks_e));
-    if (sch) SJ_TRY(launch_join(e, h->ix.dim, h->k, kCount, blocks_e, s));
+    if (!fused) {
+        JoinArgs e = base_args(h);
+        e.head = h->d_ctr + 5;
+        e.emit_ctr = h->d_ctr + 4;
+        e.v_begin = 0;
+        e.v_end = sv1;  // the sample: chunks 0, sstride, ... < sv1 (sch of them)
+        e.v_stride = (uint32_t)sstride;
+        int blocks_e;
+        SJ_TRY(join_blocks(h, kCount, &blocks_e));
+        if (sch) SJ_TRY(launch_join(e, h->ix.dim, h->k, kCount, blocks_e, s));
+    }
     SJ_CUDA_TRY(cudaEventRecord(h->ev_e, s));
     JoinArgs a = base_args(h);
     a.out = out;
@@ -604,6 +656,10 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
     a.head = h->d_ctr + 1;
     a.v_begin = 0;
     a.v_end = V;
+    if (fused) {
+        a.sample_ctr = h->d_ctr + 4;
+        a.sample_v1 = sv1;
+    }
     int blocks;
     SJ_TRY(join_blocks(h, kPairs, &blocks));
     if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, kPairs, blocks, s));
@@ -615,8 +671,59 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
     SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_e, h->ev_d));
     h->st.join_launches = V ? 1u : 0u;
     h->st.batches = 1;
-    h->st.ms_estimate = ms_est;              // the estimator launch
-    h->st.ms_join = h->st.ms_join_sum = ms;  // the join launch
+    h->st.ms_estimate = fused ? 0.0 : ms_est;  // fused: inside the join launch
+    h->st.ms_join = h->st.ms_join_sum = ms;   // the join launch
+    h->st.est_fused = fused ? 1u : 0u;
+    *spairs = h->mail[4];
+    *total = h->mail[0];
+    if (fused && h->mail[1] < sv1) {  // overflowed before the sample was handed out: count it apart
+        const uint64_t emitted = *total;
+        const uint64_t calcs = h->mail[2];
+        float ms_c = 0;
+        SJ_TRY(count_range(h, 0, sv1, spairs, &ms_c));
+        h->st.ms_estimate = ms_c;
+        h->st.est_fused = 0;
+        h->mail[0] = emitted;
+        h->mail[2] = calcs;
+    }
+    return SJ_OK;
+}
+
+// The fast path right after sj_create, before the build's tail reached the host: ONE
+// device-sized launch (the kernel reads the chunk count the build left in ix.d_meta and sizes
+// the fused estimator's sample from it), so the GPU goes from the last build kernel straight
+// into the join.  *spairs = the sample's pairs, *total = all pairs emitted.
+int run_in_place_lazy(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *spairs, uint64_t *total) {
+    cudaStream_t s = h->s_main;
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_e, s));
+    JoinArgs a = base_args(h);
+    a.n_chunks = 0xFFFFFFFFu;      // bounded by the device-side V instead
+    a.n_runs = h->ix.runs_cap;     // the allocation (>= E): bounds of the staged run copies
+    a.d_nchunks = h->ix.d_meta;
+    a.sample_ppm = h->sample_ppm;
+    a.sample_ctr = h->d_ctr + 4;
+    a.out = out;
+    a.emit_ctr = h->d_ctr;
+    a.out_cap = cap;
+    a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
+    a.head = h->d_ctr + 1;
+    a.v_begin = 0;
+    a.v_end = 0xFFFFFFFFull;  // v_count = ~0u: the kernel bounds the queue by the device-side V
+    int blocks;
+    SJ_TRY(join_blocks(h, kPairs, &blocks));
+    SJ_TRY(launch_join(a, h->ix.dim, h->k, kPairs, blocks, s));
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 5 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    SJ_TRY(ix_ready(h));
+    float ms = 0;
+    SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_e, h->ev_d));
+    h->st.join_launches = 1;
+    h->st.batches = 1;
+    h->st.ms_estimate = 0.0;
+    h->st.ms_join = h->st.ms_join_sum = ms;
+    h->st.est_fused = 1;
     *spairs = h->mail[4];
     *total = h->mail[0];
     return SJ_OK;
@@ -710,13 +817,27 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     h->st.join_launches = 0;
     h->st.ms_join = h->st.ms_join_sum = h->st.ms_estimate = h->st.ms_transfer = h->st.ms_total = 0;
     h->st.fast_path = 0;
+    h->st.est_fused = 0;
     h->st.k = (uint32_t)h->k;
     h->jobs.clear();
     for (int i = 0; i < kMaxStreams; ++i) h->slots[i].busy = false;
 
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_a, h->s_main));
+    const bool dev_out = out && is_device_ptr(out, h->device);
+    // right after sj_create, the in-place WorkQueue join needs nothing from the build on the
+    // host (run_in_place_lazy); every other path reads the build's tail first
+    const bool lazy = h->pending && dev_out && h->fast_path && !h->exact && h->queue && h->grab == 1 &&
+                      !getenv("SJ_DEBUG_VRANGE") && !getenv("SJ_SEPARATE_EST") &&
+                      !(reinterpret_cast<uintptr_t>(out) & 15u);
+    uint64_t lazy_spairs = 0, lazy_total = 0;
+    if (lazy) {
+        SJ_TRY(run_in_place_lazy(h, out, cap, &lazy_spairs, &lazy_total));
+        debug_mark("join: lazy fast path");
+    } else {
+        SJ_TRY(ix_ready(h));
+    }
     const uint64_t nch = slice_chunks(h);
     const uint64_t V = nch;
-    SJ_CUDA_TRY(cudaEventRecord(h->ev_a, h->s_main));
 
     if (out == nullptr) {  // count-only (whole slice, one launch)
         uint64_t pairs = 0;
@@ -736,7 +857,6 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         return SJ_OK;
     }
 
-    const bool dev_out = is_device_ptr(out, h->device);
     if (dev_out && (reinterpret_cast<uintptr_t>(out) & 15u)) {
         set_error("sj_self_join: device out_pairs must be 16-byte aligned");
         return SJ_EINVAL;
@@ -764,7 +884,21 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         // (the join stops early) and falls back to the staged path below, whose batches are
         // sized by the estimate.
         uint64_t total = 0;
-        SJ_TRY(run_in_place_est(h, out, cap, sch, sv1, sstride, V, &spairs, &total));
+        if (lazy) {  // already ran; the sample is complete unless the output overflowed early
+            spairs = lazy_spairs;
+            total = lazy_total;
+            if (h->mail[1] < sv1) {
+                const uint64_t calcs = h->mail[2];
+                float ms_c = 0;
+                SJ_TRY(count_range(h, 0, sv1, &spairs, &ms_c));
+                h->st.ms_estimate = ms_c;
+                h->st.est_fused = 0;
+                h->mail[0] = total;
+                h->mail[2] = calcs;
+            }
+        } else {
+            SJ_TRY(run_in_place_est(h, out, cap, sch, sv1, sstride, V, &spairs, &total));
+        }
         debug_mark("join: fast path");
         h->st.est_pairs = nch ? (uint64_t)((double)spairs * (double)nch / (double)sch) : 0;
         if (total <= cap) return finish_in_place(h, total, count);
@@ -815,6 +949,7 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
 // Device CSR (sj_neighbor_csr): degrees (GCG row owners, no atomics) -> exclusive scan ->
 // row fill.  Temporaries come from the stream-ordered pool.
 int neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, uint64_t *total) {
+    SJ_TRY(ix_ready(h));
     if (h->ix.pattern != SJ_PATTERN_GCG) {
         set_error("sj_neighbor_csr: needs a handle created with SJ_PATTERN_GCG (every query owns its row)");
         return SJ_EINVAL;
@@ -974,22 +1109,6 @@ static int create_common(sj_handle **out_h) {
     return SJ_OK;
 }
 
-static void fill_static_stats(sj_handle *h) {
-    sj_stats &st = h->st;
-    st.n = h->ix.n;
-    st.dim = (uint32_t)h->ix.dim;
-    st.key_bits = (uint32_t)h->ix.key_bits;
-    st.n_cells = h->ix.n_cells;
-    st.fwd_runs = h->ix.n_runs;
-    st.dist_calcs = h->ix.dist_calcs;
-    st.max_cell_load = h->ix.max_w;
-    st.k = (uint32_t)h->k;
-    for (int d = 0; d < SJ_MAX_DIM; ++d) st.nc[d] = d < h->ix.dim ? (uint32_t)h->ix.nc[d] : 0;
-    st.n_chunks = h->ix.n_chunks;
-    st.tiled_min = kBigCell;
-    st.pattern = (uint32_t)h->ix.pattern;
-    st.order = (uint32_t)h->ix.order;
-}
 
 sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps) {
     return sj_create_ex(points, n, dim, eps, SJ_PATTERN_LID_UNICOMP, SJ_ORDER_WORKLOAD);
@@ -1070,11 +1189,19 @@ static sj_handle *create_impl(const double *points, uint64_t n, int dim, double 
         }
     }
     debug_mark("create: upload issued");
-    if (rc == SJ_OK) rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_a, h->ev_b, &ms, origin ? &part : nullptr);
+    // The build returns without a final host round trip (its tail is read by ix_ready) unless
+    // SJ_SYNC_BUILD=1; errors of its last kernels surface at the next synchronisation.
+    static const bool sync_build = [] {
+        const char *e = getenv("SJ_SYNC_BUILD");
+        return e && e[0] == '1';
+    }();
+    if (rc == SJ_OK)
+        rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_ba, h->ev_bb, &ms, origin ? &part : nullptr,
+                         sync_build ? nullptr : h->mail + 48);
     debug_mark("create: build_index");
     dev_free(d_copy, s);
     dev_free(d_ids, s);
-    if (rc == SJ_OK && cudaStreamSynchronize(s) != cudaSuccess) {
+    if (rc == SJ_OK && sync_build && cudaStreamSynchronize(s) != cudaSuccess) {
         set_error("sj_create: %s", cudaGetErrorString(cudaGetLastError()));
         rc = SJ_ECUDA;
     }
@@ -1084,8 +1211,12 @@ static sj_handle *create_impl(const double *points, uint64_t n, int dim, double 
         snprintf(g_err, sizeof g_err, "%s", keep.c_str());
         return nullptr;
     }
-    fill_static_stats(h);
-    h->st.ms_build = ms;
+    if (sync_build) {
+        fill_static_stats(h);
+        h->st.ms_build = ms;
+    } else {
+        h->pending = 1;
+    }
     return h;
 }
 
@@ -1146,6 +1277,8 @@ void sj_destroy(sj_handle *h) {
         if (h->ev_c) cudaEventDestroy(h->ev_c);
         if (h->ev_d) cudaEventDestroy(h->ev_d);
         if (h->ev_e) cudaEventDestroy(h->ev_e);
+        if (h->ev_ba) cudaEventDestroy(h->ev_ba);
+        if (h->ev_bb) cudaEventDestroy(h->ev_bb);
         pinned_release(h->mail);
     }
     delete h;
@@ -1212,6 +1345,7 @@ int sj_set_slice(sj_handle *h, int rank, int world) {
 
 int sj_get_stats(const sj_handle *h, sj_stats *s) {
     if (!h || !s) return SJ_EINVAL;
+    SJ_TRY(ix_ready(const_cast<sj_handle *>(h)));
     *s = h->st;
     return SJ_OK;
 }
@@ -1274,6 +1408,7 @@ BlobHeader make_header(const Index &ix) {
 
 int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes) {
     if (!h || !bytes) return SJ_EINVAL;
+    SJ_TRY(ix_ready(const_cast<sj_handle *>(h)));
     BlobHeader b = make_header(h->ix);
     *bytes = b.total;
     if (!dst) return SJ_OK;
