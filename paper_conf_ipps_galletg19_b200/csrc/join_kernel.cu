@@ -75,6 +75,17 @@ struct BufCap {
 };
 
 // Per-warp shared memory: emission buffer, the chunk's queries, one candidate tile.
+#ifndef SJ_GSTAGE
+#define SJ_GSTAGE 1  // generic path: stage the chunk's query data and first runs in shared memory
+#endif
+// Generic path staging: the LID-UNICOMP forward runs of one cell (3-D: 5, the rows of
+// pattern_rows()); other patterns' further runs are read from global memory.  Measured (join
+// ms, B200): 3-D C3 K64 0.721 -> 0.697, K256 1.814 -> 1.679; 2-D C5 1.027 -> 1.035, C5 eps 0.2
+// 2.97 -> 3.10 (the staging's wait costs more than the run loads it hides), so 3-D only.
+template <int DIM>
+struct GStage {
+    static constexpr int runs = !SJ_GSTAGE ? 0 : DIM == 3 ? 5 : 0;
+};
 // Per-warp control words (shared memory, lane 0 writes).
 struct WarpCtl {
     // kExact: next output slot of the current chunk; kPairs: nonzero once a flush of this warp
@@ -98,6 +109,7 @@ struct WarpSmem {
     unsigned qorig[32];                 // input ids of the chunk's queries
     unsigned qrr[32];                   // the queries' positions in their (common) cell
     unsigned char glist[32];            // generic path: lanes of the chunk's remaining queries
+    uint2 gruns[32 * (GStage<DIM>::runs > 0 ? GStage<DIM>::runs : 1)];  // generic path: staged first runs
     // 4-D..6-D: the segment cell's forward runs (<= 122) staged once, so the per-tile run walk
     // reads shared memory instead of chasing L2 latency run by run
     uint2 runs_s[(DIM >= 4 && DIM <= 6) ? 128 : 1];
@@ -422,6 +434,24 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         if ((gmask >> lane) & 1u) glist[__popc(gmask & lt)] = (unsigned char)lane;
         __syncwarp();
     }
+    // Every generic query's point, input id and first forward runs are copied into shared
+    // memory at once (cp.async, all lanes in parallel): a round then starts from shared memory
+    // and its only global loads are the candidates -- one dependent global access per round
+    // instead of two (the sparse tail of D' is latency-bound, not issue-bound).
+    constexpr int GRS = GStage<DIM>::runs;
+    if constexpr (GRS > 0) {
+        __syncwarp();
+        if ((gmask >> lane) & 1u) {
+            cp_async_point<DIM>(ws.qry + lane * PAD, a.pts + (size_t)qm_lane.x * PAD);
+            cp_async_4(ws.qorig + lane, a.orig + qm_lane.x);
+#pragma unroll
+            for (int j = 0; j < GRS; ++j)
+                if (ci_lane.z + (unsigned)j < a.n_runs) cp_async_8(ws.gruns + lane * GRS + j, a.runs + ci_lane.z + j);
+        }
+        cp_async_commit();
+        cp_async_wait<0>();
+        __syncwarp();
+    }
     for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
         const unsigned qi = r0 + grp;
         const bool valid = qi < nq;
@@ -438,10 +468,19 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         uint2 nxt = make_uint2(0, 0);
         if (!valid) ci = make_uint4(0, 0, 0, 0);
         unsigned long long cur = 0;  // kRows: the query's row cursor
+        // staged runs of this query: grs[e] for e < elim (GRS > 0)
+        const uint2 *grs = ws.gruns + src * (GRS > 0 ? GRS : 1) - ci.z;
+        const unsigned elim = ci.z + (unsigned)GRS;
         if (valid) {
-            load_point<DIM>(a.pts + (size_t)qlid * PAD, qp);
-            oq = __ldg(a.orig + qlid);
-            if (ci.w) nxt = __ldg(a.runs + ci.z);  // prefetched next run
+            if constexpr (GRS > 0) {
+                load_smem_point<DIM>(ws.qry + src * PAD, qp);
+                oq = ws.qorig[src];
+                if (ci.w) nxt = grs[ci.z];
+            } else {
+                load_point<DIM>(a.pts + (size_t)qlid * PAD, qp);
+                oq = __ldg(a.orig + qlid);
+                if (ci.w) nxt = __ldg(a.runs + ci.z);  // prefetched next run
+            }
             if constexpr (MODE == kRows) cur = __ldg(a.row_off + oq);
         } else {
 #pragma unroll
@@ -473,7 +512,10 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
                         seg_base = nxt.x;
                         seg_len = nxt.y;
                         rem -= nxt.y;
-                        if (rem) nxt = __ldg(a.runs + (++e));
+                        if (rem) {
+                            ++e;
+                            nxt = (GRS > 0 && e < elim) ? grs[e] : __ldg(a.runs + e);
+                        }
                     } else {
                         seg_base = hb;
                         seg_len = home_len;
@@ -677,6 +719,9 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
     }
 }
 
+#ifndef SJ_TINY_W
+#define SJ_TINY_W 0  // chunks whose longest candidate list is <= this go through k = 1 (0: off)
+#endif
 #ifndef SJ_HOMEWIN
 #define SJ_HOMEWIN 1
 #endif
@@ -941,7 +986,20 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
                 const unsigned n0 = __shfl_sync(kFull, nseg, s0);
                 tiled_chunk<DIM, K, MODE, GCG>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
             }
-            if (gmask) generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
+            if (gmask) {
+                bool tiny = false;
+                if constexpr (SJ_TINY_W > 0 && K > 1 && DIM <= 3 && !GCG) {
+                    // short candidate lists (the sparse tail of D', sorted by W): one lane per query
+                    // and the whole chunk in one round, instead of 32/k queries per round
+                    const unsigned tot = ((gmask >> lane) & 1u) ? ci.w + home_count(ci.y, qm.x - ci.x) : 0u;
+                    tiny = __reduce_max_sync(kFull, tot) <= (unsigned)SJ_TINY_W;
+                }
+                if (tiny)
+                    generic_chunk<DIM, (SJ_TINY_W > 0 && DIM <= 3 && !GCG) ? 1 : K, MODE, GCG>(
+                        a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
+                else
+                    generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
+            }
             if constexpr (MODE == kExact) {  // exact sizing: a chunk's pairs never share a flush
                 flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
             } else if constexpr (MODE == kChunkCount) {  // exact sizing, pass 1: pairs per chunk
