@@ -86,6 +86,21 @@ template <int DIM>
 struct GStage {
     static constexpr int runs = !SJ_GSTAGE ? 0 : DIM == 3 ? 5 : 0;
 };
+#ifndef SJ_FLAT_W
+#define SJ_FLAT_W 64  // flat path for chunks whose longest candidate list is <= this (0: off)
+#endif
+// Flat path (flat_chunk): 1-D..3-D, half patterns, the pair / count modes.  runs = the
+// LID-UNICOMP forward runs per cell (pattern_rows()), staged per query.
+template <int DIM, int MODE, bool GCG>
+struct Flat {
+    static constexpr int runs = DIM == 1 ? 1 : DIM == 2 ? 2 : DIM == 3 ? 5 : 0;
+    static constexpr bool on = SJ_FLAT_W > 0 && runs > 0 && !GCG && MODE != kRows && MODE != kDegree;
+};
+template <int DIM>
+struct StagedRuns {  // entries of WarpSmem::gruns per query
+    static constexpr int a = GStage<DIM>::runs, b = Flat<DIM, kPairs, false>::runs;
+    static constexpr int value = (a > b ? a : b) > 0 ? (a > b ? a : b) : 1;
+};
 // Per-warp control words (shared memory, lane 0 writes).
 struct WarpCtl {
     // kExact: next output slot of the current chunk; kPairs: nonzero once a flush of this warp
@@ -102,14 +117,30 @@ struct WarpCtl {
 
 template <int DIM, int MODE>
 struct WarpSmem {
+    // (2-D / 3-D: the staging fits inside the tiles; 4-D+ stage one run per query, and their
+    // shared memory is what limits the occupancy: 6-D must stay under 7 KB per warp)
+    static_assert(DIM < 2 || DIM > 3 ||
+                      2 * 32 * PointPad<DIM>::value * 8 + 2 * 32 * 4 >=
+                          32 * 8 * StagedRuns<DIM>::value + 32 * 4 + 32 * 16,
+                  "the staging union must not grow the warp's shared memory");
     static constexpr int PAD = PointPad<DIM>::value;
-    alignas(16) double tile[2][32 * PAD];  // staged candidates (lid order), double-buffered
+    // the tiled path's candidate tiles and the generic / flat paths' per-query staging are
+    // never live together (a chunk's tiled segments finish before its generic queries start)
+    union {
+        struct {
+            alignas(16) double tile[2][32 * PAD];  // staged candidates (lid order), double-buffered
+            unsigned tile_orig[2][32];             // input ids of the staged candidates
+        };
+        struct {
+            uint2 gruns[32 * StagedRuns<DIM>::value];  // generic (3-D) / flat: the queries' first runs
+            unsigned wpre[32];                         // flat: exclusive prefix of the list lengths
+            uint4 fq[32];                              // flat: per query {home begin, m, rr, S}
+        };
+    };
     alignas(16) double qry[32 * PAD];   // the chunk's query points
-    unsigned tile_orig[2][32];             // input ids of the staged candidates
     unsigned qorig[32];                 // input ids of the chunk's queries
     unsigned qrr[32];                   // the queries' positions in their (common) cell
     unsigned char glist[32];            // generic path: lanes of the chunk's remaining queries
-    uint2 gruns[32 * (GStage<DIM>::runs > 0 ? GStage<DIM>::runs : 1)];  // generic path: staged first runs
     // 4-D..6-D: the segment cell's forward runs (<= 122) staged once, so the per-tile run walk
     // reads shared memory instead of chasing L2 latency run by run
     uint2 runs_s[(DIM >= 4 && DIM <= 6) ? 128 : 1];
@@ -121,6 +152,7 @@ struct WarpSmem {
     // kRows: the segment's per-query row cursors; kDegree: their running neighbour counts
     unsigned long long qcur[(MODE == kRows || MODE == kDegree) ? 32 : 1];
 };
+static_assert(sizeof(WarpSmem<6, kPairs>) <= 7168, "6-D: four 256-thread CTAs per SM");
 
 template <int DIM>
 __device__ __forceinline__ void load_point(const double *__restrict__ p, double (&x)[DIM]) {
@@ -446,7 +478,8 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
             cp_async_4(ws.qorig + lane, a.orig + qm_lane.x);
 #pragma unroll
             for (int j = 0; j < GRS; ++j)
-                if (ci_lane.z + (unsigned)j < a.n_runs) cp_async_8(ws.gruns + lane * GRS + j, a.runs + ci_lane.z + j);
+                if (ci_lane.z + (unsigned)j < a.n_runs)
+                    cp_async_8(ws.gruns + lane * StagedRuns<DIM>::value + j, a.runs + ci_lane.z + j);
         }
         cp_async_commit();
         cp_async_wait<0>();
@@ -469,7 +502,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
         if (!valid) ci = make_uint4(0, 0, 0, 0);
         unsigned long long cur = 0;  // kRows: the query's row cursor
         // staged runs of this query: grs[e] for e < elim (GRS > 0)
-        const uint2 *grs = ws.gruns + src * (GRS > 0 ? GRS : 1) - ci.z;
+        const uint2 *grs = ws.gruns + src * StagedRuns<DIM>::value - ci.z;
         const unsigned elim = ci.z + (unsigned)GRS;
         if (valid) {
             if constexpr (GRS > 0) {
@@ -544,6 +577,107 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
             if (valid && t == 0) a.qdeg[oq] = deg;
         }
     }
+}
+
+// Flat path for short candidate lists (the sparse tail of D', whose chunks hold queries of
+// small cells with similar W): the (query, candidate) pairs of all the chunk's generic queries
+// are numbered f = 0 .. T-1 (query by query, each query's list as in generic_chunk: forward runs,
+// then the home half scan) and lane l evaluates pairs l, l+32, ... -- two per step, independent,
+// so their candidate loads are in flight together.  The k-lane rounds of generic_chunk instead
+// walk 32/k queries per round with a dependent global load chain each round, which is what the
+// sparse tail's time is made of (it is latency-bound, not issue-bound).  The queries' points,
+// ids and forward runs are staged in shared memory first; the query of pair f is found by a
+// binary search over the prefix sums of the list lengths.  Returns false (nothing evaluated)
+// when a list is longer than SJ_FLAT_W or a cell has more runs than are staged (UNICOMP).
+template <int DIM, int MODE, bool GCG>
+__device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
+                                           WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
+                                           unsigned long long &ncalcs, int lane, unsigned lt) {
+    constexpr int PAD = PointPad<DIM>::value;
+    constexpr int FRS = Flat<DIM, MODE, GCG>::runs;
+    constexpr int SR = StagedRuns<DIM>::value;
+    const bool mine = (gmask >> lane) & 1u;
+    const unsigned rr_l = qm_lane.x - ci_lane.x;
+    const unsigned W = mine ? ci_lane.w + home_count(ci_lane.y, rr_l) : 0u;
+    if (__reduce_max_sync(kFull, W) > (unsigned)SJ_FLAT_W) return false;
+    __syncwarp();
+    if (mine) {
+        cp_async_point<DIM>(ws.qry + lane * PAD, a.pts + (size_t)qm_lane.x * PAD);
+        cp_async_4(ws.qorig + lane, a.orig + qm_lane.x);
+#pragma unroll
+        for (int j = 0; j < FRS; ++j)
+            if (ci_lane.z + (unsigned)j < a.n_runs) cp_async_8(ws.gruns + lane * SR + j, a.runs + ci_lane.z + j);
+    }
+    unsigned incl = W;  // inclusive warp scan of the list lengths
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned v = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += v;
+    }
+    const unsigned T = __shfl_sync(kFull, incl, 31);
+    ws.wpre[lane] = incl - W;
+    ws.fq[lane] = make_uint4(ci_lane.x, ci_lane.y, rr_l, ci_lane.w);
+    cp_async_commit();
+    cp_async_wait<0>();
+    __syncwarp();
+    // the staged runs must cover the forward list (LID-UNICOMP: always; UNICOMP may have more)
+    bool covered = true;
+    if (mine) {
+        unsigned acc = 0;
+#pragma unroll
+        for (int j = 0; j < FRS; ++j)
+            if (acc < ci_lane.w) acc += ws.gruns[lane * SR + j].y;
+        covered = acc == ci_lane.w;
+    }
+    if (!__all_sync(kFull, covered)) return false;
+    ncalcs += W;
+    unsigned long long cur = 0;
+    for (unsigned f0 = 0; f0 < T; f0 += 64) {
+        double qq[2][DIM], cp[2][DIM];
+        unsigned oq[2], oc[2];
+        bool ok[2];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            const unsigned f = f0 + (unsigned)(u * 32 + lane);
+            ok[u] = f < T;
+            unsigned q = 0;  // the last query whose prefix is <= f (zero-length lists are skipped)
+#pragma unroll
+            for (unsigned st = 16; st > 0; st >>= 1)
+                if (ws.wpre[q + st] <= f) q += st;
+            unsigned j = f - ws.wpre[q];
+            const uint4 d = ws.fq[q];  // {home begin, m, rr, S}
+            unsigned idx;
+            if (j < d.w) {  // forward runs, in order
+                idx = 0;
+                bool found = false;
+#pragma unroll
+                for (int r = 0; r < FRS; ++r) {
+                    const uint2 run = ws.gruns[q * SR + r];
+                    if (!found && j < run.y) {
+                        idx = run.x + j;
+                        found = true;
+                    }
+                    if (!found) j -= run.y;
+                }
+            } else {  // home cell: circulant half scan, offset j - S past rr (reading c8)
+                unsigned p = d.z + 1u + (j - d.w);
+                if (p >= d.y) p -= d.y;
+                idx = d.x + p;
+            }
+            if (!ok[u]) idx = d.x;  // a valid address; masked below
+            load_point<DIM>(a.pts + (size_t)idx * PAD, cp[u]);
+            oc[u] = Mode<MODE>::pairs ? __ldg(a.orig + idx) : 0u;
+            load_smem_point<DIM>(ws.qry + q * PAD, qq[u]);
+            oq[u] = ws.qorig[q];
+        }
+        bool hit[2];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) hit[u] = ok[u] && sqdist<DIM>(qq[u], cp[u]) <= a.e2;
+        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.ctl);
+#pragma unroll
+        for (int u = 0; u < 2; ++u) emit<DIM, MODE, GCG>(hit[u], oq[u], oc[u], ws.buf, nbuf, nhits, lt, kFull, cur, a, lane);
+    }
+    return true;
 }
 
 // Evaluate one staged tile against every query of the chunk.  HOME: the tile holds home-cell
@@ -719,9 +853,6 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
     }
 }
 
-#ifndef SJ_TINY_W
-#define SJ_TINY_W 0  // chunks whose longest candidate list is <= this go through k = 1 (0: off)
-#endif
 #ifndef SJ_HOMEWIN
 #define SJ_HOMEWIN 1
 #endif
@@ -987,18 +1118,10 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
                 tiled_chunk<DIM, K, MODE, GCG>(a, (unsigned)s0, n0, qm, cs, ws, nbuf, nhits, ncalcs, lane, lt);
             }
             if (gmask) {
-                bool tiny = false;
-                if constexpr (SJ_TINY_W > 0 && K > 1 && DIM <= 3 && !GCG) {
-                    // short candidate lists (the sparse tail of D', sorted by W): one lane per query
-                    // and the whole chunk in one round, instead of 32/k queries per round
-                    const unsigned tot = ((gmask >> lane) & 1u) ? ci.w + home_count(ci.y, qm.x - ci.x) : 0u;
-                    tiny = __reduce_max_sync(kFull, tot) <= (unsigned)SJ_TINY_W;
-                }
-                if (tiny)
-                    generic_chunk<DIM, (SJ_TINY_W > 0 && DIM <= 3 && !GCG) ? 1 : K, MODE, GCG>(
-                        a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
-                else
-                    generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
+                bool done = false;
+                if constexpr (Flat<DIM, MODE, GCG>::on)
+                    done = flat_chunk<DIM, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
+                if (!done) generic_chunk<DIM, K, MODE, GCG>(a, gmask, qm, ci, ws, nbuf, nhits, ncalcs, lane, lt);
             }
             if constexpr (MODE == kExact) {  // exact sizing: a chunk's pairs never share a flush
                 flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
