@@ -10,6 +10,7 @@
 //      contiguous runs of the lid-ordered point storage
 //   a7 workload W(A) = ceil((m_A-1)/2) + sum_{B in fwd(A)} m_B and D_alg
 //   a8 SortByWL: cells in non-increasing W (stable, ties by lid, c10) -> D' (index array)
+#include <algorithm>
 #include <cmath>
 #include <cstring>
 #include <vector>
@@ -19,7 +20,6 @@
 
 namespace sj {
 
-__constant__ uint64_t c_fwd_off[SJ_MAX_FWD];  // rows of the cell pattern (pattern_rows()), packed
 
 namespace {
 
@@ -221,6 +221,9 @@ struct FwdGeom {
     int rows;   // rows of the cell pattern (see pattern_rows())
     int small;  // prod(nc) < 2^32: 32-bit lid arithmetic
     int full;   // GCG: the rows cover the whole 3^n neighbourhood incl. the home cell
+    // rows of the cell pattern, resolved against this grid (RowEnt), in this build's workspace:
+    // read through L1 (lanes of a 32-lane cell read different rows)
+    const struct RowEnt *rows_ent;
     // partitioned index (sj_create_part): a cell is a query cell iff its first member (lowest
     // input id, the sort is stable) is < nq; halo cells get no runs and no workload
     const uint32_t *idx;  // sorted position -> input id, or null (every cell is a query cell)
@@ -277,45 +280,61 @@ __device__ __forceinline__ void decode_lid(unsigned long long lid, const FwdGeom
     }
 }
 
-// One row of cell c (see pattern_rows()): the non-empty cells among the row's <= 3 cells
-// (consecutive along the last dimension) have consecutive ranks, so their points are one
-// run [b, b+len) of the lid-ordered storage.  The <= 3 lookups are issued together.
-// Row encoding: byte d = o'_d (d < dim-1 <= 7); byte 7 = lo+1 | (hi+1) << 2 | (pdim+1) << 4,
-// the last-dimension offsets lo..hi and (UNICOMP) the dimension whose coordinate must be odd.
-__device__ __forceinline__ bool eval_row(int j, const long long (&c)[SJ_MAX_DIM], const FwdGeom &g, const Lookup &L,
-                                         const uint32_t *cell_start, uint32_t &b, uint32_t &len) {
-    const unsigned long long off = c_fwd_off[j];
-    const int last = g.dim - 1;
-    const unsigned meta = (unsigned)(off >> 56);
-    const int pdim = (int)(meta >> 4) - 1;
-    if (pdim >= 0) {  // UNICOMP rule (Alg. 2): only cells with an odd coordinate in pdim
-        long long cp = 0;
+// One row of the cell pattern resolved against the grid (host, row_entries()): the linear-id
+// delta of its first cell (offsets o' of the first n-1 dimensions and lo in the last), the
+// dimensions it steps down (neg) / up (pos) in, and its meta byte (see pattern_rows()).
+struct RowEnt {
+    long long delta;  // sum_{d<last} o_d * stride_d + lo
+    unsigned nm;      // bits 0-7: o_d == -1, bits 8-15: o_d == +1 (d < last)
+    unsigned meta;    // lo+1 | (hi+1) << 2 | (pdim+1) << 4
+};
+
+// Per-cell data the rows are tested against: coordinates at the grid's edges and parities.
+struct CellPos {
+    unsigned long long lid;
+    long long clast;  // coordinate in the last dimension
+    unsigned lo_mask, hi_mask, odd_mask;  // c_d == 0 / c_d == nc_d - 1 (d < last); c_d odd (all d)
+};
+
+__device__ __forceinline__ CellPos cell_pos(unsigned long long lid, const FwdGeom &g) {
+    long long c[SJ_MAX_DIM];
+    decode_lid(lid, g, c);
+    CellPos p;
+    p.lid = lid;
+    p.lo_mask = p.hi_mask = p.odd_mask = 0;
+    p.clast = 0;
 #pragma unroll
-        for (int d = 0; d < SJ_MAX_DIM; ++d)
-            if (d == pdim) cp = c[d];
-        if ((cp & 1) == 0) return false;
-    }
-    bool in = true;
-    long long base = 0;
-#pragma unroll
-    for (int d = 0; d < SJ_MAX_DIM - 1; ++d) {
-        if (d < last) {
-            const long long o = (long long)(signed char)((off >> (8 * d)) & 0xFF);
-            const long long v = c[d] + o;
-            in = in && (v >= 0) && (v < (long long)g.nc[d]);
-            base += v * (long long)g.stride[d];
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        if (d < g.dim - 1) {
+            p.lo_mask |= (c[d] == 0 ? 1u : 0u) << d;
+            p.hi_mask |= (c[d] == (long long)g.nc[d] - 1 ? 1u : 0u) << d;
         }
+        if (d < g.dim) p.odd_mask |= (unsigned)(c[d] & 1) << d;
+        if (d == g.dim - 1) p.clast = c[d];
     }
-    if (!in) return false;
-    const int lo = (int)(meta & 3u) - 1, hi = (int)((meta >> 2) & 3u) - 1;
-    const long long x0 = c[last] + lo;
+    return p;
+}
+
+// The non-empty cells among the row's <= 3 cells (consecutive along the last dimension) have
+// consecutive ranks, so their points are one run [b, b+len) of the lid-ordered storage.  The
+// <= 3 lookups are issued together.
+__device__ __forceinline__ bool eval_row(int j, const CellPos &cp, const FwdGeom &g, const Lookup &L,
+                                         const uint32_t *cell_start, uint32_t &b, uint32_t &len) {
+    const RowEnt e = g.rows_ent[j];
+    const int pdim = (int)(e.meta >> 4) - 1;
+    if (pdim >= 0 && !((cp.odd_mask >> pdim) & 1u)) return false;  // UNICOMP rule (Alg. 2)
+    if ((e.nm & cp.lo_mask) | ((e.nm >> 8) & cp.hi_mask)) return false;  // leaves the grid
+    const int lo = (int)(e.meta & 3u) - 1, hi = (int)((e.meta >> 2) & 3u) - 1;
+    const long long x0 = cp.clast + lo;
     const int nx = hi - lo + 1;
+    const long long ncl = (long long)g.nc[g.dim - 1];
+    const unsigned long long base = cp.lid + (unsigned long long)e.delta;
     uint32_t nb[3];
 #pragma unroll
     for (int u = 0; u < 3; ++u) {
         const long long x = x0 + u;
-        const bool ok = u < nx && x >= 0 && x < (long long)g.nc[last];
-        nb[u] = ok ? lookup_cell(L, (unsigned long long)(base + x)) : 0xFFFFFFFFu;
+        const bool ok = u < nx && x >= 0 && x < ncl;
+        nb[u] = ok ? lookup_cell(L, base + (unsigned long long)u) : 0xFFFFFFFFu;
     }
     uint32_t r_lo = 0xFFFFFFFFu, r_hi = 0xFFFFFFFFu;
 #pragma unroll
@@ -337,34 +356,31 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
                                                         const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *rcnt,
                                                         uint32_t *wload, const uint32_t *rbegin, uint2 *runs,
                                                         BuildTotals *tot) {
+    // grid-stride over the cells (M is only known on the device): a bounded grid, so the block
+    // reduction below runs once per resident block, not once per n-sized block
     const uint64_t M = *d_M;
     const uint64_t gt = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const uint64_t r = gt / LPC;
+    const uint64_t cstride = (uint64_t)gridDim.x * blockDim.x / LPC;
     const unsigned sub = (unsigned)(gt % LPC);
     const unsigned lane = threadIdx.x & 31;
     unsigned long long calcs = 0;
     uint32_t w = 0;
-    const bool valid = r < M;  // uniform across the LPC lanes of a cell
-    if (!FILL && r == M && sub == 0) rcnt[M] = 0;  // the scan runs over M + 1 entries
-    if (LPC == 1 ? valid : __any_sync(0xffffffffu, valid)) {
-        long long c[SJ_MAX_DIM];
-        uint32_t m = 0, out = 0;
-        bool qcell = valid;
-        if (valid) {
-            decode_lid(cell_lid[r], g, c);
-            m = cell_start[r + 1] - cell_start[r];
-            if (FILL) out = rbegin[r];
-            if (g.idx) {
-                qcell = g.idx[cell_start[r]] < g.nq;
-                if (!FILL && sub == 0 && qcell != (g.idx[cell_start[r + 1] - 1] < g.nq)) atomicOr(g.mixed, 1u);
-            }
+    if (!FILL && gt == 0) rcnt[M] = 0;  // the scan runs over M + 1 entries
+    for (uint64_t r = gt / LPC; r < M; r += cstride) {  // uniform across the LPC lanes of a cell
+        const CellPos cp = cell_pos(cell_lid[r], g);
+        const uint32_t m = cell_start[r + 1] - cell_start[r];
+        uint32_t out = FILL ? rbegin[r] : 0u;
+        bool qcell = true;
+        if (g.idx) {
+            qcell = g.idx[cell_start[r]] < g.nq;
+            if (!FILL && sub == 0 && qcell != (g.idx[cell_start[r + 1] - 1] < g.nq)) atomicOr(g.mixed, 1u);
         }
         uint32_t cnt = 0;
         unsigned long long summ = 0;
         for (int jb = 0; jb < g.rows; jb += LPC) {
             const int j = jb + (int)sub;
             uint32_t b = 0, len = 0;
-            const bool found = qcell && j < g.rows && eval_row(j, c, g, L, cell_start, b, len);
+            const bool found = qcell && j < g.rows && eval_row(j, cp, g, L, cell_start, b, len);
             if (FILL) {
                 if (LPC == 1) {
                     if (found) runs[out++] = make_uint2(b, len);
@@ -386,19 +402,20 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
                     summ += __shfl_xor_sync(0xffffffffu, summ, o);
                 }
             }
-            if (valid && sub == 0) {
+            if (sub == 0) {
                 rcnt[r] = cnt;
+                uint32_t wr;
                 if (!qcell) {  // halo cell (partitioned index): candidates only
-                    w = 0;
-                    calcs = 0;
+                    wr = 0;
                 } else if (g.full) {  // GCG: every candidate of the 3^n neighbourhood but the query itself
-                    w = (uint32_t)(summ - 1);
-                    calcs = (unsigned long long)m * (summ - 1);
+                    wr = (uint32_t)(summ - 1);
+                    calcs += (unsigned long long)m * (summ - 1);
                 } else {       // half patterns: ceil((m-1)/2) = floor(m/2) home + the forward runs
-                    w = (uint32_t)(m / 2 + summ);
-                    calcs = (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
+                    wr = (uint32_t)(m / 2 + summ);
+                    calcs += (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
                 }
-                wload[r] = w;
+                wload[r] = wr;
+                w = max(w, wr);
             }
         }
     }
@@ -912,18 +929,36 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // ---- a6 + a7: forward runs, workload, D_alg
     std::vector<uint64_t> rows;
     const int R = pattern_rows(dim, ix.pattern, rows);
-    if (R * sizeof(uint64_t) <= 2048) {  // through the pinned mailbox: a truly asynchronous copy
-        memcpy((char *)mail + 1024, rows.data(), R * sizeof(uint64_t));
-        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, (char *)mail + 1024, R * sizeof(uint64_t), 0,
-                                            cudaMemcpyHostToDevice, s));
-    } else {
-        SJ_CUDA_TRY(cudaMemcpyToSymbolAsync(c_fwd_off, rows.data(), R * sizeof(uint64_t), 0, cudaMemcpyHostToDevice, s));
+    // the rows resolved against this grid: linear-id delta, edge masks, meta (eval_row)
+    std::vector<RowEnt> ents(R);
+    for (int j = 0; j < R; ++j) {
+        const uint64_t off = rows[j];
+        const unsigned meta = (unsigned)(off >> 56);
+        long long delta = (long long)(meta & 3u) - 1;  // lo
+        unsigned nm = 0;
+        for (int d = 0; d < dim - 1; ++d) {
+            const int o = (int)(signed char)((off >> (8 * d)) & 0xFF);
+            delta += (long long)o * (long long)ix.stride[d];
+            if (o < 0) nm |= 1u << d;
+            if (o > 0) nm |= 1u << (8 + d);
+        }
+        ents[j] = RowEnt{delta, nm, meta};
+    }
+    RowEnt *d_rows;
+    SJ_TRY(tmp.alloc(&d_rows, R));
+    const size_t rbytes = R * sizeof(RowEnt);
+    if (rbytes <= 3072) {  // through the pinned mailbox: a truly asynchronous copy
+        memcpy((char *)mail + 1024, ents.data(), rbytes);
+        SJ_CUDA_TRY(cudaMemcpyAsync(d_rows, (char *)mail + 1024, rbytes, cudaMemcpyHostToDevice, s));
+    } else {  // pageable: staged by the driver before the call returns
+        SJ_CUDA_TRY(cudaMemcpyAsync(d_rows, ents.data(), rbytes, cudaMemcpyHostToDevice, s));
     }
     FwdGeom fg{};
     fg.dim = dim;
     fg.rows = R;
     fg.small = ncells_total <= 0xFFFFFFFFull ? 1 : 0;
     fg.full = ix.pattern == SJ_PATTERN_GCG ? 1 : 0;
+    fg.rows_ent = d_rows;
     unsigned int *d_mixed = nullptr;
     if (part) {
         SJ_TRY(tmp.alloc_zero(&d_mixed, 1));
@@ -941,13 +976,21 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wload, n));
     SJ_TRY(tmp.alloc_zero(&d_tot, 1));
     const bool wide = R >= 16;  // one warp per cell for many rows
-    // (n + 1 cells' worth of threads: the one with r == M zeroes rcnt[M] for the scan below)
+    // grid-stride kernels (M is on the device): at most 8 resident blocks per SM
+    int nsm = 148;
+    {
+        int dev = 0;
+        if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    }
+    auto runs_grid = [&](uint64_t cells, int lpc) {
+        return std::min<unsigned>(grid_for(cells * (uint64_t)lpc), (unsigned)nsm * 8u);
+    };
     if (wide)
-        runs_kernel<false, 32><<<grid_for((n + 1) * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt,
-                                                                           wload, nullptr, nullptr, d_tot);
+        runs_kernel<false, 32><<<runs_grid(n, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
+                                                                    nullptr, nullptr, d_tot);
     else
-        runs_kernel<false, 1><<<grid_for(n + 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                   nullptr, nullptr, d_tot);
+        runs_kernel<false, 1><<<runs_grid(n, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
+                                                                  nullptr, nullptr, d_tot);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin;
@@ -996,10 +1039,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     ix.runs_cap = bounded ? runs_bound : E + 2;
     SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
     if (wide)
-        runs_kernel<true, 32><<<grid_for(M * 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
+        runs_kernel<true, 32><<<runs_grid(M, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
                                                                     rbegin, ix.runs, nullptr);
     else
-        runs_kernel<true, 1><<<grid_for(M), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
+        runs_kernel<true, 1><<<runs_grid(M, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
                                                               rbegin, ix.runs, nullptr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
