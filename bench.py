@@ -399,7 +399,9 @@ def main():
                        "output": "HBM-resident pairs (uint32 x2), written in place"},
             "self_join_s": total_ms / args.steps / 1e3,
             "phases_ms": {"build": statistics.mean(build_ms), "estimate": statistics.mean(est_ms),
-                          "join": mean_join_ms, "step": total_ms / args.steps},
+                          "join": mean_join_ms, "step": total_ms / args.steps,
+                          "join_min": min(join_ms), "join_max": max(join_ms),
+                          "step_min": min(step_ms), "step_max": max(step_ms)},
             "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": e2e,
