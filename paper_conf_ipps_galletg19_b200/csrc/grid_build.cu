@@ -363,13 +363,15 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
     const uint64_t cstride = (uint64_t)gridDim.x * blockDim.x / LPC;
     const unsigned sub = (unsigned)(gt % LPC);
     const unsigned lane = threadIdx.x & 31;
-    unsigned long long calcs = 0;
+    unsigned long long calcs = 0, nruns = 0;
     uint32_t w = 0;
     if (!FILL && gt == 0) rcnt[M] = 0;  // the scan runs over M + 1 entries
     for (uint64_t r = gt / LPC; r < M; r += cstride) {  // uniform across the LPC lanes of a cell
         const CellPos cp = cell_pos(cell_lid[r], g);
         const uint32_t m = cell_start[r + 1] - cell_start[r];
-        uint32_t out = FILL ? rbegin[r] : 0u;
+        // FILL: the compacted layout (rbegin = scan of the counts); counting with `runs` set: the
+        // slot layout, cell r's runs at r * rows (no second pass, no scan)
+        uint32_t out = FILL ? rbegin[r] : (uint32_t)(r * (uint64_t)g.rows);
         bool qcell = true;
         if (g.idx) {
             qcell = g.idx[cell_start[r]] < g.nq;
@@ -381,7 +383,7 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
             const int j = jb + (int)sub;
             uint32_t b = 0, len = 0;
             const bool found = qcell && j < g.rows && eval_row(j, cp, g, L, cell_start, b, len);
-            if (FILL) {
+            if (FILL || runs) {
                 if (LPC == 1) {
                     if (found) runs[out++] = make_uint2(b, len);
                 } else {
@@ -389,7 +391,8 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
                     if (found) runs[out + __popc(fm & ((1u << lane) - 1u))] = make_uint2(b, len);
                     out += __popc(fm);
                 }
-            } else if (found) {
+            }
+            if (!FILL && found) {
                 ++cnt;
                 summ += len;
             }
@@ -404,6 +407,7 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
             }
             if (sub == 0) {
                 rcnt[r] = cnt;
+                nruns += cnt;
                 uint32_t wr;
                 if (!qcell) {  // halo cell (partitioned index): candidates only
                     wr = 0;
@@ -420,24 +424,28 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
         }
     }
     if (!FILL) {  // block reduction, then ONE pair of global atomics per block
-        __shared__ unsigned long long s_calcs[kThreads / 32];
+        __shared__ unsigned long long s_calcs[kThreads / 32], s_runs[kThreads / 32];
         __shared__ uint32_t s_w[kThreads / 32];
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             calcs += __shfl_xor_sync(0xffffffffu, calcs, o);
+            nruns += __shfl_xor_sync(0xffffffffu, nruns, o);
             w = max(w, __shfl_xor_sync(0xffffffffu, w, o));
         }
         if (lane == 0) {
             s_calcs[threadIdx.x >> 5] = calcs;
+            s_runs[threadIdx.x >> 5] = nruns;
             s_w[threadIdx.x >> 5] = w;
         }
         __syncthreads();
         if (threadIdx.x == 0) {
             for (int i = 1; i < kThreads / 32; ++i) {
                 calcs += s_calcs[i];
+                nruns += s_runs[i];
                 w = max(w, s_w[i]);
             }
             if (calcs) atomicAdd(&tot->dist_calcs, calcs);
+            if (nruns) atomicAdd(&tot->E, nruns);
             if (w) atomicMax(&tot->max_w, w);
         }
     }
@@ -465,6 +473,7 @@ __global__ void __launch_bounds__(kThreads) queue_m_kernel(const uint32_t *qorde
 
 __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t *qorder, const uint32_t *qb,
                                                                   const uint32_t *cell_start, const uint32_t *rbegin,
+                                                                  uint32_t slot_rows,
                                                                   const uint32_t *wload,
                                                                   const unsigned long long *cell_lid, uint64_t M,
                                                                   int full, uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
@@ -473,8 +482,9 @@ __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t
     if (i >= M) return;
     uint32_t r = qorder[i];
     uint32_t m = cell_start[r + 1] - cell_start[r];
+    const uint32_t rb = rbegin ? rbegin[r] : r * slot_rows;  // first forward run
     if (idx && idx[cell_start[r]] >= nq) {  // halo cell: never queued (m = 0 in its record)
-        cellq[i] = make_uint4(cell_start[r], 0u, rbegin[r], 0u);
+        cellq[i] = make_uint4(cell_start[r], 0u, rb, 0u);
         r2q[r] = (uint32_t)i;
         qbr[r] = qb[i];
         lid_q[i] = cell_lid[r];
@@ -482,7 +492,7 @@ __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t
     }
     // {begin in the lid-ordered storage, m, first run, S = sum of the runs' lengths}
     // (half patterns: W = floor(m/2) + S; GCG: W = S - 1, the query itself excluded)
-    cellq[i] = make_uint4(cell_start[r], m, rbegin[r], full ? wload[r] + 1 : wload[r] - m / 2);
+    cellq[i] = make_uint4(cell_start[r], m, rb, full ? wload[r] + 1 : wload[r] - m / 2);
     r2q[r] = (uint32_t)i;
     qbr[r] = qb[i];
     lid_q[i] = cell_lid[r];
@@ -976,6 +986,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wload, n));
     SJ_TRY(tmp.alloc_zero(&d_tot, 1));
     const bool wide = R >= 16;  // one warp per cell for many rows
+    // Slot layout (1-D..3-D at the configs' sizes): cell r's runs at r * R, written by the counting
+    // pass itself -- no scan, no second pass; the array is sized by n >= M before M is known.
+    const bool slots = (uint64_t)n * R * sizeof(uint2) <= (512ull << 20);
+    if (slots) {
+        ix.runs_cap = (uint64_t)n * R + 2;
+        SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
+    }
     // grid-stride kernels (M is on the device): at most 8 resident blocks per SM
     int nsm = 148;
     {
@@ -987,14 +1004,14 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     };
     if (wide)
         runs_kernel<false, 32><<<runs_grid(n, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                    nullptr, nullptr, d_tot);
+                                                                    nullptr, slots ? ix.runs : nullptr, d_tot);
     else
         runs_kernel<false, 1><<<runs_grid(n, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                  nullptr, nullptr, d_tot);
+                                                                  nullptr, slots ? ix.runs : nullptr, d_tot);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
-    uint32_t *rbegin;
-    SJ_TRY(tmp.alloc(&rbegin, n + 1));
+    uint32_t *rbegin = nullptr;
+    if (!slots) SJ_TRY(tmp.alloc(&rbegin, n + 1));
     // host round trip 2: M, plus the workload totals (max W sizes the SortByWL keys, D_alg)
     SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_M, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 64, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
@@ -1021,13 +1038,17 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // device-sized launch needs no host round trip after the build)
     SJ_TRY(dev_alloc_t(&ix.d_meta, 4, s));
     uint32_t *d_E32 = ix.d_meta + 1;
-    SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s, &tmp.ws));
+    if (!slots) SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s, &tmp.ws));
     // The runs array is allocated at its bound M * rows when that is small (every 1-D..4-D
     // index), so the run total E is read with the final round trip instead of a third one.
     const uint64_t runs_bound = M * (uint64_t)R + 2;
-    const bool bounded = runs_bound * sizeof(uint2) <= (256ull << 20);
+    const bool bounded = slots || runs_bound * sizeof(uint2) <= (256ull << 20);
     uint64_t E = 0;
-    if (!bounded) {
+    if (slots) {
+        E = bt.E;
+        ix.n_runs = E;
+        ix.runs_len = M * (uint64_t)R;
+    } else if (!bounded) {
         SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         SJ_CUDA_TRY(cudaStreamSynchronize(s));
         debug_mark("build: scan sync");
@@ -1036,9 +1057,13 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         E = E32;
         ix.n_runs = E;
     }
-    ix.runs_cap = bounded ? runs_bound : E + 2;
-    SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
-    if (wide)
+    if (!slots) {
+        ix.runs_cap = bounded ? runs_bound : E + 2;
+        SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
+    }
+    if (slots) {
+        // (the counting pass wrote them)
+    } else if (wide)
         runs_kernel<true, 32><<<runs_grid(M, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
                                                                     rbegin, ix.runs, nullptr);
     else
@@ -1079,7 +1104,8 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     uint32_t *r2q, *qbr;
     SJ_TRY(tmp.alloc(&r2q, M));
     SJ_TRY(tmp.alloc(&qbr, M));
-    cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, rbegin, wload, cell_lid, M,
+    cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, rbegin, (uint32_t)R, wload,
+                                                           cell_lid, M,
                                                            fg.full, ix.cellq, r2q, qbr, ix.cell_lid,
                                                            part ? idx_sorted : nullptr, (uint32_t)nq);
     note_launch();
@@ -1105,7 +1131,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         // stream has passed ev1 (the join reads n_chunks on the device meanwhile)
         tail_mail[0] = tail_mail[1] = 0;
         SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-        if (bounded)
+        if (bounded && !slots)  // E from the scan of the counts
             SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail + 1, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         else
             tail_mail[1] = E;
@@ -1113,7 +1139,8 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         return SJ_OK;
     }
     SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 512, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    if (bounded) SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    if (bounded && !slots)
+        SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 256, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     if (ev1) SJ_CUDA_TRY(cudaEventRecord(ev1, s));
     debug_mark("build: tail issued");
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
@@ -1122,7 +1149,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     uint32_t nchunks;
     memcpy(&nchunks, (char *)mail + 512, sizeof nchunks);
     ix.n_chunks = nchunks;
-    if (bounded) {
+    if (bounded && !slots) {
         uint32_t E32;
         memcpy(&E32, (char *)mail + 256, sizeof E32);
         ix.n_runs = E32;

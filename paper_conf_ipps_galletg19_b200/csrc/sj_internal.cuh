@@ -145,7 +145,10 @@ struct Index {
     uint64_t n_query = 0;       // queries: D' positions [0, n_query) (n unless partitioned)
     uint32_t *d_meta = nullptr; // [4]        device {n_chunks, E}, written by the build
     uint64_t runs_cap = 0;      // entries allocated for runs (>= E + 2)
+    uint64_t runs_len = 0;      // entries the cells' run indices span: M * rows in the slot
+                                // layout (cell r's runs at r * rows), 0 = compact (E)
 };
+inline uint64_t runs_entries(const Index &ix) { return ix.runs_len ? ix.runs_len : ix.n_runs; }
 
 struct BuildTimes {
     float ms = 0;

@@ -350,7 +350,7 @@ JoinArgs base_args(const sj_handle *h) {
     a.runs = h->ix.runs;
     a.chunks = h->ix.chunks;
     a.n_chunks = (uint32_t)h->ix.n_chunks;
-    a.n_runs = h->ix.n_runs;
+    a.n_runs = h->ix.runs_cap ? h->ix.runs_cap : h->ix.n_runs;  // bound of the run reads: the allocation
     a.e2 = h->ix.e2;
     a.grab = h->grab;
     a.v_stride = 1;
@@ -1353,7 +1353,7 @@ int sj_get_stats(const sj_handle *h, sj_stats *s) {
 // ---------------------------------------------------------------- index export / import
 namespace {
 struct BlobHeader {
-    uint64_t magic;  // "SJIDX003"
+    uint64_t magic;  // "SJIDX004"
     uint64_t n;
     int32_t dim, pad, key_bits, pattern_order;
     double eps, e2, w;
@@ -1365,8 +1365,9 @@ struct BlobHeader {
     uint64_t off[7], bytes[7];  // pts, orig, qmap, cellq, runs, cell_lid, chunks
     uint64_t total;
     uint64_t n_query;  // queries of a partitioned index (D' positions [0, n_query))
+    uint64_t runs_len; // entries of the runs array (slot layout: M * rows; else = n_runs)
 };
-constexpr uint64_t kMagic = 0x3330305844494a53ull;  // "SJIDX003"
+constexpr uint64_t kMagic = 0x3430305844494a53ull;  // "SJIDX004"
 constexpr uint64_t kHdr = 1024;
 static_assert(sizeof(BlobHeader) <= kHdr, "header");
 
@@ -1392,7 +1393,7 @@ BlobHeader make_header(const Index &ix) {
     b.dist_calcs = ix.dist_calcs;
     b.max_w = ix.max_w;
     const uint64_t sz[7] = {ix.n * ix.pad * sizeof(double), ix.n * sizeof(uint32_t), ix.n * sizeof(uint2),
-                            ix.n_cells * sizeof(uint4), ix.n_runs * sizeof(uint2), ix.n_cells * sizeof(uint64_t),
+                            ix.n_cells * sizeof(uint4), runs_entries(ix) * sizeof(uint2), ix.n_cells * sizeof(uint64_t),
                             (ix.n_chunks + 1) * sizeof(uint32_t)};
     uint64_t o = kHdr;
     for (int i = 0; i < 7; ++i) {
@@ -1402,6 +1403,7 @@ BlobHeader make_header(const Index &ix) {
     }
     b.total = o;
     b.n_query = ix.n_query;
+    b.runs_len = ix.runs_len;
     return b;
 }
 }  // namespace
@@ -1466,6 +1468,8 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
     }
     ix.n_cells = b.n_cells;
     ix.n_runs = b.n_runs;
+    ix.runs_len = b.runs_len;
+    ix.runs_cap = runs_entries(ix) + 2;
     ix.n_chunks = b.n_chunks;
     ix.n_query = b.n_query ? b.n_query : b.n;
     ix.dist_calcs = b.dist_calcs;

@@ -85,12 +85,20 @@ def parse_blob(blob: np.ndarray):
 
 
 def runs_per_cell(ix):
+    """Runs of each cell: from its first run (cellq.z), the runs whose lengths add up to the
+    cell's forward candidates (cellq.w) -- valid for the compact layout and for the slot
+    layout (cell r's runs at r * rows, unused slots never read)."""
     z = ix["cellq"][:, 2].astype(np.int64)
-    order = np.argsort(z, kind="stable")
-    counts = np.empty_like(z)
-    zs = z[order]
-    nxt = np.append(zs[1:], ix["n_runs"])
-    counts[order] = nxt - zs
+    S = ix["cellq"][:, 3].astype(np.int64)
+    lens = ix["runs"][:, 1].astype(np.int64)
+    counts = np.zeros_like(z)
+    for c in range(z.shape[0]):
+        acc, k = 0, 0
+        while acc < S[c]:
+            acc += lens[z[c] + k]
+            k += 1
+        assert acc == S[c]
+        counts[c] = k
     return counts
 
 
