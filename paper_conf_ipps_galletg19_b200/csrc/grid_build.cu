@@ -501,14 +501,13 @@ __global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t
 // Points gathered into lid (spatial) order, padded AoS, plus D' = the queue as an index
 // array: qmap[D' position] = {lid-storage position, queue-order cell}.  With
 // input_order the queue is the input order itself (the ablation's unsorted D).
-__global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, uint64_t n, int dim, int pad,
-                                                           const uint32_t *idx_sorted, const uint32_t *cellof,
-                                                           const uint32_t *cell_start, const uint32_t *qbr,
-                                                           const uint32_t *r2q, double *pts, uint32_t *orig,
-                                                           uint2 *qmap, int input_order, const uint32_t *ids) {
+// Two kernels, so the gather (the larger, depending only on the point sort) runs on a side
+// stream while the main stream resolves runs, sorts cells and builds the queue.
+__global__ void __launch_bounds__(kThreads) gather_kernel(const double *raw, uint64_t n, int dim, int pad,
+                                                          const uint32_t *idx_sorted, double *pts, uint32_t *orig,
+                                                          const uint32_t *ids) {
     uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
-    const uint32_t r = cellof[p];
     const uint32_t src = idx_sorted[p];
     if (pad == 2 && dim == 2) {
         reinterpret_cast<double2 *>(pts)[p] = reinterpret_cast<const double2 *>(raw)[src];
@@ -516,7 +515,14 @@ __global__ void __launch_bounds__(kThreads) permute_kernel(const double *raw, ui
         for (int d = 0; d < pad; ++d) pts[p * pad + d] = d < dim ? raw[(uint64_t)src * dim + d] : 0.0;
     }
     orig[p] = ids ? ids[src] : src;  // partitioned index: the caller's global ids
-    const uint64_t dest = input_order ? (uint64_t)src : (uint64_t)qbr[r] + (p - cell_start[r]);
+}
+__global__ void __launch_bounds__(kThreads) qmap_kernel(uint64_t n, const uint32_t *idx_sorted, const uint32_t *cellof,
+                                                        const uint32_t *cell_start, const uint32_t *qbr,
+                                                        const uint32_t *r2q, uint2 *qmap, int input_order) {
+    uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    const uint32_t r = cellof[p];
+    const uint64_t dest = input_order ? (uint64_t)idx_sorted[p] : (uint64_t)qbr[r] + (p - cell_start[r]);
     qmap[dest] = make_uint2((uint32_t)p, r2q[r]);
 }
 
@@ -801,8 +807,17 @@ static int rle(const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *ce
 }
 
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s, cudaEvent_t ev0,
-                cudaEvent_t ev1, float *ms, const BuildPart *part, uint64_t *tail_mail) {
+                cudaEvent_t ev1, float *ms, const BuildPart *part, uint64_t *tail_mail, const BuildSide *side) {
     Temps tmp(s);
+    // on every exit, the main stream waits for the side stream before the temporaries are freed
+    // (stream-ordered, on s) -- also on the error returns
+    struct SideJoin {
+        const BuildSide *side;
+        cudaStream_t s;
+        ~SideJoin() {
+            if (side && cudaEventRecord(side->ej, side->s2) == cudaSuccess) cudaStreamWaitEvent(s, side->ej, 0);
+        }
+    } side_join{side, s};
     ix.n = n;
     const uint64_t nq = part ? part->n_query : n;  // queries: input points [0, nq)
     ix.n_query = nq;
@@ -913,6 +928,18 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         SJ_TRY(sort_points<uint64_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
         SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
     }
+    // the gather of the points into cell order needs only the point sort: side stream
+    SJ_TRY(dev_alloc_t(&ix.pts, n * ix.pad, s));
+    SJ_TRY(dev_alloc_t(&ix.orig, n, s));
+    cudaStream_t sg = side ? side->s2 : s;
+    if (side) {
+        SJ_CUDA_TRY(cudaEventRecord(side->ea, s));
+        SJ_CUDA_TRY(cudaStreamWaitEvent(sg, side->ea, 0));
+    }
+    gather_kernel<<<grid_for(n), kThreads, 0, sg>>>(d_raw, n, dim, ix.pad, idx_sorted, ix.pts, ix.orig,
+                                                     part ? part->d_ids : nullptr);
+    note_launch();
+    if (side) SJ_CUDA_TRY(cudaEventRecord(side->eg, sg));
     if (dense) {
         uint32_t *tab;
         SJ_TRY(tmp.alloc(&tab, ncells_total));
@@ -1098,8 +1125,6 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // ---- final arrays
     SJ_TRY(dev_alloc_t(&ix.cellq, M, s));
     SJ_TRY(dev_alloc_t(&ix.cell_lid, M, s));
-    SJ_TRY(dev_alloc_t(&ix.pts, n * ix.pad, s));
-    SJ_TRY(dev_alloc_t(&ix.orig, n, s));
     SJ_TRY(dev_alloc_t(&ix.qmap, n, s));
     uint32_t *r2q, *qbr;
     SJ_TRY(tmp.alloc(&r2q, M));
@@ -1109,10 +1134,19 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
                                                            fg.full, ix.cellq, r2q, qbr, ix.cell_lid,
                                                            part ? idx_sorted : nullptr, (uint32_t)nq);
     note_launch();
-    permute_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, dim, ix.pad, idx_sorted, cellof, cell_start, qbr, r2q,
-                                                    ix.pts, ix.orig, ix.qmap, ix.order == SJ_ORDER_INPUT ? 1 : 0,
-                                                    part ? part->d_ids : nullptr);
+    // D' (qmap): after the cells' queue positions; on the side stream too (the chunk scan below
+    // needs it only in input order), the main stream waits for it before the build ends
+    if (side) {
+        SJ_CUDA_TRY(cudaEventRecord(side->ea, s));
+        SJ_CUDA_TRY(cudaStreamWaitEvent(sg, side->ea, 0));
+    }
+    qmap_kernel<<<grid_for(n), kThreads, 0, sg>>>(n, idx_sorted, cellof, cell_start, qbr, r2q, ix.qmap,
+                                                  ix.order == SJ_ORDER_INPUT ? 1 : 0);
     note_launch();
+    if (side) {
+        SJ_CUDA_TRY(cudaEventRecord(side->eq, sg));
+        if (ix.order == SJ_ORDER_INPUT) SJ_CUDA_TRY(cudaStreamWaitEvent(s, side->eq, 0));
+    }
     SJ_CUDA_TRY(cudaGetLastError());
 
     // ---- WorkQueue chunks over D'
@@ -1126,6 +1160,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     else
         SJ_TRY(scan_fused(M, CellChunkLoad{ix.cellq, qb, big_min}, CellChunkStore{ix.cellq, qb, big_min, ix.chunks}, s,
                           ChunkDone{nq, ix.chunks, d_nc}, &tmp.ws));
+    if (side) {
+        SJ_CUDA_TRY(cudaStreamWaitEvent(s, side->eq, 0));  // points, ids and D' complete
+        // the caller's points are read by the gather last: done before sj_create returns
+        SJ_CUDA_TRY(cudaEventSynchronize(side->eg));
+    }
     if (tail_mail) {
         // no final round trip: {n_chunks, E} land in the caller's pinned mailbox, read once the
         // stream has passed ev1 (the join reads n_chunks on the device meanwhile)

@@ -164,10 +164,18 @@ struct BuildPart {
     uint64_t n_query = 0;
 };
 
+// Side stream of the build (the gather of the points into cell order and D' run there,
+// overlapping the main stream's forward runs, cell sort and queue); ea: main -> side, eg: the
+// gather done, eq: D' done, ej: side -> main at exit.  nullptr: everything on the main stream.
+struct BuildSide {
+    cudaStream_t s2;
+    cudaEvent_t ea, eg, eq, ej;
+};
+
 // Builds the index from device-resident raw points (n x dim AoS).  Returns sj_status.
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s,
                 cudaEvent_t ev0, cudaEvent_t ev1, float *ms, const BuildPart *part = nullptr,
-                uint64_t *tail_mail = nullptr);
+                uint64_t *tail_mail = nullptr, const BuildSide *side = nullptr);
 // tail_mail (pinned host, 2 words): the build ends without a host round trip; {n_chunks, E}
 // arrive there once the stream passes ev1, and ix.n_chunks / ix.n_runs / *ms stay unset
 // until the caller reads them (sj_runtime.cu: ix_ready).  nullptr: synchronous, all set.

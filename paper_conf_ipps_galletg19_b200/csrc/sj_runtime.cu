@@ -138,6 +138,7 @@ struct sj_handle {
     cudaStream_t s_main = nullptr;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr, ev_c = nullptr, ev_d = nullptr, ev_e = nullptr;
     cudaEvent_t ev_ba = nullptr, ev_bb = nullptr;  // build start / end
+    sj::BuildSide side{};                         // the build's side stream and its events
     int pending = 0;  // 1: the build's tail {n_chunks, E} and its timing not read yet (ix_ready)
     sj::Index ix;
     bool owns_index = true;
@@ -198,6 +199,7 @@ struct Core {
     int num_sms;
     cudaStream_t s;
     cudaEvent_t ev[7];
+    sj::BuildSide side;
     unsigned long long *d_ctr;
     uint64_t *mail;
 };
@@ -221,6 +223,7 @@ int handle_init_common(sj_handle *h) {
                 h->ev_e = c.ev[4];
                 h->ev_ba = c.ev[5];
                 h->ev_bb = c.ev[6];
+                h->side = c.side;
                 h->d_ctr = c.d_ctr;
                 h->mail = c.mail;
                 return SJ_OK;
@@ -228,7 +231,11 @@ int handle_init_common(sj_handle *h) {
     }
     pool_setup(h->device);
     SJ_CUDA_TRY(cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, h->device));
-    SJ_CUDA_TRY(cudaStreamCreateWithFlags(&h->s_main, cudaStreamNonBlocking));
+    // priorities: the build's side stream (the gather of the points, D') yields the SMs to the
+    // main stream's critical path, block by block
+    int prio_least = 0, prio_greatest = 0;
+    SJ_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&prio_least, &prio_greatest));
+    SJ_CUDA_TRY(cudaStreamCreateWithPriority(&h->s_main, cudaStreamNonBlocking, prio_greatest));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_a));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_b));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_c));
@@ -236,6 +243,11 @@ int handle_init_common(sj_handle *h) {
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_e));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_ba));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_bb));
+    SJ_CUDA_TRY(cudaStreamCreateWithPriority(&h->side.s2, cudaStreamNonBlocking, prio_least));
+    SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.ea, cudaEventDisableTiming));
+    SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.eg, cudaEventDisableTiming));
+    SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.eq, cudaEventDisableTiming));
+    SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.ej, cudaEventDisableTiming));
     h->mail = static_cast<uint64_t *>(pinned_acquire());
     if (!h->mail) return SJ_ENOMEM;
     SJ_TRY(dev_alloc_t(&h->d_ctr, 8, h->s_main));
@@ -245,15 +257,19 @@ int handle_init_common(sj_handle *h) {
 // Returns the handle's core to the cache (stream drained first); false if it must be freed.
 bool core_release(sj_handle *h) {
     if (!h->s_main || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->ev_e || !h->ev_ba || !h->ev_bb || !h->d_ctr ||
-        !h->mail)
+        !h->mail || !h->side.s2 || !h->side.ea || !h->side.eg || !h->side.eq || !h->side.ej)
         return false;
+    if (cudaStreamSynchronize(h->side.s2) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
     if (cudaStreamSynchronize(h->s_main) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
     std::lock_guard<std::mutex> lk(g_core_mu);
     if (g_core_cache.size() >= 64) return false;
-    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e, h->ev_ba, h->ev_bb}, h->d_ctr,
+    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e, h->ev_ba, h->ev_bb}, h->side, h->d_ctr,
                                 h->mail});
     return true;
 }
@@ -1197,7 +1213,7 @@ static sj_handle *create_impl(const double *points, uint64_t n, int dim, double 
     }();
     if (rc == SJ_OK)
         rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_ba, h->ev_bb, &ms, origin ? &part : nullptr,
-                         sync_build ? nullptr : h->mail + 48);
+                         sync_build ? nullptr : h->mail + 48, h->side.s2 ? &h->side : nullptr);
     debug_mark("create: build_index");
     dev_free(d_copy, s);
     dev_free(d_ids, s);
@@ -1279,6 +1295,14 @@ void sj_destroy(sj_handle *h) {
         if (h->ev_e) cudaEventDestroy(h->ev_e);
         if (h->ev_ba) cudaEventDestroy(h->ev_ba);
         if (h->ev_bb) cudaEventDestroy(h->ev_bb);
+        if (h->side.s2) {
+            cudaStreamSynchronize(h->side.s2);
+            cudaStreamDestroy(h->side.s2);
+        }
+        if (h->side.ea) cudaEventDestroy(h->side.ea);
+        if (h->side.eg) cudaEventDestroy(h->side.eg);
+        if (h->side.eq) cudaEventDestroy(h->side.eq);
+        if (h->side.ej) cudaEventDestroy(h->side.ej);
         pinned_release(h->mail);
     }
     delete h;

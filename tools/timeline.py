@@ -7,6 +7,7 @@ step's first GPU activity, its duration and the idle gap before it, then the tot
 (busy vs idle).  Diagnostic only; the numbers are not bench values.
 """
 import sys
+import time
 
 import torch
 from torch.profiler import ProfilerActivity, profile
@@ -40,14 +41,22 @@ marks = []
 with profile(activities=[ProfilerActivity.CUDA, ProfilerActivity.CPU]) as prof:
     for _ in range(steps):
         torch.cuda.synchronize()
+        time.sleep(0.02)  # an idle gap that separates the steps on the GPU timeline
         with torch.profiler.record_function('STEP'):
             st = step()
         torch.cuda.synchronize()
-evs = [e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA]
+evs = [e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA and e.name != 'STEP']
 steps_cpu = [e for e in prof.events() if e.name == 'STEP']
 last = steps_cpu[-1]
 t0c, t1c = last.time_range.start, last.time_range.end
-gpu = sorted([e for e in evs if t0c <= e.time_range.start <= t1c + 50000], key=lambda e: e.time_range.start)
+allg = sorted(evs, key=lambda e: e.time_range.start)
+# the last step = the GPU activity after the last idle gap of > 10 ms (CPU and GPU clocks may be
+# skewed, and sj_create returns before its kernels ran, so the CPU range does not bracket it)
+cut = 0
+for i in range(1, len(allg)):
+    if allg[i].time_range.start - max(e.time_range.end for e in allg[max(0, i - 64):i]) > 10000:
+        cut = i
+gpu = allg[cut:]
 if not gpu:
     print('no gpu events')
     sys.exit(0)
