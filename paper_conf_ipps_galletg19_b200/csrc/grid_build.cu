@@ -1013,9 +1013,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&wload, n));
     SJ_TRY(tmp.alloc_zero(&d_tot, 1));
     const bool wide = R >= 16;  // one warp per cell for many rows
-    // Slot layout (1-D..3-D at the configs' sizes): cell r's runs at r * R, written by the counting
-    // pass itself -- no scan, no second pass; the array is sized by n >= M before M is known.
-    const bool slots = (uint64_t)n * R * sizeof(uint2) <= (512ull << 20);
+    // Slot layout: cell r's runs at r * R, written by the counting pass itself -- no scan, no
+    // second pass, no third host round trip; the array is sized by n >= M before M is known
+    // (up to 4 GB of the 180 GB: every configuration, 6-D at 2M points included: 1.95 GB).
+    const bool slots = (uint64_t)n * R * sizeof(uint2) <= (4ull << 30);
     if (slots) {
         ix.runs_cap = (uint64_t)n * R + 2;
         SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
