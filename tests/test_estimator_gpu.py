@@ -127,3 +127,21 @@ def test_lazy_first_join_overflow():
     got, rc, st, total, _ = _first_call_join(pts, cfg.eps, cap=64, sample_ppm=100_000)
     assert rc == 1 and got.shape[0] == 64  # SJ_MORE
     assert st["est_pairs"] == ref["est_pairs"]
+
+
+def test_points_reusable_when_create_returns():
+    # sj_create may return before the build's last kernels ran (lazy tail), but never before the
+    # last read of the caller's points: overwriting them right away must not change the result
+    cfg = workloads.get_config("c5").scaled(200_003)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    d = torch.from_numpy(np.ascontiguousarray(pts)).to(DEV)
+    out = torch.empty((want.shape[0], 2), dtype=torch.int32, device=DEV)
+    for _ in range(2):
+        d.copy_(torch.from_numpy(pts))
+        torch.cuda.synchronize()
+        with sj.Handle(d, cfg.eps, k=8) as h:
+            d.fill_(float("nan"))  # torch's stream, right after sj_create returned
+            rc, got = h.self_join(out, want.shape[0])
+        assert rc == 0 and got == want.shape[0]
+        np.testing.assert_array_equal(oracle.canonical(out.cpu().numpy().view(np.uint32).reshape(-1, 2)), want)
