@@ -48,12 +48,110 @@ struct BBox {
     unsigned long long mn_c[SJ_MAX_DIM];  // ~ordered_key(min)
     unsigned long long mx[SJ_MAX_DIM];
     unsigned int nonfinite;
+    unsigned int done;  // blocks finished (the last one derives the grid geometry)
 };
 
-// a2: exact per-dimension min/max (order-independent) + non-finite check (a1 validation).
-// The coordinates are read as a flat array of double2; the total thread count T is chosen
-// with 2T % dim == 0, so every thread always sees the same two dimensions.
-__global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint64_t n, int dim, BBox *bb) {
+// The grid geometry (a3, readings c5-c7), derived on the device by the bounding box's last
+// block: the cell-id kernel reads it from device memory and the host reads the copy written
+// into its pinned mailbox (zero-copy, behind `flag`), so the first kernels after the bounding
+// box are queued without a host round trip in between.
+struct GeomDev {
+    double mins[SJ_MAX_DIM];
+    unsigned long long nc[SJ_MAX_DIM];
+    unsigned long long stride[SJ_MAX_DIM];
+    double w;
+    double errq;
+    int dim, key_bits;
+    int err;     // 0 ok, 1 non-finite coordinate, 2 below the given origin, 3 quotient >= 2^30, 4 cells >= 2^64
+    int errdim;
+    unsigned flag;  // host copy: the build's epoch once the fields are written
+    unsigned pad;
+};
+struct GeomArgs {
+    double w;
+    double origin[SJ_MAX_DIM];
+    int has_origin;
+    GeomDev *dev;        // device copy (read by cell_id_kernel)
+    GeomDev *host;       // pinned host copy, or nullptr
+    unsigned epoch;
+};
+
+// Called by the first warp of the bounding box's last block: lane d handles dimension d.
+__device__ void derive_geometry(const BBox *bb, int dim, const GeomArgs &ga) {
+    const int lane = threadIdx.x & 31;
+    const volatile BBox *vb = bb;
+    int err = vb->nonfinite ? 1 : 0, errdim = 0;
+    double mn = 0, q = 0;
+    unsigned long long nc = 1;
+    int my_err = 0;
+    if (lane < dim && !err) {
+        mn = from_ordered_key(~vb->mn_c[lane]);
+        const double mx = from_ordered_key(vb->mx[lane]);
+        if (ga.has_origin) {  // partition of a larger grid: its origin (all partitions' cells align)
+            if (!(ga.origin[lane] <= mn) || !isfinite(ga.origin[lane])) my_err = 2;
+            mn = ga.origin[lane];
+        }
+        // nc_d = max c_d + 1; c_d is monotone in x_d so max c_d = c_d(max x_d)
+        q = __ddiv_rn(__dsub_rn(mx, mn), ga.w);
+        if (!my_err && !(q < 0x1p30)) my_err = 3;
+        if (!my_err) nc = (unsigned long long)floor(q) + 1ull;
+    }
+    const unsigned emask = __ballot_sync(0xffffffffu, my_err != 0);
+    if (!err && emask) {
+        errdim = __ffs(emask) - 1;
+        err = __shfl_sync(0xffffffffu, my_err, errdim);
+    }
+    const double errq = __shfl_sync(0xffffffffu, q, errdim);
+    GeomDev *g = ga.dev;
+    if (lane < dim) {
+        g->mins[lane] = mn;
+        g->nc[lane] = nc;
+    }
+    unsigned long long ncd[SJ_MAX_DIM];  // every lane: the counts of all dimensions
+#pragma unroll
+    for (int d = 0; d < SJ_MAX_DIM; ++d) ncd[d] = __shfl_sync(0xffffffffu, nc, d);
+    if (lane == 0) {
+        unsigned long long total = 1;
+        for (int d = 0; d < dim && !err; ++d) {
+            if (total > ~0ull / ncd[d] || total * ncd[d] == ~0ull) err = 4;
+            else total *= ncd[d];
+        }
+        unsigned long long st = 1;
+        for (int d = dim - 1; d >= 0; --d) {
+            g->stride[d] = st;
+            st *= ncd[d];
+        }
+        const unsigned long long mx_id = total - 1ull;
+        g->key_bits = err ? 0 : (mx_id ? 64 - __clzll((long long)mx_id) : 0);
+        g->dim = dim;
+        g->w = ga.w;
+        g->err = err;
+        g->errdim = errdim;
+        g->errq = errq;
+    }
+}
+
+// The host copy of the geometry (first block of the cell-id kernel, so the host reads it while
+// the cell ids are computed): fields, a system-scope fence, then the flag.
+__device__ void publish_geometry(const GeomDev *g, const GeomArgs &ga) {
+    volatile GeomDev *h = ga.host;
+    for (int d = 0; d < SJ_MAX_DIM; ++d) {
+        h->mins[d] = g->mins[d];
+        h->nc[d] = g->nc[d];
+        h->stride[d] = g->stride[d];
+    }
+    h->w = g->w;
+    h->errq = g->errq;
+    h->dim = g->dim;
+    h->key_bits = g->key_bits;
+    h->err = g->err;
+    h->errdim = g->errdim;
+    __threadfence_system();
+    h->flag = ga.epoch;
+}
+
+__global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint64_t n, int dim, BBox *bb,
+                                                        GeomArgs ga) {
     const uint64_t total = n * (uint64_t)dim;  // doubles
     const uint64_t T = (uint64_t)gridDim.x * blockDim.x;
     const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -101,33 +199,44 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
         atomicMax(&bb->mx[threadIdx.x], s_mx[threadIdx.x]);
     }
     if (threadIdx.x == 0 && s_bad) atomicOr(&bb->nonfinite, 1u);
+    // the last block to finish derives the grid geometry from the final box (its first warp)
+    __syncthreads();
+    __shared__ unsigned s_last;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        s_last = atomicAdd(&bb->done, 1u) == gridDim.x - 1u ? 1u : 0u;
+        if (s_last) __threadfence();
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x < 32) derive_geometry(bb, dim, ga);
 }
 
-struct GridGeom {
-    double mins[SJ_MAX_DIM];
-    unsigned long long nc[SJ_MAX_DIM];
-    unsigned long long stride[SJ_MAX_DIM];
-    double w;
-    int dim;
-};
 
 // a3: cell linearisation.  IEEE RN intrinsics so the result does not depend on
 // contraction flags (reading c1): c_d = floor( (x_d - min_d) / w ).
-template <class K>
-__global__ void __launch_bounds__(kThreads) cell_id_kernel(const double *raw, uint64_t n, GridGeom g, K *keys,
-                                                           uint32_t *vals) {
+// The geometry comes from device memory (bbox_kernel's last block); keys are 32-bit when the
+// grid has at most 2^32 cells, else 64-bit (the host picks the buffer once it reads key_bits).
+__global__ void __launch_bounds__(kThreads) cell_id_kernel(const double *raw, uint64_t n,
+                                                           const GeomDev *__restrict__ gp, uint32_t *keys32,
+                                                           unsigned long long *keys64, uint32_t *vals, GeomArgs ga) {
     uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= n) return;
+    if (i == 0 && ga.host) publish_geometry(gp, ga);
+    if (i >= n || gp->err) return;
+    const int dim = gp->dim;
+    const double w = gp->w;
     unsigned long long lid = 0;
 #pragma unroll
     for (int d = 0; d < SJ_MAX_DIM; ++d) {
-        if (d < g.dim) {
-            double q = __ddiv_rn(__dsub_rn(raw[i * g.dim + d], g.mins[d]), g.w);
+        if (d < dim) {
+            double q = __ddiv_rn(__dsub_rn(raw[i * dim + d], gp->mins[d]), w);
             unsigned long long c = __double2ull_rd(q);
-            lid += c * g.stride[d];
+            lid += c * gp->stride[d];
         }
     }
-    keys[i] = (K)lid;
+    if (gp->key_bits <= 32)
+        keys32[i] = (uint32_t)lid;
+    else
+        keys64[i] = lid;
     vals[i] = (uint32_t)i;
 }
 
@@ -781,17 +890,12 @@ struct Temps {
 }  // namespace
 
 template <class K>
-static int sort_points(Temps &tmp, const double *d_raw, uint64_t n, const GridGeom &geo, int bits, cudaStream_t s,
-                       K **keys_sorted, uint32_t **idx_sorted) {
-    K *ka, *kb;
-    uint32_t *va, *vb;
-    SJ_TRY(tmp.alloc(&ka, n));
+static int sort_points(Temps &tmp, K *ka, uint32_t *va, uint64_t n, int bits, cudaStream_t s, K **keys_sorted,
+                       uint32_t **idx_sorted) {
+    K *kb;
+    uint32_t *vb;
     SJ_TRY(tmp.alloc(&kb, n));
-    SJ_TRY(tmp.alloc(&va, n));
     SJ_TRY(tmp.alloc(&vb, n));
-    cell_id_kernel<K><<<grid_for(n), kThreads, 0, s>>>(d_raw, n, geo, ka, va);
-    note_launch();
-    SJ_CUDA_TRY(cudaGetLastError());
     if constexpr (sizeof(K) == 4)
         SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws));
     else
@@ -842,69 +946,90 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // zeroed region holds the counters and every scan's look-back status words.
     {
         const uint64_t tiles = (n + 2047) / 2048 + 1;
-        const size_t bytes = (size_t)n * 84 + (size_t)2 * 256 * 4 * tiles + 64 * 512;
+        const size_t bytes = (size_t)n * 100 + (size_t)2 * 256 * 4 * tiles + 64 * 512;
         const size_t zbytes = (size_t)8 * (12 * tiles + 64) + 48 * 512;
         SJ_TRY(tmp.reserve(bytes, zbytes));
     }
 
-    // ---- a2: bounding box + non-finite check
+    // ---- a2: bounding box + non-finite check; its last block derives the grid geometry (a3)
     BBox *d_bb;
+    GeomDev *d_geo;
     SJ_TRY(tmp.alloc_zero(&d_bb, 1));
+    SJ_TRY(tmp.alloc(&d_geo, 1));
+    GeomArgs ga{};
+    ga.w = ix.w;
+    if (part) {
+        ga.has_origin = 1;
+        for (int d = 0; d < dim; ++d) ga.origin[d] = part->origin[d];
+    }
+    ga.dev = d_geo;
+    // zero-copy: the last block writes the geometry into the pinned mailbox (the device alias of
+    // the same pages), and the host waits on its flag instead of a copy + stream synchronisation
+    volatile GeomDev *h_geo = static_cast<volatile GeomDev *>(mail);
+    // (unified addressing: the device alias of pinned host memory is the host pointer itself --
+    // checked once per process, then used directly)
+    static const int uva = [&] {
+        void *d_alias = nullptr;
+        const bool ok = cudaHostGetDevicePointer(&d_alias, mail, 0) == cudaSuccess && d_alias == mail;
+        if (!ok) cudaGetLastError();
+        return ok ? 1 : 0;
+    }();
+    const bool zero_copy = uva != 0;
+    ga.host = zero_copy ? static_cast<GeomDev *>(mail) : nullptr;
+    ga.epoch = next_epoch();
+    h_geo->flag = 0;
     {
         // 2 * threads must be a multiple of dim (see bbox_kernel): blocks a multiple of dim
         const uint64_t pairs = n * (uint64_t)dim / 2;
         unsigned blocks = (unsigned)std::min<uint64_t>((pairs + kThreads * 8 - 1) / (kThreads * 8), 148ull * 8);
         blocks = std::max(1u, blocks);
         blocks = ((blocks + dim - 1) / dim) * dim;
-        bbox_kernel<<<blocks, kThreads, 0, s>>>(d_raw, n, dim, d_bb);
+        bbox_kernel<<<blocks, kThreads, 0, s>>>(d_raw, n, dim, d_bb, ga);
         note_launch();
     }
     SJ_CUDA_TRY(cudaGetLastError());
-    SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_bb, sizeof(BBox), cudaMemcpyDeviceToHost, s));
-    SJ_CUDA_TRY(cudaStreamSynchronize(s));
-    debug_mark("build: bbox sync");
-    BBox bb;
-    memcpy(&bb, mail, sizeof bb);
-    if (bb.nonfinite) {
+    if (!zero_copy) SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_geo, sizeof(GeomDev), cudaMemcpyDeviceToHost, s));
+    // a3: cell ids, queued at once (they read the device copy of the geometry); 32- or 64-bit keys
+    uint32_t *keys32, *vals0;
+    unsigned long long *keys64;
+    SJ_TRY(tmp.alloc(&keys32, n));
+    SJ_TRY(tmp.alloc(&keys64, n));
+    SJ_TRY(tmp.alloc(&vals0, n));
+    cell_id_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, d_geo, keys32, keys64, vals0, ga);
+    note_launch();
+    SJ_CUDA_TRY(cudaGetLastError());
+    if (zero_copy) {
+        SJ_TRY(wait_flag(&h_geo->flag, ga.epoch, s));
+    } else {
+        SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    }
+    debug_mark("build: geometry");
+    GeomDev g;
+    memcpy(&g, const_cast<const GeomDev *>(h_geo), sizeof g);
+    if (g.err == 1) {
         set_error("sj_create: non-finite coordinate");
         return SJ_EINVAL;
     }
-    GridGeom geo{};
-    geo.dim = dim;
-    geo.w = ix.w;
-    unsigned __int128 total = 1;
-    for (int d = 0; d < dim; ++d) {
-        double mn = from_ordered_key(~bb.mn_c[d]);
-        double mx = from_ordered_key(bb.mx[d]);
-        if (part) {  // partition of a larger grid: its origin, so the cells of all partitions align
-            if (!(part->origin[d] <= mn) || !std::isfinite(part->origin[d])) {
-                set_error("sj_create_part: a coordinate in dimension %d lies below the grid origin", d);
-                return SJ_EINVAL;
-            }
-            mn = part->origin[d];
-        }
-        ix.mins[d] = mn;
-        geo.mins[d] = mn;
-        // nc_d = max c_d + 1; c_d is monotone in x_d so max c_d = c_d(max x_d)
-        double q = (mx - mn) / ix.w;
-        if (!(q < 0x1p30)) {
-            set_error("sj_create: grid too large in dimension %d (%.3g cells >= 2^30)", d, q);
-            return SJ_EGRID;
-        }
-        ix.nc[d] = (uint64_t)floor(q) + 1;
-        total *= ix.nc[d];
-        if (total >= ((unsigned __int128)1 << 64)) {
-            set_error("sj_create: grid too large (prod nc_d >= 2^64)");
-            return SJ_EGRID;
-        }
+    if (g.err == 2) {
+        set_error("sj_create_part: a coordinate in dimension %d lies below the grid origin", g.errdim);
+        return SJ_EINVAL;
     }
-    for (int d = dim - 1; d >= 0; --d) ix.stride[d] = (d == dim - 1) ? 1 : ix.stride[d + 1] * ix.nc[d + 1];
-    for (int d = 0; d < dim; ++d) {
-        geo.nc[d] = ix.nc[d];
-        geo.stride[d] = ix.stride[d];
+    if (g.err == 3) {
+        set_error("sj_create: grid too large in dimension %d (%.3g cells >= 2^30)", g.errdim, g.errq);
+        return SJ_EGRID;
     }
-    const unsigned long long ncells_total = (unsigned long long)total;
-    ix.key_bits = bits_for(ncells_total - 1);
+    if (g.err) {
+        set_error("sj_create: grid too large (prod nc_d >= 2^64)");
+        return SJ_EGRID;
+    }
+    unsigned long long ncells_total = 1;
+    for (int d = 0; d < dim; ++d) {
+        ix.mins[d] = g.mins[d];
+        ix.nc[d] = g.nc[d];
+        ix.stride[d] = g.stride[d];
+        ncells_total *= g.nc[d];
+    }
+    ix.key_bits = g.key_bits;
 
     // ---- a3 + a4 + a5: cell ids, point -> cell sort, compaction of the non-empty cells
     uint32_t *idx_sorted = nullptr;
@@ -921,11 +1046,12 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
     if (ix.key_bits <= 32) {
         uint32_t *ks;
-        SJ_TRY(sort_points<uint32_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
+        SJ_TRY(sort_points<uint32_t>(tmp, keys32, vals0, n, ix.key_bits, s, &ks, &idx_sorted));
         SJ_TRY(rle<uint32_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
     } else {
         uint64_t *ks;
-        SJ_TRY(sort_points<uint64_t>(tmp, d_raw, n, geo, ix.key_bits, s, &ks, &idx_sorted));
+        SJ_TRY(sort_points<uint64_t>(tmp, reinterpret_cast<uint64_t *>(keys64), vals0, n, ix.key_bits, s, &ks,
+                                     &idx_sorted));
         SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
     }
     // the gather of the points into cell order needs only the point sort: side stream

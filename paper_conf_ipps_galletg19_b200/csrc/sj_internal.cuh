@@ -94,6 +94,12 @@ constexpr size_t kMailBytes = 4096;
 void *pinned_acquire();
 void pinned_release(void *p);
 
+// Zero-copy host waits: a kernel writes its result into pinned host memory, then `epoch` into
+// *flag (after a system-scope fence); the host spins on the flag, polling the stream for errors
+// (and for a stream that drained without the flag: an error).  next_epoch() never returns 0.
+unsigned next_epoch();
+int wait_flag(volatile unsigned *flag, unsigned epoch, cudaStream_t s);
+
 // --------------------------------------------------------------------------- primitives
 // Exclusive scan of u32 (out may alias in).  total (device, optional) receives the sum.
 int scan_exclusive_u32(const uint32_t *in, uint32_t *out, uint64_t n, uint32_t *d_total, cudaStream_t s,

@@ -99,6 +99,39 @@ void pinned_release(void *p) {
     g_pin_free.push_back(p);
 }
 
+// ------------------------------------------------------------------------- zero-copy waits
+static std::atomic<unsigned> g_epoch{0};
+
+unsigned next_epoch() {
+    unsigned e = g_epoch.fetch_add(1, std::memory_order_relaxed) + 1;
+    if (e == 0) e = g_epoch.fetch_add(1, std::memory_order_relaxed) + 1;
+    return e;
+}
+
+int wait_flag(volatile unsigned *flag, unsigned epoch, cudaStream_t s) {
+    for (unsigned long long spin = 0;; ++spin) {
+        if (*flag == epoch) {
+            std::atomic_thread_fence(std::memory_order_acquire);
+            return SJ_OK;
+        }
+        if ((spin & 255) == 255) {
+            const cudaError_t e = cudaStreamQuery(s);
+            if (e == cudaSuccess) {  // the stream drained: the flag must be there
+                if (*flag == epoch) {
+                    std::atomic_thread_fence(std::memory_order_acquire);
+                    return SJ_OK;
+                }
+                set_error("zero-copy wait: the stream completed without the result flag");
+                return SJ_ECUDA;
+            }
+            if (e != cudaErrorNotReady) {
+                set_error("zero-copy wait: %s", cudaGetErrorString(e));
+                return SJ_ECUDA;
+            }
+        }
+    }
+}
+
 // ------------------------------------------------------------------------- small kernels
 __global__ void set_u64_kernel(unsigned long long *p, unsigned long long v) { *p = v; }
 
