@@ -29,6 +29,10 @@
 //     points shares that cell's forward runs; the warp stages them 32 candidates at a
 //     time in shared memory and every query of the chunk is evaluated against each
 //     tile (loads per distance calculation / (chunk size / k)).
+#include <map>
+#include <mutex>
+#include <utility>
+
 #include "sj_internal.cuh"
 
 namespace sj {
@@ -1157,7 +1161,10 @@ typedef void (*join_fn)(const JoinArgs);
 struct KernelInfo {
     join_fn f = nullptr;
     size_t smem = 0;
+    int occ = 0;  // resident CTAs per SM
 };
+std::mutex g_prep_mu;
+std::map<std::pair<int, const void *>, int> g_prep;  // (device, kernel) -> occupancy, attribute set
 
 template <int DIM, int K, int MODE, bool GCG>
 KernelInfo info() {
@@ -1229,7 +1236,25 @@ int prepare(int dim, int k, int mode, bool gcg, KernelInfo *out) {
                   gcg ? " for the GCG pattern (k in {1, 8, 32})" : " (CSR modes need the GCG pattern)");
         return SJ_EINVAL;
     }
+    // the shared-memory attribute and the occupancy are per (device, kernel): set / queried once
+    // (each costs the host microseconds, on the path from sj_create to the join's launch)
+    int dev = 0;
+    SJ_CUDA_TRY(cudaGetDevice(&dev));
+    {
+        std::lock_guard<std::mutex> lk(g_prep_mu);
+        auto it = g_prep.find(std::make_pair(dev, (const void *)ki.f));
+        if (it != g_prep.end()) {
+            ki.occ = it->second;
+            *out = ki;
+            return SJ_OK;
+        }
+    }
     SJ_CUDA_TRY(cudaFuncSetAttribute(ki.f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ki.smem));
+    SJ_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ki.occ, ki.f, kJoinThreads, ki.smem));
+    {
+        std::lock_guard<std::mutex> lk(g_prep_mu);
+        g_prep[std::make_pair(dev, (const void *)ki.f)] = ki.occ;
+    }
     *out = ki;
     return SJ_OK;
 }
@@ -1239,7 +1264,7 @@ int prepare(int dim, int k, int mode, bool gcg, KernelInfo *out) {
 int join_occupancy(int dim, int k, int mode, bool gcg, int *blocks_per_sm) {
     KernelInfo ki;
     SJ_TRY(prepare(dim, k, mode, gcg, &ki));
-    SJ_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, ki.f, kJoinThreads, ki.smem));
+    *blocks_per_sm = ki.occ;
     return SJ_OK;
 }
 
