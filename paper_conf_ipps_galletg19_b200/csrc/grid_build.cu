@@ -345,7 +345,14 @@ struct BuildTotals {
     unsigned long long E;
     unsigned long long dist_calcs;
     unsigned int max_w;
-    unsigned int pad;
+    unsigned int done;  // blocks of the counting pass finished (the last one publishes)
+};
+
+// Zero-copy publication of the counting pass (the host's second wait): {M, E, D_alg, max W,
+// mixed cells} into pinned memory, then the epoch into word 5.
+struct TotalsPub {
+    unsigned long long *host;  // pinned host words [6], or nullptr (copy + synchronisation)
+    unsigned epoch;
 };
 
 // a6 + a7.  LID-UNICOMP (Alg. 3) visits the neighbour cells with a higher linear
@@ -464,7 +471,7 @@ template <bool FILL, int LPC>
 __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
                                                         const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *rcnt,
                                                         uint32_t *wload, const uint32_t *rbegin, uint2 *runs,
-                                                        BuildTotals *tot) {
+                                                        BuildTotals *tot, TotalsPub pub) {
     // grid-stride over the cells (M is only known on the device): a bounded grid, so the block
     // reduction below runs once per resident block, not once per n-sized block
     const uint64_t M = *d_M;
@@ -556,6 +563,21 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
             if (calcs) atomicAdd(&tot->dist_calcs, calcs);
             if (nruns) atomicAdd(&tot->E, nruns);
             if (w) atomicMax(&tot->max_w, w);
+            if (pub.host) {  // the last block publishes the totals
+                __threadfence();
+                if (atomicAdd(&tot->done, 1u) == gridDim.x - 1u) {
+                    __threadfence();
+                    const volatile BuildTotals *vt = tot;
+                    volatile unsigned long long *hp = pub.host;
+                    hp[0] = M;
+                    hp[1] = vt->E;
+                    hp[2] = vt->dist_calcs;
+                    hp[3] = vt->max_w;
+                    hp[4] = g.mixed ? *(const volatile unsigned *)g.mixed : 0u;
+                    __threadfence_system();
+                    *reinterpret_cast<volatile unsigned *>(pub.host + 5) = pub.epoch;
+                }
+            }
         }
     }
 }
@@ -1156,30 +1178,47 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     auto runs_grid = [&](uint64_t cells, int lpc) {
         return std::min<unsigned>(grid_for(cells * (uint64_t)lpc), (unsigned)nsm * 8u);
     };
+    volatile unsigned long long *h_pub = reinterpret_cast<volatile unsigned long long *>((char *)mail + 768);
+    TotalsPub pub{};
+    if (zero_copy) {
+        pub.host = reinterpret_cast<unsigned long long *>((char *)mail + 768);
+        pub.epoch = next_epoch();
+        h_pub[5] = 0;
+    }
     if (wide)
         runs_kernel<false, 32><<<runs_grid(n, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                    nullptr, slots ? ix.runs : nullptr, d_tot);
+                                                                    nullptr, slots ? ix.runs : nullptr, d_tot, pub);
     else
         runs_kernel<false, 1><<<runs_grid(n, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                  nullptr, slots ? ix.runs : nullptr, d_tot);
+                                                                  nullptr, slots ? ix.runs : nullptr, d_tot, pub);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin = nullptr;
     if (!slots) SJ_TRY(tmp.alloc(&rbegin, n + 1));
-    // host round trip 2: M, plus the workload totals (max W sizes the SortByWL keys, D_alg)
-    SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_M, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 64, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
-    if (d_mixed) SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 128, d_mixed, sizeof(unsigned int), cudaMemcpyDeviceToHost, s));
-    SJ_CUDA_TRY(cudaStreamSynchronize(s));
-    debug_mark("build: sort+rle+runcount sync");
+    // host wait 2: M, plus the workload totals (max W sizes the SortByWL keys, D_alg)
     uint64_t M;
-    memcpy(&M, mail, sizeof M);
+    BuildTotals bt{};
+    unsigned int mixed = 0;
+    if (zero_copy) {  // published by the counting pass's last block
+        SJ_TRY(wait_flag(reinterpret_cast<volatile unsigned *>(h_pub + 5), pub.epoch, s));
+        M = h_pub[0];
+        bt.E = h_pub[1];
+        bt.dist_calcs = h_pub[2];
+        bt.max_w = (unsigned)h_pub[3];
+        mixed = (unsigned)h_pub[4];
+    } else {
+        SJ_CUDA_TRY(cudaMemcpyAsync(mail, d_M, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 64, d_tot, sizeof(BuildTotals), cudaMemcpyDeviceToHost, s));
+        if (d_mixed)
+            SJ_CUDA_TRY(cudaMemcpyAsync((char *)mail + 128, d_mixed, sizeof(unsigned int), cudaMemcpyDeviceToHost, s));
+        SJ_CUDA_TRY(cudaStreamSynchronize(s));
+        memcpy(&M, mail, sizeof M);
+        memcpy(&bt, (char *)mail + 64, sizeof bt);
+        if (d_mixed) memcpy(&mixed, (char *)mail + 128, sizeof mixed);
+    }
+    debug_mark("build: sort+rle+runcount wait");
     ix.n_cells = M;
-    BuildTotals bt;
-    memcpy(&bt, (char *)mail + 64, sizeof bt);
     if (d_mixed) {
-        unsigned int mixed = 0;
-        memcpy(&mixed, (char *)mail + 128, sizeof mixed);
         if (mixed) {
             set_error("sj_create_part: a grid cell holds both query and halo points (partition the data by "
                       "whole cell columns)");
@@ -1219,10 +1258,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         // (the counting pass wrote them)
     } else if (wide)
         runs_kernel<true, 32><<<runs_grid(M, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
-                                                                    rbegin, ix.runs, nullptr);
+                                                                    rbegin, ix.runs, nullptr, TotalsPub{});
     else
         runs_kernel<true, 1><<<runs_grid(M, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
-                                                              rbegin, ix.runs, nullptr);
+                                                              rbegin, ix.runs, nullptr, TotalsPub{});
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
