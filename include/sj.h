@@ -132,8 +132,12 @@ typedef struct sj_stats {
  *   eps    : finite, > 0.
  * Runs steps a1..a8 of DESIGN.md §1 (upload+validate, bounding box, cell
  * linearisation, radix sort, compaction, forward neighbours, workload, SortByWL).
+ * Returns once the caller's points are no longer read (they may be freed or overwritten);
+ * the build's last kernels may still be running on the handle's stream -- every other call
+ * on the handle is ordered after them (set SJ_SYNC_BUILD=1 for a fully synchronous build).
  * Returns NULL on error (see sj_last_error): NaN/Inf coordinate or bad argument
- * (SJ_EINVAL), grid overflow (SJ_EGRID), allocation (SJ_ENOMEM), CUDA (SJ_ECUDA). */
+ * (SJ_EINVAL), grid overflow (SJ_EGRID), allocation (SJ_ENOMEM), CUDA (SJ_ECUDA); an
+ * asynchronous CUDA error of the build's last kernels surfaces at the next call instead. */
 sj_handle *sj_create(const double *points, uint64_t n, int dim, double eps);
 
 /* sj_create with an explicit cell pattern (enum sj_pattern) and queue order (enum sj_order),
@@ -215,7 +219,7 @@ int sj_get_stats(const sj_handle *h, sj_stats *s);
 
 /* Serialise the built index (header + device arrays) into one contiguous blob
  * for an NCCL broadcast.  dst: device or host pointer of cap bytes, or NULL to
- * only query the size in *bytes. */
+ * only query the size in *bytes.  Format "SJIDX004" (this library version only). */
 int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes);
 
 /* Create a handle from a blob produced by sj_export_index (device or host
