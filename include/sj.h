@@ -122,6 +122,8 @@ typedef struct sj_stats {
     uint32_t pattern;         /* enum sj_pattern of the index                        */
     uint32_t order;           /* enum sj_order of the index                          */
     uint32_t est_fused;       /* 1 if the estimator (a9) ran fused into the in-place join */
+    uint32_t lookup_hash;     /* a6's lid -> cell lookup: 0 dense table over prod nc_d cells,
+                                 1 open-addressing hash of the non-empty cells (sparse grids) */
 } sj_stats;
 
 /* Build the eps-grid index of `n` points of dimension `dim` (row-major AoS,

@@ -62,6 +62,12 @@ def _load():
     lib.orc_grid_rows.argtypes = [_dblp, c.c_uint64, c.c_int, c.c_double, _u32p, c.c_uint64, _u64p, _u32p, c.c_uint64]
     lib.orc_grid_pairs.argtypes = [_dblp, c.c_uint64, c.c_int, c.c_double, _u32p, c.c_uint64, _u64p]
     lib.orc_grid_cells.argtypes = [_dblp, c.c_uint64, c.c_int, c.c_double, _i64p, _u64p, _u32p, _u64p]
+    lib.orc_grid_new.argtypes = [_dblp, c.c_uint64, c.c_int, c.c_double, c.POINTER(c.c_int)]
+    lib.orc_grid_new.restype = c.c_void_p
+    lib.orc_grid_delete.argtypes = [c.c_void_p]
+    lib.orc_grid_delete.restype = None
+    lib.orc_grid_rows_range.argtypes = [c.c_void_p, c.c_uint64, c.c_uint64, _u64p, _u32p, c.c_uint64]
+    lib.orc_grid_rows_range.restype = c.c_int
     lib.orc_hash_pairs.argtypes = [_u32p, c.c_uint64]
     lib.orc_hash_pairs.restype = c.c_uint64
     lib.orc_num_threads.restype = c.c_int
@@ -171,6 +177,53 @@ def grid_pairs(points, eps: float) -> np.ndarray:
 def grid_rows(points, eps: float, rows):
     """O2 neighbour rows of the given query ids: (offsets, cols), rows ascending."""
     return _rows("orc_grid_rows", points, eps, rows)
+
+
+class Grid:
+    """A persistent O2 grid (built once) whose rows are read in blocks of query ids:
+    ``rows_range(lo, hi)`` -> (offsets[hi-lo+1], cols), each row ascending, i.e. the
+    canonical (i, j) order of the queries lo .. hi-1.  Context manager."""
+
+    def __init__(self, points, eps: float):
+        self.p = _pts(points)  # kept alive: the C grid points into it
+        lib = _load()
+        rc = ctypes.c_int(0)
+        self.g = lib.orc_grid_new(_ptr(self.p, _dblp), self.p.shape[0], self.p.shape[1], float(eps),
+                                  ctypes.byref(rc))
+        if not self.g:
+            raise OracleError(f"orc_grid_new failed with code {rc.value}")
+
+    def rows_range(self, lo: int, hi: int):
+        lib = _load()
+        off = np.zeros(hi - lo + 1, dtype=np.uint64)
+        _check(lib.orc_grid_rows_range(self.g, int(lo), int(hi), _ptr(off, _u64p), None, 0), "orc_grid_rows_range")
+        cols = np.empty(max(int(off[-1]), 1), dtype=np.uint32)
+        _check(lib.orc_grid_rows_range(self.g, int(lo), int(hi), _ptr(off, _u64p), _ptr(cols, _u32p), cols.shape[0]),
+               "orc_grid_rows_range")
+        return off, cols[: int(off[-1])]
+
+    def keys_range(self, lo: int, hi: int) -> np.ndarray:
+        """The pairs of queries lo .. hi-1 as canonical uint64 keys i << 32 | j (ascending)."""
+        off, cols = self.rows_range(lo, hi)
+        i = np.repeat(np.arange(lo, hi, dtype=np.uint64), np.diff(off).astype(np.int64))
+        return (i << np.uint64(32)) | cols.astype(np.uint64)
+
+    def close(self):
+        if getattr(self, "g", None):
+            _load().orc_grid_delete(self.g)
+            self.g = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def grid_cells(points, eps: float):

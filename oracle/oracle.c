@@ -438,6 +438,56 @@ int orc_grid_cells(const double *pts, uint64_t n, int dim, double eps,
     return ORC_OK;
 }
 
+/* A persistent O2 grid (the same grid_build / grid_query as above, built once) for the
+ * full-size element-wise comparisons, which walk the queries in blocks of ids and would
+ * otherwise rebuild the grid per block.  The caller keeps `pts` alive until
+ * orc_grid_delete.  No new arithmetic: only the lifetime of the grid differs. */
+void *orc_grid_new(const double *pts, uint64_t n, int dim, double eps, int *rc_out) {
+    int rc = check_args(pts, n, dim, eps);
+    grid_t *g = NULL;
+    if (!rc) {
+        g = (grid_t *)malloc(sizeof(grid_t));
+        if (!g) rc = ORC_ENOMEM;
+        else if ((rc = grid_build(g, pts, n, dim, eps)) != ORC_OK) { free(g); g = NULL; }
+    }
+    if (rc_out) *rc_out = rc;
+    return g;
+}
+
+void orc_grid_delete(void *gp) {
+    if (!gp) return;
+    grid_free((grid_t *)gp);
+    free(gp);
+}
+
+/* Rows of the queries lo .. hi-1 (each row ascending), offsets[hi-lo+1]; cols NULL for a
+ * sizing call.  Rows in query order, so (i, cols) is already canonical (i, j) order. */
+int orc_grid_rows_range(void *gp, uint64_t lo, uint64_t hi, uint64_t *offsets, uint32_t *cols, uint64_t cap) {
+    const grid_t *g = (const grid_t *)gp;
+    if (!g || !offsets || lo > hi || hi > g->n) return ORC_EINVAL;
+    const uint64_t nr = hi - lo;
+    uint64_t *cnt = (uint64_t *)calloc(nr + 1, sizeof(uint64_t));
+    if (!cnt) return ORC_ENOMEM;
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t r = 0; r < (int64_t)nr; ++r) {
+        uint64_t e;
+        cnt[r] = grid_query(g, lo + (uint64_t)r, NULL, &e);
+    }
+    offsets[0] = 0;
+    for (uint64_t r = 0; r < nr; ++r) offsets[r + 1] = offsets[r] + cnt[r];
+    free(cnt);
+    if (!cols) return ORC_OK;
+    if (offsets[nr] > cap) return ORC_ECAP;
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t r = 0; r < (int64_t)nr; ++r) {
+        uint64_t e;
+        uint32_t *row = cols + offsets[r];
+        uint64_t k = grid_query(g, lo + (uint64_t)r, row, &e);
+        qsort(row, k, sizeof(uint32_t), cmp_u32);
+    }
+    return ORC_OK;
+}
+
 /* The multiset hash of an explicit pair list (so tests hash GPU output with the same
  * function the oracle uses, without re-implementing it). */
 uint64_t orc_hash_pairs(const uint32_t *pairs, uint64_t count) {

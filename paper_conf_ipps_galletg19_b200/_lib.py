@@ -38,7 +38,7 @@ class SJStats(ctypes.Structure):
         ("ms_join_sum", ctypes.c_double), ("ms_transfer", ctypes.c_double), ("ms_total", ctypes.c_double),
         ("fast_path", ctypes.c_uint32), ("nc", ctypes.c_uint32 * 8), ("n_chunks", ctypes.c_uint64),
         ("tiled_min", ctypes.c_uint32), ("pattern", ctypes.c_uint32), ("order", ctypes.c_uint32),
-        ("est_fused", ctypes.c_uint32),
+        ("est_fused", ctypes.c_uint32), ("lookup_hash", ctypes.c_uint32),
     ]
 
     def as_dict(self) -> dict:

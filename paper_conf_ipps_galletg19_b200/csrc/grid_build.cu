@@ -1066,6 +1066,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // lid -> rank lookup: a dense table when prod(nc) is small, else a hash table
     Lookup L{};
     const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
+    ix.lookup_hash = dense ? 0 : 1;
     if (ix.key_bits <= 32) {
         uint32_t *ks;
         SJ_TRY(sort_points<uint32_t>(tmp, keys32, vals0, n, ix.key_bits, s, &ks, &idx_sorted));

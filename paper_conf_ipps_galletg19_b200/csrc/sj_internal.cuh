@@ -139,6 +139,7 @@ struct Index {
     uint64_t n_runs = 0;      // E, forward runs over all cells
     uint64_t dist_calcs = 0;  // D_alg
     uint32_t max_w = 0;
+    int lookup_hash = 0;      // a6's lid -> cell lookup: 0 dense table, 1 open-addressing hash
 
     double *pts = nullptr;      // [n * pad]  points in lid (spatial) order, padded AoS
     uint32_t *orig = nullptr;   // [n]        lid position -> input id

@@ -425,6 +425,7 @@ void fill_static_stats(sj_handle *h) {
     st.tiled_min = kBigCell;
     st.pattern = (uint32_t)h->ix.pattern;
     st.order = (uint32_t)h->ix.order;
+    st.lookup_hash = (uint32_t)h->ix.lookup_hash;
 }
 
 // The build's tail (sj_create returns without a final round trip): {n_chunks, E} from the
@@ -1418,7 +1419,7 @@ struct BlobHeader {
     uint64_t nc[SJ_MAX_DIM];
     uint64_t stride[SJ_MAX_DIM];
     uint64_t n_cells, n_runs, dist_calcs, n_chunks;
-    uint32_t max_w, reserved2;
+    uint32_t max_w, lookup_hash;
     uint64_t off[7], bytes[7];  // pts, orig, qmap, cellq, runs, cell_lid, chunks
     uint64_t total;
     uint64_t n_query;  // queries of a partitioned index (D' positions [0, n_query))
@@ -1449,6 +1450,7 @@ BlobHeader make_header(const Index &ix) {
     b.n_chunks = ix.n_chunks;
     b.dist_calcs = ix.dist_calcs;
     b.max_w = ix.max_w;
+    b.lookup_hash = (uint32_t)ix.lookup_hash;
     const uint64_t sz[7] = {ix.n * ix.pad * sizeof(double), ix.n * sizeof(uint32_t), ix.n * sizeof(uint2),
                             ix.n_cells * sizeof(uint4), runs_entries(ix) * sizeof(uint2), ix.n_cells * sizeof(uint64_t),
                             (ix.n_chunks + 1) * sizeof(uint32_t)};
@@ -1531,6 +1533,7 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
     ix.n_query = b.n_query ? b.n_query : b.n;
     ix.dist_calcs = b.dist_calcs;
     ix.max_w = b.max_w;
+    ix.lookup_hash = (int)b.lookup_hash;
     cudaStream_t s = h->s_main;
     void **dst[7] = {(void **)&ix.pts,  (void **)&ix.orig,     (void **)&ix.qmap,  (void **)&ix.cellq,
                      (void **)&ix.runs, (void **)&ix.cell_lid, (void **)&ix.chunks};

@@ -258,3 +258,79 @@ def test_workload_generators_are_deterministic():
     assert math.isclose(workloads.get_config("c1").eps, 0.0319154, rel_tol=1e-5)
     assert math.isclose(workloads.get_config("c3").eps, 9.84745e-4, rel_tol=1e-5)
     assert math.isclose(workloads.get_config("c4").eps, 0.120727, rel_tol=1e-5)
+
+
+# ----------------------------------------------------------------- the distance-calculation count
+
+def _numpy_cells(p, eps):
+    """Cell tuples of reading c5/c6 computed with numpy (independent of oracle.c):
+    c_d = floor(fl(fl(x_d - min_d) / w)), w = eps (1 + 2^-20)."""
+    w = eps * (1.0 + 2.0 ** -20)
+    return np.floor((p - p.min(axis=0)) / w).astype(np.int64)
+
+
+def _numpy_full_scan_calcs(p, eps):
+    """Distance calculations of a full 3^n neighbourhood scan that skips j == i, from the cell
+    multiplicities alone: sum_A m_A * (sum_{B in N(A)} m_B) - N, N(A) the 3^n cells around A
+    (A included)."""
+    import itertools
+
+    cells = _numpy_cells(p, eps)
+    uniq, m = np.unique(cells, axis=0, return_counts=True)
+    mult = {tuple(c): int(k) for c, k in zip(uniq.tolist(), m.tolist())}
+    offs = list(itertools.product((-1, 0, 1), repeat=p.shape[1]))
+    tot = 0
+    for c, k in mult.items():
+        tot += k * sum(mult.get(tuple(a + o for a, o in zip(c, off)), 0) for off in offs)
+    return tot - p.shape[0]
+
+
+@pytest.mark.parametrize("dim,g", [(1, 40), (2, 12), (3, 7), (4, 5), (6, 3)])
+def test_grid_calcs_lattice_closed_form(dim, g):
+    # unit lattice, eps = 1 - 2^-19: w = eps (1 + 2^-20) < 1, so every point has a cell of its
+    # own at its lattice coordinate, and a full 3^n scan evaluates prod_d (neighbours in d) - 1
+    # candidates per point: sum over the lattice = prod_d sum_x n_d(x) - g^n = (3g - 2)^n - g^n
+    # (n_d = 2 at the two faces, 3 inside).  No pair is within eps (spacing 1).
+    p = workloads.lattice(g, dim)
+    res = oracle.grid_count(p, 1.0 - 2.0 ** -19)
+    assert res["ncells"] == g ** dim
+    assert res["count"] == 0
+    assert res["calcs"] == (3 * g - 2) ** dim - g ** dim
+
+
+@pytest.mark.parametrize("dist,dim,n,k", [("uniform", 2, 3000, 30), ("exponential", 3, 3000, 40),
+                                          ("uniform", 6, 1500, 20), ("uniform", 1, 2000, 10)])
+def test_grid_calcs_equal_cell_multiplicity_count(dist, dim, n, k):
+    # the oracle counts its calculations query by query; the same number follows from the cell
+    # multiplicities (numpy cells, no oracle code): a dropped / doubled neighbour offset or a
+    # counted self-comparison fails here
+    p = workloads.gen_points(dist, n, dim, 500 + dim)
+    eps = workloads.eps_for_k(dist, n, dim, k)
+    res = oracle.grid_count(p, eps, with_hash=False)
+    assert res["calcs"] == _numpy_full_scan_calcs(p, eps)
+    assert res["ncells"] == np.unique(_numpy_cells(p, eps), axis=0).shape[0]
+
+
+def test_grid_calcs_sw_shaped_and_duplicates():
+    p = workloads.sw_shaped(4000, 21)
+    assert oracle.grid_count(p, 1.5, with_hash=False)["calcs"] == _numpy_full_scan_calcs(p, 1.5)
+    d = workloads.duplicates(300, 3)
+    assert oracle.grid_count(d, 1e-6, with_hash=False)["calcs"] == 300 * 299
+
+
+# ----------------------------------------------------------------- persistent grid (block rows)
+
+@pytest.mark.parametrize("dist,dim", [("uniform", 2), ("exponential", 3), ("uniform", 6)])
+def test_grid_rows_range_equals_rows_and_bruteforce(dist, dim):
+    n = 2500 if dim <= 3 else 1200
+    p = workloads.gen_points(dist, n, dim, 600 + dim)
+    eps = workloads.eps_for_k(dist, n, dim, 25)
+    want = oracle.bf_pairs(p, eps)
+    keys_want = (want[:, 0].astype(np.uint64) << np.uint64(32)) | want[:, 1].astype(np.uint64)
+    with oracle.Grid(p, eps) as g:
+        parts = [g.keys_range(lo, min(lo + 333, n)) for lo in range(0, n, 333)]
+        off, cols = g.rows_range(17, 29)
+    np.testing.assert_array_equal(np.concatenate(parts), keys_want)
+    off2, cols2 = oracle.grid_rows(p, eps, np.arange(17, 29, dtype=np.uint32))
+    np.testing.assert_array_equal(off, off2)
+    np.testing.assert_array_equal(cols, cols2)

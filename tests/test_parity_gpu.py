@@ -2,9 +2,8 @@
 
 Bar (BASELINE.json north_star): the GPU pair SET is bit-exact against
 the oracle after canonical (i, j) sorting -- integer/index output, both sides with
-FP64 RN dimension-order accumulation, no FMA, s <= fl(eps^2).  Mid sizes are compared
-element by element; full sizes by count + order-independent multiset hash against
-O2, sampled rows against O1 brute force, and the distance-calculation accounting.
+FP64 RN dimension-order accumulation, no FMA, s <= fl(eps^2).  Every size is compared
+element by element (full BASELINE sizes in tests/test_fullsize_gpu.py).
 """
 import math
 import os
@@ -268,36 +267,4 @@ def test_index_blob_roundtrip():
     with sj.Handle.from_index(host_blob, nbytes) as h3:
         assert h3.count() == want.shape[0]
 
-
-# ------------------------------------------------------------------ full BASELINE sizes
-
-FULL = ["c1", "c2k16", "c2k64", "c2k256", "c3k64", "c4k32", "c5"]
-
-
-@pytest.mark.parametrize("name", FULL)
-def test_full_size_count_hash_rows(name):
-    """Full configuration in the bench's launch configuration (k=8, fast path, device output):
-    count + multiset hash vs O2, distance-calc accounting vs O2, 400 sampled rows vs O1."""
-    cfg = workloads.get_config(name)
-    pts = cfg.points()
-    p = torch.from_numpy(pts).to(DEV)
-    with sj.Handle(p, cfg.eps, k=cfg.k) as h:
-        got = sj.self_join_pairs(h, DEV)
-        st = h.stats()
-    a = got.cpu().numpy().view(np.uint32).reshape(-1, 2)
-    del got
-    g = oracle.grid_count(pts, cfg.eps, with_hash=True)
-    assert a.shape[0] == g["count"]
-    assert oracle.hash_pairs(a) == g["hash"]
-    assert st["dist_calcs"] * 2 == g["calcs"]
-    assert st["n_cells"] == g["ncells"]
-    assert not np.any(a[:, 0] == a[:, 1])
-    rng = np.random.default_rng(123)
-    rows = np.unique(rng.integers(0, cfg.n, size=400)).astype(np.uint32)
-    off, cols = oracle.bf_rows(pts, cfg.eps, rows)
-    order = np.argsort(a[:, 0], kind="stable")
-    first = a[order, 0]
-    for r, i in enumerate(rows):
-        lo, hi = np.searchsorted(first, i, "left"), np.searchsorted(first, i, "right")
-        mine = np.sort(a[order[lo:hi], 1])
-        np.testing.assert_array_equal(mine, cols[off[r]:off[r + 1]])
+# (full BASELINE sizes: tests/test_fullsize_gpu.py, element by element)

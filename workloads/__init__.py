@@ -27,7 +27,7 @@ import numpy as np
 
 __all__ = [
     "Config", "CONFIGS", "get_config", "gen_points", "eps_for_k",
-    "uniform", "exponential", "sw_shaped", "lattice", "duplicates",
+    "uniform", "exponential", "sw_shaped", "lattice", "duplicates", "clusters",
 ]
 
 
@@ -84,6 +84,16 @@ def lattice(g: int, dim: int, spacing: float = 1.0) -> np.ndarray:
 def duplicates(n: int, dim: int, value: float = 0.25) -> np.ndarray:
     """n copies of the same point (every i != j pair is at distance 0)."""
     return np.full((n, dim), value, dtype=np.float64)
+
+
+def clusters(centres, per_cluster: int, sigma: float, seed: int) -> np.ndarray:
+    """Gaussian clusters (isotropic sigma) of ``per_cluster`` points around each row of
+    ``centres`` (k, dim), shuffled: sparse grids whose non-empty cells are few and far apart
+    (the hashed lid -> cell lookup, 64-bit cell keys)."""
+    rng = np.random.default_rng(seed)
+    c = np.asarray(centres, dtype=np.float64)
+    pts = np.repeat(c, per_cluster, axis=0) + sigma * rng.standard_normal((c.shape[0] * per_cluster, c.shape[1]))
+    return np.ascontiguousarray(pts[rng.permutation(pts.shape[0])])
 
 
 def eps_for_k(dist: str, n: int, dim: int, k: float, lam: float = 40.0) -> float:
