@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--k", type=int, default=None)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--batched-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-stride", type=int, default=0, help="oracle sample: every s-th query (0 = auto)")
     ap.add_argument("--json-out", default=None)
@@ -125,13 +126,64 @@ def load_peaks():
 
 
 def load_profile_facts(cfg_name: str):
-    """ncu-derived facts committed under profiles/ (traffic per launch, warp execution efficiency)."""
+    """ncu facts of THIS configuration (DRAM traffic per launch, warp execution efficiency),
+    committed under profiles/ by tools/r02_facts.py from an `ncu --set full` capture of the same
+    launch in a separate process (bench numbers are never taken under a profiler).  Each entry
+    names its source file and capture date; a configuration without its own capture gets none
+    (no other configuration's numbers are reused)."""
     p = os.path.join(ROOT, "profiles", "ncu_facts.json")
     try:
         with open(p) as f:
-            return json.load(f).get(cfg_name, {})
+            e = json.load(f).get(cfg_name, {})
     except (OSError, ValueError):
         return {}
+    return e if e.get("config") == cfg_name else {}
+
+
+def build_algorithmic_bytes(st: dict, dim: int, pad: int) -> int:
+    """Compulsory HBM bytes of the build (a2-a8): the raw points read once and the
+    index written once -- points in cell order (8*pad), input ids (4) and D' (8) per point, the
+    cell record (16) and lid (8) per cell, 8 B per forward run slot, 4 B per WorkQueue chunk.
+    The sort passes and temporaries are the build's own overhead, not counted."""
+    n, m, e, c = st["n"], st["n_cells"], st["fwd_runs"], st["n_chunks"]
+    return n * 8 * dim + n * (8 * pad + 12) + m * 24 + 8 * e + 4 * (c + 1)
+
+
+def pcie_rates(dev, nbytes: int = 1 << 30):
+    """Measured pinned host<->device copy rates (bytes/s), best of 3 (the e2e denominator)."""
+    import torch
+
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    out = {}
+    for name, dst, src in (("h2d", d, h), ("d2h", h, d)):
+        best = float("inf")
+        for _ in range(3):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            a.record()
+            dst.copy_(src, non_blocking=True)
+            b.record()
+            torch.cuda.synchronize()
+            best = min(best, a.elapsed_time(b) * 1e-3)
+        out[name] = nbytes / best
+    del h, d
+    return out
+
+
+def o1_c1_timing():
+    """O1 brute force (two nested loops over all ordered pairs) on C1, timed on the
+    host cores: the SURVEY §8(d) brute-force reference point."""
+    import oracle
+
+    cfg = workloads.get_config("c1")
+    pts = cfg.points()
+    t0 = time.perf_counter()
+    cnt, _ = oracle.bf_count(pts, cfg.eps)
+    dt = time.perf_counter() - t0
+    n = pts.shape[0]
+    return {"config": "c1", "pairs": cnt, "distance_calcs": n * (n - 1), "seconds": dt,
+            "calcs_per_s": n * (n - 1) / dt, "cores": oracle.num_threads()}
 
 
 def algorithmic_bytes(st: dict, pad: int) -> int:
@@ -142,10 +194,18 @@ def algorithmic_bytes(st: dict, pad: int) -> int:
     return 8 * st["pairs"] + n * (8 * pad + 12) + 16 * m + 8 * e
 
 
-def oracle_baseline(pts, eps, d_alg: int, stride: int, budget_s: float = 20.0):
-    """The CPU oracle (O2 grid, as it stands) on a strided sample of the queries."""
+def oracle_baseline(pts, eps, d_alg: int, stride: int, budget_s: float = 20.0, threads: int = 0):
+    """The CPU oracle (O2 grid, as it stands) on a strided sample of the queries; threads > 0
+    limits its OpenMP threads for this call (the 1-core run)."""
     import oracle
 
+    if threads:
+        full = oracle.num_threads()
+        oracle.set_threads(threads)
+        try:
+            return oracle_baseline(pts, eps, d_alg, stride, budget_s, 0)
+        finally:
+            oracle.set_threads(full)
     n = pts.shape[0]
     if stride <= 0:
         # calibrate on a tiny sample so the measured call lands near budget_s
@@ -297,6 +357,7 @@ def main():
     l0 = sj.sj_kernel_launches()
     for i in range(args.steps):
         flush_buf.fill_(i & 0xFF)
+        torch.cuda.synchronize()  # the flush is complete before the step's start event
         evs[i][0].record(stream)
         rc, c, tot, st = step(out, cap)
         evs[i][1].record(stream)
@@ -311,6 +372,7 @@ def main():
     launches = sj.sj_kernel_launches() - l0
     step_ms = [a.elapsed_time(b) for a, b in evs]
     total_ms = sum(step_ms)
+    step_sorted = sorted(step_ms)
     if world > 1:
         total_ms = sjdist.allreduce_counts([int(total_ms * 1e6)], group, dev, op=dist.ReduceOp.MAX)[0] / 1e6
     sampler.stop()
@@ -344,6 +406,54 @@ def main():
     roof["fp64_frac"] = (fp64_instr / (mean_join_ms * 1e-3)) / fp64_peak
     roof["hbm_frac"] = achieved / hbm_peak
     roof["fp64_peak_instr_per_s"] = fp64_peak
+    if facts:
+        roof["traffic_source"] = f"{facts.get('source')} ({facts.get('measured')})"
+    # the build (a2-a8) and the whole step against the HBM roofline, compulsory bytes only
+    bbytes = build_algorithmic_bytes(st0, cfg.dim, pad)
+    mean_build_ms = statistics.mean(build_ms)
+    build_roof = {"bound": "hbm", "algorithmic_bytes": bbytes, "ms": mean_build_ms,
+                  "achieved": bbytes / (mean_build_ms * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s"}
+    build_roof["frac"] = build_roof["achieved"] / hbm_peak
+    if facts.get("build_traffic_bytes"):
+        build_roof["traffic"] = facts["build_traffic_bytes"]
+    step_bytes = abytes + bbytes
+    step_roof = {"bound": "hbm", "algorithmic_bytes": step_bytes, "ms": total_ms / args.steps,
+                 "achieved": step_bytes / (total_ms / args.steps * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s"}
+    step_roof["frac"] = step_roof["achieved"] / hbm_peak
+
+    # the paper's batch scheme on the device: b_s = 1e8-pair buffers on 3 streams, sized
+    # by the 1 % estimator, each batch copied into the caller's HBM buffer -- the same step with
+    # the in-place fast path switched off
+    batched = None
+    if args.batched_steps > 0:
+        def step_batched():
+            h = build()
+            h.set_option("fast_path", 0)
+            rc, c = h.self_join(out, cap)
+            st = h.stats()
+            h.close()
+            return rc, c, st
+        step_batched()
+        torch.cuda.synchronize()
+        bms, nbat = [], 0
+        for i in range(args.batched_steps):
+            flush_buf.fill_(i & 0xFF)
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            rc, c, stb = step_batched()
+            b.record(stream)
+            torch.cuda.synchronize()
+            assert rc == sj.SJ_OK and c == local_pairs
+            bms.append(a.elapsed_time(b))
+            nbat = stb["batches"]
+        b_ms = sum(bms)
+        if world > 1:
+            b_ms = sjdist.allreduce_counts([int(b_ms * 1e6)], group, dev, op=dist.ReduceOp.MAX)[0] / 1e6
+        batched = {"value": d_alg * args.batched_steps / (b_ms * 1e-3), "unit": "calcs/s",
+                   "ms_per_step": b_ms / args.batched_steps, "steps": args.batched_steps, "batches": nbat,
+                   "batch_pairs": 100_000_000, "streams": 3,
+                   "note": "P:71 batch scheme on the device (fast path off): estimator-sized b_s buffers, D2D copies"}
 
     # e2e: the same step through the C ABI from pinned host buffers (H2D + D2H inside)
     e2e = None
@@ -371,6 +481,7 @@ def main():
         es = []
         for i in range(args.e2e_steps):
             flush_buf.fill_(i & 0xFF)
+            torch.cuda.synchronize()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(stream)
             rc, c = step_host()
@@ -384,11 +495,19 @@ def main():
         e2e = {"value": d_alg * args.e2e_steps / (e_ms * 1e-3), "unit": "calcs/s",
                "h2d_bytes_per_step": int(pts.nbytes) if (world == 1 or rank == 0) else 0,
                "d2h_bytes_per_step": int(local_pairs * 8), "ms_per_step": e_ms / args.e2e_steps,
-               "steps": args.e2e_steps}
+               "steps": args.e2e_steps, "ms_min": min(es)}
+        # against the measured PCIe rates: the time the step's copies need at the link's speed
+        rates = pcie_rates(dev)
+        t_link = e2e["h2d_bytes_per_step"] / rates["h2d"] + e2e["d2h_bytes_per_step"] / rates["d2h"]
+        e2e["pcie"] = {"h2d_gbs": rates["h2d"] / 1e9, "d2h_gbs": rates["d2h"] / 1e9,
+                       "copy_ms_at_link_rate": t_link * 1e3, "frac": t_link / (e2e["ms_per_step"] * 1e-3)}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = oracle_baseline(pts, cfg.eps, d_alg, args.ref_stride)
+        one = oracle_baseline(pts, cfg.eps, d_alg, 0, budget_s=8.0, threads=1)
+        cpu["one_core"] = {"value": one["value"], "unit": "calcs/s", "cores": 1, "sample": one["sample"]}
+        cpu["o1_bruteforce_c1"] = o1_c1_timing()
         cpu.pop("seconds", None)
         cpu.pop("stride", None)
 
@@ -404,18 +523,27 @@ def main():
                        "l2": "flushed before every step (256 MiB write, outside the step events)",
                        "output": "HBM-resident pairs (uint32 x2), written in place"},
             "self_join_s": total_ms / args.steps / 1e3,
+            "ms_per_step_median": statistics.median(step_ms), "ms_per_step_min": step_sorted[0],
+            "ms_per_step_max": step_sorted[-1],
             "phases_ms": {"build": statistics.mean(build_ms), "estimate": statistics.mean(est_ms),
                           "join": mean_join_ms, "step": total_ms / args.steps,
                           "join_min": min(join_ms), "join_max": max(join_ms),
+                          "join_median": statistics.median(join_ms), "build_median": statistics.median(build_ms),
                           "step_min": min(step_ms), "step_max": max(step_ms)},
             "roofline": roof,
+            "build_roofline": build_roof,
+            "step_roofline": step_roof,
+            "batched": batched,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches),
             "clocks": clocks,
         }
         if "wee" in facts:
-            line["warp_exec_efficiency"] = facts["wee"]
+            line["warp_exec_efficiency"] = {"value": facts["wee"], "source": facts.get("source"),
+                                            "measured": facts.get("measured"),
+                                            "kind": "ncu smsp__thread_inst_executed_per_inst_executed / 32, "
+                                                    "this config's emitting join launch, separate process"}
         emit(line, args)
     if world > 1:
         dist.destroy_process_group()

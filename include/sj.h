@@ -22,7 +22,19 @@
  *
  * Threading: a handle is not thread-safe; distinct handles are independent.
  * Every call runs on the CUDA device that was current when the handle was
- * created.  All calls are synchronous: they return after their GPU work ended.
+ * created.
+ *
+ * Stream ordering: the library runs on streams of its own.  Every call that reads or
+ * writes caller memory (sj_create*, sj_self_join, sj_neighbor_csr, sj_export_index,
+ * sj_create_from_index) first makes them wait for the work queued so far on the
+ * caller's stream -- the legacy default stream, or the one named with sj_set_stream
+ * -- so device inputs written asynchronously by the caller are complete before they
+ * are read.  Completion: sj_self_join, sj_neighbor_csr, sj_export_index and
+ * sj_create_from_index return after their GPU work ended.  sj_create / sj_create_ex /
+ * sj_create_part return once the caller's points (and ids) are no longer read; the
+ * build's last kernels may still run on the handle's stream, every later call on the
+ * handle is ordered after them, and an asynchronous error of theirs surfaces at the
+ * next call (SJ_SYNC_BUILD=1 in the environment makes the build fully synchronous).
  */
 #ifndef SJ_H
 #define SJ_H
@@ -33,7 +45,7 @@
 extern "C" {
 #endif
 
-#define SJ_ABI_VERSION 2
+#define SJ_ABI_VERSION 3
 
 typedef struct sj_handle sj_handle;
 
@@ -228,11 +240,53 @@ int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes
  * pointer, possibly on another GPU / process).  NULL on error. */
 sj_handle *sj_create_from_index(const void *blob, uint64_t bytes);
 
+/* The caller's CUDA stream (a cudaStream_t) for the ordering rule above, for the calling
+ * thread; NULL = the legacy default stream (the initial value).  The Python binding passes
+ * torch's current stream before every call. */
+void sj_set_stream(void *stream);
+
 /* ABI version (SJ_ABI_VERSION). */
 int sj_abi_version(void);
 
 /* Number of CUDA kernels libsj.so has launched in this process (diagnostics). */
 uint64_t sj_kernel_launches(void);
+
+/* ---- slab partition of a multi-GPU join -------------------
+ * The device-side arithmetic of cutting the global grid into slabs of whole dimension-0 cell
+ * columns; the caller only runs the collectives between the calls (all-reduce MIN/MAX of the
+ * bounds, all-reduce SUM of the histogram, all_to_all of the packed rows), then builds its
+ * partition with sj_create_part.  Column of a point: c = floor(fl(fl(x_0 - origin_0) / w)),
+ * w = fl(eps (1 + 2^-20)) -- the build's own cell arithmetic (readings c5, c6), so a cut never
+ * splits a cell.  These calls run on the caller's stream (sj_set_stream) and return after
+ * their GPU work ended.  points: n x dim row-major doubles on the current device; 0 <= n < 2^32. */
+
+/* Local per-dimension bounds: mn[d] / mx[d] (host double[dim]) = min / max of points[:, d]
+ * (+inf / -inf when n = 0).  SJ_EINVAL for a non-finite coordinate or bad arguments. */
+int sj_part_bounds(const double *points, uint64_t n, int dim, double *mn, double *mx);
+
+/* Number of dimension-0 cell columns of the global grid: c(max0) + 1 for the global origin0 and
+ * maximum max0 (host arithmetic, the same binary64 operations).  SJ_EINVAL, or SJ_EGRID when the
+ * column count reaches 2^30 (reading c5's bound). */
+int64_t sj_part_columns(double origin0, double max0, double eps);
+
+/* Column histogram of the local points: hist (device uint64[ncol], overwritten) counts the
+ * points of every column.  SJ_EINVAL if a point lies below origin0 or in a column >= ncol. */
+int sj_part_histogram(const double *points, uint64_t n, int dim, double origin0, double eps, uint64_t ncol,
+                      uint64_t *hist);
+
+/* Routes and packs the local points for the all-to-all, given the GLOBAL histogram (device
+ * uint64[ncol], the sum over the ranks).  Column c is owned by rank
+ * min(world - 1, floor(start_c * world / total)), start_c = the points of columns < c: slabs of
+ * whole columns balanced by points.  own_pts / own_ids (device, n rows of dim doubles / uint32)
+ * receive every point, grouped by owner rank ascending, input order inside a rank;
+ * own_counts (host uint64[world]) the rows per rank.  A point of column c >= 1 whose owner
+ * differs from owner(c - 1) is also packed into halo_pts / halo_ids (device, room for n rows)
+ * for rank owner(c - 1) -- the LID-UNICOMP forward cells lie at most one column ahead (P:174,
+ * Alg. 3) -- with halo_counts (host uint64[world]).  ids: device uint32[n] global ids, or NULL
+ * (ids = local positions).  1 <= world <= 2^20. */
+int sj_part_pack(const double *points, const uint32_t *ids, uint64_t n, int dim, double origin0, double eps,
+                 const uint64_t *hist, uint64_t ncol, int world, double *own_pts, uint32_t *own_ids,
+                 uint64_t *own_counts, double *halo_pts, uint32_t *halo_ids, uint64_t *halo_counts);
 
 /* ---- host-only helpers (no GPU needed) ------------------------------------ */
 

@@ -4,6 +4,7 @@ from __future__ import annotations
 import ctypes
 import os
 import re
+import sys
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _ROOT = os.path.dirname(_HERE)
@@ -73,6 +74,11 @@ _sig = {
     "sj_measure_fp64": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
     "sj_measure_atomics": (_int, [ctypes.POINTER(_dbl), ctypes.POINTER(_dbl)]),
     "sj_neighbor_csr": (_int, [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]),
+    "sj_set_stream": (None, [_vp]),
+    "sj_part_bounds": (_int, [_vp, _u64, _int, _vp, _vp]),
+    "sj_part_columns": (_i64, [_dbl, _dbl, _dbl]),
+    "sj_part_histogram": (_int, [_vp, _u64, _int, _dbl, _dbl, _u64, _vp]),
+    "sj_part_pack": (_int, [_vp, _vp, _u64, _int, _dbl, _dbl, _vp, _u64, _int, _vp, _vp, _vp, _vp, _vp, _vp]),
 }
 for _n, (_r, _a) in _sig.items():
     if os.environ.get("SJ_LIB_PATH") and not hasattr(_lib, _n):
@@ -102,6 +108,17 @@ def _ptr(x) -> int:
     return ctypes.addressof(x)
 
 
+def _order_after_torch() -> None:
+    """Name torch's current CUDA stream as the caller's stream (sj_set_stream), so the library
+    orders its work after whatever torch queued there (inputs still being written, buffers
+    still in use).  Argument marshalling only: no device work happens here."""
+    torch = sys.modules.get("torch")
+    if torch is None or not torch.cuda.is_available() or not torch.cuda.is_initialized():
+        _lib.sj_set_stream(None)
+        return
+    _lib.sj_set_stream(torch.cuda.current_stream().cuda_stream or None)
+
+
 def _err(code: int) -> SJError:
     return SJError(code, (_lib.sj_last_error() or b"").decode())
 
@@ -116,6 +133,12 @@ def _check(code: int) -> int:
 
 def sj_abi_version() -> int:
     return _lib.sj_abi_version()
+
+
+def sj_set_stream(stream) -> None:
+    """stream: a torch.cuda.Stream, a raw cudaStream_t (int) or None (legacy default stream)."""
+    raw = getattr(stream, "cuda_stream", stream)
+    _lib.sj_set_stream(raw or None)
 
 
 def sj_kernel_launches() -> int:
@@ -145,6 +168,7 @@ def _shape(points, n, dim, eps):
 def sj_create(points, n: int | None = None, dim: int | None = None, eps: float | None = None) -> int:
     """sj_create(points, eps) or sj_create(ptr, n, dim, eps).  Returns the raw handle (int)."""
     n, dim, eps = _shape(points, n, dim, eps)
+    _order_after_torch()
     h = _lib.sj_create(_ptr(points), int(n), int(dim), float(eps))
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
@@ -154,6 +178,7 @@ def sj_create(points, n: int | None = None, dim: int | None = None, eps: float |
 def sj_create_ex(points, n=None, dim=None, eps=None, pattern: int = 0, order: int = 0) -> int:
     """sj_create_ex(points, eps, pattern=, order=) or (ptr, n, dim, eps, pattern, order)."""
     n, dim, eps = _shape(points, n, dim, eps)
+    _order_after_torch()
     h = _lib.sj_create_ex(_ptr(points), int(n), int(dim), float(eps), int(pattern), int(order))
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
@@ -169,6 +194,7 @@ def sj_create_part(points, ids, n_query: int, eps: float, origin) -> int:
     org = np.ascontiguousarray(np.asarray(origin, dtype=np.float64).reshape(-1))
     if org.shape[0] != dim:
         raise SJError(SJ_EINVAL, f"origin needs {dim} values")
+    _order_after_torch()
     h = _lib.sj_create_part(_ptr(points), _ptr(ids), int(n), int(n_query), int(dim), float(eps), org.ctypes.data)
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
@@ -176,6 +202,7 @@ def sj_create_part(points, ids, n_query: int, eps: float, origin) -> int:
 
 
 def sj_create_from_index(blob, nbytes: int) -> int:
+    _order_after_torch()
     h = _lib.sj_create_from_index(_ptr(blob), int(nbytes))
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
@@ -185,6 +212,7 @@ def sj_create_from_index(blob, nbytes: int) -> int:
 def sj_self_join(h: int, out, cap: int):
     """Returns (status, count) with status SJ_OK or SJ_MORE; raises SJError on error."""
     cnt = _u64(0)
+    _order_after_torch()
     rc = _lib.sj_self_join(h, _ptr(out), int(cap), ctypes.byref(cnt))
     _check(rc)
     return rc, int(cnt.value)
@@ -194,6 +222,7 @@ def sj_neighbor_csr(h: int, row_off, nbrs, cap: int) -> int:
     """Fills row_off (uint64[n+1]) and, if nbrs is given, nbrs (uint32[cap]); returns the
     total number of neighbour entries.  Raises SJError on error (incl. cap < total)."""
     tot = _u64(0)
+    _order_after_torch()
     _check(_lib.sj_neighbor_csr(h, _ptr(row_off), _ptr(nbrs), int(cap), ctypes.byref(tot)))
     return int(tot.value)
 
@@ -218,6 +247,7 @@ def sj_get_stats(h: int) -> dict:
 
 def sj_export_index(h: int, dst=None, cap: int = 0) -> int:
     nbytes = _u64(0)
+    _order_after_torch()
     _check(_lib.sj_export_index(h, _ptr(dst), int(cap), ctypes.byref(nbytes)))
     return int(nbytes.value)
 
@@ -247,6 +277,64 @@ def sj_batch_chunks(n_chunks: int, n_batches: int, batch: int, queue: int = 1):
     out = np.zeros(max(cnt, 1), dtype=np.uint32)
     _check(_lib.sj_batch_chunks(int(n_chunks), int(n_batches), int(batch), int(queue), out.ctypes.data, out.size))
     return out[:cnt]
+
+
+# ------------------------------------------------------------------ slab partition (sj_part_*)
+
+def _part_points(points):
+    n, dim, _ = _shape(points, 0.0, None, None)
+    if not (hasattr(points, "is_cuda") and points.is_cuda):
+        raise SJError(SJ_EINVAL, "sj_part_*: points must be a CUDA float64 tensor")
+    return n, dim
+
+
+def sj_part_bounds(points):
+    """(min list, max list) per dimension of a CUDA (n, dim) float64 tensor."""
+    import numpy as np
+
+    n, dim = _part_points(points)
+    mn, mx = np.empty(dim), np.empty(dim)
+    _order_after_torch()
+    _check(_lib.sj_part_bounds(_ptr(points), n, dim, mn.ctypes.data, mx.ctypes.data))
+    return mn.tolist(), mx.tolist()
+
+
+def sj_part_columns(origin0: float, max0: float, eps: float) -> int:
+    return int(_check(_lib.sj_part_columns(float(origin0), float(max0), float(eps))))
+
+
+def sj_part_histogram(points, origin0: float, eps: float, ncol: int):
+    """Column histogram (CUDA int64 tensor of ncol counts) of the local points."""
+    import torch
+
+    n, dim = _part_points(points)
+    hist = torch.empty(ncol, dtype=torch.int64, device=points.device)
+    _order_after_torch()
+    _check(_lib.sj_part_histogram(_ptr(points), n, dim, float(origin0), float(eps), int(ncol), _ptr(hist)))
+    return hist
+
+
+def sj_part_pack(points, ids, origin0: float, eps: float, hist, world: int):
+    """Rows packed per destination: (own_pts, own_ids, own_counts, halo_pts, halo_ids, halo_counts);
+    the point / id tensors are CUDA (n, dim) float64 / (n,) int32 (uint32 bits), counts lists."""
+    import numpy as np
+    import torch
+
+    n, dim = _part_points(points)
+    dev = points.device
+    if ids is not None and (ids.dtype != torch.int32 or ids.numel() != n or not ids.is_contiguous()):
+        raise SJError(SJ_EINVAL, "sj_part_pack: ids must be a contiguous int32 tensor of n global ids")
+    own_p = torch.empty((max(n, 1), dim), dtype=torch.float64, device=dev)
+    own_i = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
+    halo_p = torch.empty((max(n, 1), dim), dtype=torch.float64, device=dev)
+    halo_i = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
+    oc = np.zeros(world, dtype=np.uint64)
+    hc = np.zeros(world, dtype=np.uint64)
+    _order_after_torch()
+    _check(_lib.sj_part_pack(_ptr(points), _ptr(ids), n, dim, float(origin0), float(eps), _ptr(hist), hist.numel(),
+                             int(world), _ptr(own_p), _ptr(own_i), oc.ctypes.data, _ptr(halo_p), _ptr(halo_i),
+                             hc.ctypes.data))
+    return own_p, own_i, [int(x) for x in oc], halo_p, halo_i, [int(x) for x in hc]
 
 
 def sj_measure_fp64():

@@ -49,6 +49,9 @@ inline void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); 
 // Host-side phase timer printed to stderr when SJ_DEBUG=1 (diagnostics only).
 void debug_mark(const char *label);
 
+// The caller's stream of the calling thread (sj_set_stream; the legacy default stream by default).
+cudaStream_t caller_stream();
+
 // --------------------------------------------------------------------------- memory
 // Stream-ordered allocations from the device's default memory pool.  The pool's
 // release threshold is raised once, so repeated create/destroy cycles reuse memory

@@ -132,6 +132,14 @@ int wait_flag(volatile unsigned *flag, unsigned epoch, cudaStream_t s) {
     }
 }
 
+// ------------------------------------------------------------------------- caller stream
+// The stream the caller produced its inputs on (sj_set_stream; thread-local).  Every entry point
+// that reads or writes caller memory first makes the handle's stream wait for it, so device
+// inputs written asynchronously by the caller (e.g. torch kernels on its current stream) are
+// complete before the library reads them, and caller buffers are not written under pending work.
+static thread_local cudaStream_t g_caller_stream = cudaStreamLegacy;
+cudaStream_t caller_stream() { return g_caller_stream; }
+
 // ------------------------------------------------------------------------- small kernels
 __global__ void set_u64_kernel(unsigned long long *p, unsigned long long v) { *p = v; }
 
@@ -171,6 +179,7 @@ struct sj_handle {
     cudaStream_t s_main = nullptr;
     cudaEvent_t ev_a = nullptr, ev_b = nullptr, ev_c = nullptr, ev_d = nullptr, ev_e = nullptr;
     cudaEvent_t ev_ba = nullptr, ev_bb = nullptr;  // build start / end
+    cudaEvent_t ev_in = nullptr;  // the caller's stream, recorded at entry (order_after_caller)
     sj::BuildSide side{};                         // the build's side stream and its events
     int pending = 0;  // 1: the build's tail {n_chunks, E} and its timing not read yet (ix_ready)
     sj::Index ix;
@@ -231,7 +240,7 @@ struct Core {
     int device;
     int num_sms;
     cudaStream_t s;
-    cudaEvent_t ev[7];
+    cudaEvent_t ev[8];
     sj::BuildSide side;
     unsigned long long *d_ctr;
     uint64_t *mail;
@@ -256,6 +265,7 @@ int handle_init_common(sj_handle *h) {
                 h->ev_e = c.ev[4];
                 h->ev_ba = c.ev[5];
                 h->ev_bb = c.ev[6];
+                h->ev_in = c.ev[7];
                 h->side = c.side;
                 h->d_ctr = c.d_ctr;
                 h->mail = c.mail;
@@ -276,6 +286,7 @@ int handle_init_common(sj_handle *h) {
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_e));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_ba));
     SJ_CUDA_TRY(cudaEventCreate(&h->ev_bb));
+    SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->ev_in, cudaEventDisableTiming));
     SJ_CUDA_TRY(cudaStreamCreateWithPriority(&h->side.s2, cudaStreamNonBlocking, prio_least));
     SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.ea, cudaEventDisableTiming));
     SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.eg, cudaEventDisableTiming));
@@ -289,7 +300,7 @@ int handle_init_common(sj_handle *h) {
 
 // Returns the handle's core to the cache (stream drained first); false if it must be freed.
 bool core_release(sj_handle *h) {
-    if (!h->s_main || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->ev_e || !h->ev_ba || !h->ev_bb || !h->d_ctr ||
+    if (!h->s_main || !h->ev_a || !h->ev_b || !h->ev_c || !h->ev_d || !h->ev_e || !h->ev_ba || !h->ev_bb || !h->ev_in || !h->d_ctr ||
         !h->mail || !h->side.s2 || !h->side.ea || !h->side.eg || !h->side.eq || !h->side.ej)
         return false;
     if (cudaStreamSynchronize(h->side.s2) != cudaSuccess) {
@@ -302,7 +313,7 @@ bool core_release(sj_handle *h) {
     }
     std::lock_guard<std::mutex> lk(g_core_mu);
     if (g_core_cache.size() >= 64) return false;
-    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e, h->ev_ba, h->ev_bb}, h->side, h->d_ctr,
+    g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e, h->ev_ba, h->ev_bb, h->ev_in}, h->side, h->d_ctr,
                                 h->mail});
     return true;
 }
@@ -445,6 +456,13 @@ int ix_ready(sj_handle *h) {
     return SJ_OK;
 }
 
+// The handle's main stream waits for the work queued so far on the caller's stream.
+int order_after_caller(sj_handle *h) {
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_in, g_caller_stream));
+    SJ_CUDA_TRY(cudaStreamWaitEvent(h->s_main, h->ev_in, 0));
+    return SJ_OK;
+}
+
 int join_blocks(const sj_handle *h, int mode, int *blocks) {
     int occ = 0;
     SJ_TRY(join_occupancy(h->ix.dim, h->k, mode, h->ix.pattern == SJ_PATTERN_GCG, &occ));
@@ -538,6 +556,11 @@ int fill_pipeline(sj_handle *h) {
 // Drives the staged batch pipeline until the caller's buffer is full or the join ends.
 int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     uint64_t written = 0;
+    // the copies into the caller's buffer run on the slot streams: order them after the caller
+    // (sj_self_join made s_main wait for the caller's stream)
+    SJ_CUDA_TRY(cudaEventRecord(h->ev_in, h->s_main));
+    for (int i = 0; i < h->streams; ++i)
+        if (h->slots[i].stream) SJ_CUDA_TRY(cudaStreamWaitEvent(h->slots[i].stream, h->ev_in, 0));
     for (;;) {
         SJ_TRY(fill_pipeline(h));
         if (h->jobs.empty()) break;
@@ -1142,6 +1165,10 @@ int sj_abi_version(void) { return SJ_ABI_VERSION; }
 
 uint64_t sj_kernel_launches(void) { return g_launches.load(); }
 
+void sj_set_stream(void *stream) {
+    g_caller_stream = stream ? static_cast<cudaStream_t>(stream) : cudaStreamLegacy;
+}
+
 const char *sj_last_error(void) { return g_err; }
 
 static int create_common(sj_handle **out_h) {
@@ -1205,7 +1232,7 @@ static sj_handle *create_impl(const double *points, uint64_t n, int dim, double 
     cudaStream_t s = h->s_main;
     const double *d_raw = points;
     double *d_copy = nullptr;
-    int rc = SJ_OK;
+    int rc = order_after_caller(h);  // device points may still be in flight on the caller's stream
     // host input, or a device pointer that is not 16-byte aligned (the build reads double2)
     if (!is_device_ptr(points, h->device) || (reinterpret_cast<uintptr_t>(points) & 15u)) {
         // a1: upload (the library owns its copy; caller keeps `points`)
@@ -1285,6 +1312,7 @@ int sj_self_join(sj_handle *h, uint32_t *out_pairs, uint64_t cap, uint64_t *coun
         return SJ_EINVAL;
     }
     int rc = ensure_device(h);
+    if (rc == SJ_OK) rc = order_after_caller(h);  // the caller's buffer may have pending work
     if (rc < 0) return fail(h, rc);
     if (h->state == 1 && out_pairs) {
         rc = continue_staged(h, out_pairs, cap, count);
@@ -1304,7 +1332,9 @@ int sj_neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t ca
         set_error("sj_neighbor_csr: handle is in the error state");
         return SJ_ESTATE;
     }
-    const int rc = neighbor_csr(h, row_off, nbrs, cap, total);
+    int rc = ensure_device(h);
+    if (rc == SJ_OK) rc = order_after_caller(h);
+    if (rc == SJ_OK) rc = neighbor_csr(h, row_off, nbrs, cap, total);
     return rc == SJ_EINVAL ? rc : fail(h, rc);
 }
 
@@ -1329,6 +1359,7 @@ void sj_destroy(sj_handle *h) {
         if (h->ev_e) cudaEventDestroy(h->ev_e);
         if (h->ev_ba) cudaEventDestroy(h->ev_ba);
         if (h->ev_bb) cudaEventDestroy(h->ev_bb);
+        if (h->ev_in) cudaEventDestroy(h->ev_in);
         if (h->side.s2) {
             cudaStreamSynchronize(h->side.s2);
             cudaStreamDestroy(h->side.s2);
@@ -1478,6 +1509,7 @@ int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes
         return SJ_EINVAL;
     }
     SJ_TRY(ensure_device(h));
+    SJ_TRY(order_after_caller(const_cast<sj_handle *>(h)));
     char *d = static_cast<char *>(dst);
     const void *src[7] = {h->ix.pts, h->ix.orig, h->ix.qmap, h->ix.cellq, h->ix.runs, h->ix.cell_lid, h->ix.chunks};
     SJ_CUDA_TRY(cudaMemcpyAsync(d, &b, sizeof b, cudaMemcpyDefault, h->s_main));
@@ -1485,6 +1517,37 @@ int sj_export_index(const sj_handle *h, void *dst, uint64_t cap, uint64_t *bytes
         if (b.bytes[i]) SJ_CUDA_TRY(cudaMemcpyAsync(d + b.off[i], src[i], b.bytes[i], cudaMemcpyDefault, h->s_main));
     SJ_CUDA_TRY(cudaStreamSynchronize(h->s_main));
     return SJ_OK;
+}
+
+// Every field of a received blob is checked before anything is copied or read by a kernel: the
+// blob crosses process boundaries (NCCL broadcast), so a truncated or corrupt one must give
+// SJ_EINVAL, not out-of-bounds copies or device reads.
+static bool blob_header_ok(const BlobHeader &b, uint64_t bytes, const char **why) {
+    *why = "";
+    if (b.magic != kMagic) return *why = "magic (not an SJIDX004 blob of this library version)", false;
+    if (b.total > bytes || b.total < kHdr) return *why = "total size exceeds the buffer", false;
+    if (b.dim < 1 || b.dim > SJ_MAX_DIM) return *why = "dim", false;
+    if (b.n < 1 || b.n >= (1ull << 32)) return *why = "n", false;
+    const int pad = b.dim == 1 ? 1 : ((b.dim + 1) & ~1);
+    if (b.pad != pad) return *why = "pad", false;
+    const int pattern = b.pattern_order & 0xFF, order = (b.pattern_order >> 8) & 0xFF;
+    if (pattern > SJ_PATTERN_UNICOMP || order > SJ_ORDER_INPUT || (b.pattern_order >> 16)) return *why = "pattern/order", false;
+    if (b.n_cells < 1 || b.n_cells > b.n) return *why = "n_cells", false;
+    if (b.n_chunks < 1 || b.n_chunks > b.n || b.n_chunks >= (1ull << 32)) return *why = "n_chunks", false;
+    if (b.n_query > b.n) return *why = "n_query", false;
+    if (b.runs_len && b.runs_len < b.n_runs) return *why = "runs_len", false;
+    if (!(b.e2 > 0.0) || !(b.w > 0.0) || b.key_bits < 0 || b.key_bits > 64) return *why = "eps/w/key_bits", false;
+    const uint64_t runs = b.runs_len ? b.runs_len : b.n_runs;
+    const uint64_t want[7] = {b.n * (uint64_t)pad * sizeof(double), b.n * sizeof(uint32_t), b.n * sizeof(uint2),
+                              b.n_cells * sizeof(uint4), runs * sizeof(uint2), b.n_cells * sizeof(uint64_t),
+                              (b.n_chunks + 1) * sizeof(uint32_t)};
+    uint64_t end = kHdr;
+    for (int i = 0; i < 7; ++i) {
+        if (b.bytes[i] != want[i]) return *why = "array size", false;
+        if (b.off[i] < end || b.off[i] > b.total || b.bytes[i] > b.total - b.off[i]) return *why = "array extent", false;
+        end = b.off[i] + b.bytes[i];
+    }
+    return true;
 }
 
 sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
@@ -1499,17 +1562,32 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
         set_error("sj_create_from_index: no CUDA device available");
         return nullptr;
     }
-    BlobHeader b;
-    if (cudaMemcpy(&b, blob, sizeof b, cudaMemcpyDefault) != cudaSuccess) {
-        set_error("sj_create_from_index: %s", cudaGetErrorString(cudaGetLastError()));
-        return nullptr;
-    }
-    if (b.magic != kMagic || b.total > bytes || b.dim < 1 || b.dim > SJ_MAX_DIM) {
-        set_error("sj_create_from_index: bad header");
-        return nullptr;
-    }
     sj_handle *h = nullptr;
     if (create_common(&h) < 0) return nullptr;
+    cudaStream_t s = h->s_main;
+    // the blob may have been written on the caller's stream (e.g. the NCCL broadcast's output)
+    BlobHeader b;
+    int rc = order_after_caller(h);
+    if (rc == SJ_OK && (cudaMemcpyAsync(h->mail, blob, sizeof b, cudaMemcpyDefault, s) != cudaSuccess ||
+                        cudaStreamSynchronize(s) != cudaSuccess)) {
+        set_error("sj_create_from_index: %s", cudaGetErrorString(cudaGetLastError()));
+        rc = SJ_ECUDA;
+    }
+    const char *why = "";
+    if (rc == SJ_OK) {
+        static_assert(sizeof(BlobHeader) <= kMailBytes, "header through the mailbox");
+        memcpy(&b, h->mail, sizeof b);
+        if (!blob_header_ok(b, bytes, &why)) {
+            set_error("sj_create_from_index: bad header (%s)", why);
+            rc = SJ_EINVAL;
+        }
+    }
+    if (rc < 0) {
+        std::string keep = g_err;
+        sj_destroy(h);
+        snprintf(g_err, sizeof g_err, "%s", keep.c_str());
+        return nullptr;
+    }
     Index &ix = h->ix;
     ix.n = b.n;
     ix.dim = b.dim;
@@ -1534,10 +1612,8 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
     ix.dist_calcs = b.dist_calcs;
     ix.max_w = b.max_w;
     ix.lookup_hash = (int)b.lookup_hash;
-    cudaStream_t s = h->s_main;
     void **dst[7] = {(void **)&ix.pts,  (void **)&ix.orig,     (void **)&ix.qmap,  (void **)&ix.cellq,
                      (void **)&ix.runs, (void **)&ix.cell_lid, (void **)&ix.chunks};
-    int rc = SJ_OK;
     for (int i = 0; i < 7 && rc == SJ_OK; ++i) {
         rc = dev_alloc(dst[i], b.bytes[i] + 32, s);
         if (rc == SJ_OK && b.bytes[i] &&

@@ -78,90 +78,112 @@ def distributed_self_join(points, eps: float, out, cap: int, group=None, src: in
 # slab needs, besides its own points, only the points of the first cell column of the next
 # non-empty slab (the halo).  Each rank builds a partitioned handle (sj_create_part: queries =
 # own points, halo = candidates, the global grid origin, global ids) and joins it; the pair
-# sets of the ranks are disjoint and their union is the global join.  Exchanges: an all-reduce
-# of the per-dimension bounds, an all-reduce of the column histogram, and two all-to-alls
-# (own points, halo points) -- NCCL over NVLink on GPUs, gloo in the CPU tests.
-
-def cell_width(eps: float) -> float:
-    """Cell side w = eps(1 + 2^-20) (reading c5), in binary64 like the library."""
-    return float(eps) * (1.0 + 2.0 ** -20)
-
-
-def cell_columns(x0: torch.Tensor, origin0: float, eps: float) -> torch.Tensor:
-    """Dimension-0 cell coordinate floor(fl(fl(x - origin) / w)) (IEEE binary64 RN, one
-    subtraction and one division: the library's a3 arithmetic), as int64."""
-    return torch.floor((x0 - origin0) / cell_width(eps)).to(torch.int64)
+# sets of the ranks are disjoint and their union is the global join.
+#
+# Every piece of the cut's arithmetic -- bounds, the dimension-0 cell column of every point,
+# the column histogram, slab ownership, the halo selection and the packing of the rows per
+# destination -- runs in libsj (sj_part_*, csrc/partition.cu).  This module only moves data
+# between the calls with collectives: an all-reduce of the bounds, an all-reduce of the column
+# histogram and two all-to-alls (own rows, halo rows) -- NCCL over NVLink on GPUs.  The router
+# argument lets the CPU tests drive the same collective plumbing with gloo and a reference
+# router (tests/slab_ref.py); the product path always uses LibRouter.
 
 
-def slab_owners(hist: torch.Tensor, world: int) -> torch.Tensor:
-    """Owner rank of every cell column: columns are dealt to ranks in order, a column wholly to
-    the rank in whose share (by point count) its first point falls -- slabs of whole columns,
-    balanced to within one column.  hist: points per column (int64)."""
-    total = int(hist.sum().item())
-    if total == 0:
-        return torch.zeros_like(hist)
-    start = torch.cumsum(hist, 0) - hist  # global position of each column's first point
-    return torch.clamp((start * world) // total, max=world - 1)
+class LibRouter:
+    """The slab arithmetic of libsj (sj_part_*): device tensors in, device tensors out."""
+
+    def bounds(self, points):
+        from ._lib import sj_part_bounds
+        return sj_part_bounds(points)
+
+    def columns(self, origin0: float, max0: float, eps: float) -> int:
+        from ._lib import sj_part_columns
+        return sj_part_columns(origin0, max0, eps)
+
+    def histogram(self, points, origin0: float, eps: float, ncol: int):
+        from ._lib import sj_part_histogram
+        return sj_part_histogram(points, origin0, eps, ncol)
+
+    def pack(self, points, ids, origin0: float, eps: float, hist, world: int):
+        from ._lib import sj_part_pack
+        return sj_part_pack(points, ids, origin0, eps, hist, world)
 
 
-def _all_to_all(x: torch.Tensor, dest: torch.Tensor, world: int, group=None):
-    """Send row i of x to rank dest[i]; returns the rows this rank receives (ordered by source
-    rank, stable within a source)."""
-    order = torch.argsort(dest, stable=True)
-    send = x[order].contiguous()
-    scount = torch.bincount(dest, minlength=world).to(torch.int64)
+def _host_staged(group) -> bool:
+    """gloo (the CPU tests, several processes sharing one GPU) moves CUDA tensors through host
+    memory; NCCL takes them as they are."""
+    return dist.get_backend(group) == "gloo"
+
+
+def _all_reduce(t: torch.Tensor, op, group=None) -> torch.Tensor:
+    if t.is_cuda and _host_staged(group):
+        c = t.cpu()
+        dist.all_reduce(c, op=op, group=group)
+        return c.to(t.device)
+    dist.all_reduce(t, op=op, group=group)
+    return t
+
+
+def _exchange(rows: torch.Tensor, ids: torch.Tensor, counts, group=None):
+    """all_to_all of packed rows (grouped by destination rank, `counts` rows each) and their
+    ids; returns the rows and ids this rank receives, ordered by source rank."""
+    world = len(counts)
+    if rows.is_cuda and _host_staged(group):
+        r, i = _exchange(rows.cpu(), ids.cpu(), counts, group)
+        return r.to(rows.device), i.to(rows.device)
+    dev = rows.device
+    dim = rows.shape[1]
+    scount = torch.tensor([int(c) for c in counts], dtype=torch.int64, device=dev)
     rcount = torch.empty_like(scount)
     dist.all_to_all_single(rcount, scount, group=group)
     sc, rc = scount.tolist(), rcount.tolist()
-    out = torch.empty((sum(rc),) + tuple(x.shape[1:]), dtype=x.dtype, device=x.device)
-    dist.all_to_all_single(out, send, rc, sc, group=group)
-    return out
+    out = torch.empty((sum(rc), dim), dtype=rows.dtype, device=dev)
+    out_ids = torch.empty(sum(rc), dtype=ids.dtype, device=dev)
+    dist.all_to_all_single(out, rows[: sum(sc)].contiguous(), rc, sc, group=group)
+    dist.all_to_all_single(out_ids, ids[: sum(sc)].contiguous(), rc, sc, group=group)
+    assert world == dist.get_world_size(group)
+    return out, out_ids
 
 
-def slab_partition(points: torch.Tensor, ids: torch.Tensor, eps: float, group=None):
+def slab_partition(points: torch.Tensor, ids: torch.Tensor, eps: float, group=None, router=None):
     """This rank's partition of a self-join whose points are spread over the ranks.
-    points: (n_local, dim) float64, ids: (n_local,) int64 global ids (any device; collectives run
-    there).  Returns (part_points, part_ids int64, n_query, origin list): own points first,
-    then the halo."""
+    points: (n_local, dim) float64, ids: (n_local,) int32 global ids (the uint32 bits) on the
+    device the collectives run on.  Returns (part_points, part_ids int32, n_query, origin list):
+    own points first, then the halo."""
+    router = router or LibRouter()
     world = dist.get_world_size(group)
-    dev = points.device
     dim = points.shape[1]
-    inf = torch.full((dim,), float("inf"), dtype=torch.float64, device=dev)
-    mn = points.min(0).values if points.shape[0] else inf
-    mx = points.max(0).values if points.shape[0] else -inf
-    dist.all_reduce(mn, op=dist.ReduceOp.MIN, group=group)
-    dist.all_reduce(mx, op=dist.ReduceOp.MAX, group=group)
+    mn, mx = router.bounds(points)
+    mn = torch.tensor(mn, dtype=torch.float64, device=points.device)
+    mx = torch.tensor(mx, dtype=torch.float64, device=points.device)
+    mn = _all_reduce(mn, dist.ReduceOp.MIN, group)
+    mx = _all_reduce(mx, dist.ReduceOp.MAX, group)
     origin = [float(v) for v in mn.tolist()]
-    ncol = int(cell_columns(mx[:1], origin[0], eps).item()) + 1
-    col = cell_columns(points[:, 0], origin[0], eps)
-    hist = torch.bincount(col, minlength=ncol).to(torch.int64)
-    dist.all_reduce(hist, group=group)
-    owner = slab_owners(hist, world)
-    own = owner[col]
-    # halo: a column's points also go to the owner of the column before it, if that differs
-    prev = owner[torch.clamp(col - 1, min=0)]
-    hsel = (col >= 1) & (prev != own)
-    rows = torch.cat([points, ids.to(torch.float64).unsqueeze(1)], 1)  # ids < 2^32: exact in binary64
-    mine = _all_to_all(rows, own, world, group)
-    halo = _all_to_all(rows[hsel], prev[hsel], world, group)
-    part = torch.cat([mine, halo], 0)
-    return part[:, :dim].contiguous(), part[:, dim].to(torch.int64), int(mine.shape[0]), origin
+    ncol = router.columns(origin[0], float(mx[0].item()), eps)
+    hist = _all_reduce(router.histogram(points, origin[0], eps, ncol), dist.ReduceOp.SUM, group)
+    own_p, own_i, own_c, halo_p, halo_i, halo_c = router.pack(points, ids, origin[0], eps, hist, world)
+    mine, mine_ids = _exchange(own_p, own_i, own_c, group)
+    halo, halo_ids = _exchange(halo_p, halo_i, halo_c, group)
+    part = torch.cat([mine, halo], 0) if halo.shape[0] else mine
+    part_ids = torch.cat([mine_ids, halo_ids], 0) if halo.shape[0] else mine_ids
+    assert part.shape[1] == dim
+    return part, part_ids, int(mine.shape[0]), origin
 
 
 def partitioned_self_join(points: torch.Tensor, ids: torch.Tensor, eps: float, group=None, **options):
     """Spatially partitioned multi-GPU join: slab_partition, then this rank's partitioned handle
-    joins into a device buffer sized by its count.  Returns (pairs (m, 2) int32 holding uint32
-    global ids, local pair count, all-reduced total)."""
+    joins into a device buffer sized by its count.  points / ids (int32 global ids) on this
+    rank's GPU.  Returns (pairs (m, 2) int32 holding uint32 global ids, local pair count,
+    all-reduced total)."""
     from ._lib import self_join_pairs
 
-    dev = torch.device("cuda", torch.cuda.current_device())
+    dev = points.device
     ppts, pids, nq, origin = slab_partition(points, ids, eps, group)
-    ids32 = (pids & 0xFFFFFFFF).to(torch.int32)  # the library reads the bits as uint32
     if ppts.shape[0] == 0:  # an empty slab (more ranks than occupied cell columns)
         pairs = torch.empty((0, 2), dtype=torch.int32, device=dev)
     else:
-        with Handle(ppts.to(dev), eps, part=(ids32.to(dev), nq, origin), **options) as h:
+        with Handle(ppts, eps, part=(pids, nq, origin), **options) as h:
             pairs = self_join_pairs(h, dev)
     local = int(pairs.shape[0])
-    total = allreduce_counts([local], group, points.device)[0]
+    total = allreduce_counts([local], group, dev)[0]
     return pairs, local, total

@@ -14,7 +14,7 @@ def test_exports_every_declared_symbol():
     assert "sj_create" in names and "sj_self_join" in names and "sj_destroy" in names
     for n in names:
         assert hasattr(_lib._lib, n), f"libsj.so does not export {n}"
-    assert sj.sj_abi_version() == 2
+    assert sj.sj_abi_version() == 3
 
 
 def test_library_is_sm100a_only():

@@ -39,13 +39,14 @@ def _worker(rank, world, port, name, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from paper_conf_ipps_galletg19_b200 import dist as sjdist
+        from slab_ref import RefRouter
 
         pts, eps = _data(name)
         # the input is spread over the ranks arbitrarily (not by space)
         home = np.random.default_rng(11).integers(0, world, pts.shape[0])
         sel = np.nonzero(home == rank)[0]
-        p, i, nq, origin = sjdist.slab_partition(torch.from_numpy(pts[sel]), torch.from_numpy(sel.astype(np.int64)),
-                                                 eps)
+        p, i, nq, origin = sjdist.slab_partition(torch.from_numpy(pts[sel]), torch.from_numpy(sel.astype(np.int32)),
+                                                 eps, router=RefRouter())
         q.put((rank, p.numpy(), i.numpy(), nq, origin))
     finally:
         dist.destroy_process_group()
@@ -55,7 +56,7 @@ def _worker(rank, world, port, name, q):
 @pytest.mark.parametrize("name", ["c1", "c5", "c3k64"])
 def test_slab_partition(world, name):
     import oracle
-    from paper_conf_ipps_galletg19_b200 import dist as sjdist
+    from slab_ref import columns_of
 
     ctx = mp.get_context("spawn")
     qq = ctx.Queue()
@@ -70,7 +71,7 @@ def test_slab_partition(world, name):
     pts, eps = _data(name)
     n = pts.shape[0]
     origin = pts.min(0)
-    col = sjdist.cell_columns(torch.from_numpy(pts[:, 0]), float(origin[0]), eps).numpy()
+    col = columns_of(pts[:, 0], float(origin[0]), eps)
     owner_of = np.full(n, -1)
     local = []
     for r in range(world):

@@ -22,6 +22,7 @@ import oracle  # noqa: E402
 import paper_conf_ipps_galletg19_b200 as sj  # noqa: E402
 import workloads  # noqa: E402
 from paper_conf_ipps_galletg19_b200 import dist as sjdist  # noqa: E402
+from slab_ref import RefRouter, columns_of, owners  # noqa: E402
 
 DEV = "cuda:0"
 
@@ -29,9 +30,8 @@ DEV = "cuda:0"
 def cut_slabs(pts, eps, nslab):
     """Slabs of whole dimension-0 cell columns (balanced by points) + the halo of each."""
     origin = pts.min(0)
-    col = sjdist.cell_columns(torch.from_numpy(pts[:, 0]), float(origin[0]), eps).numpy()
-    hist = torch.from_numpy(np.bincount(col).astype(np.int64))
-    owner_col = sjdist.slab_owners(hist, nslab).numpy()
+    col = columns_of(pts[:, 0], float(origin[0]), eps)
+    owner_col = owners(np.bincount(col), nslab)
     own = owner_col[col]
     prev = owner_col[np.maximum(col - 1, 0)]
     out = []
@@ -121,8 +121,8 @@ def _worker(rank, world, port, name, n, q):
         pts = cfg.points()
         home = np.random.default_rng(5).integers(0, world, pts.shape[0])
         sel = np.nonzero(home == rank)[0]
-        pairs, local, total = sjdist.partitioned_self_join(torch.from_numpy(pts[sel]),
-                                                           torch.from_numpy(sel.astype(np.int64)), cfg.eps, k=8)
+        pairs, local, total = sjdist.partitioned_self_join(torch.from_numpy(pts[sel]).cuda(),
+                                                           torch.from_numpy(sel.astype(np.int32)).cuda(), cfg.eps, k=8)
         q.put((rank, pairs.cpu().numpy().view(np.uint32).reshape(-1, 2).copy(), local, total))
     finally:
         dist.destroy_process_group()
@@ -147,3 +147,97 @@ def test_partitioned_join_across_processes(world, name, n):
     np.testing.assert_array_equal(oracle.canonical(cat), want)
     for r in range(world):
         assert res[r][2] == want.shape[0] and res[r][1] == res[r][0].shape[0]
+
+
+# ------------------------------------------------------------------ the slab arithmetic in libsj
+
+def boundary_points(seed=3):
+    """Points on, just below and just above dimension-0 column boundaries (x = o + k w (1 + d),
+    d in {-2^-52, 0, 2^-52}): where a rounding difference between two column computations would
+    put a point in another column than the build's own cell ids."""
+    rng = np.random.default_rng(seed)
+    eps = 0.013
+    w = eps * (1.0 + 2.0 ** -20)
+    k = rng.integers(0, 300, 6000).astype(np.float64)
+    d = rng.choice([-2.0 ** -52, 0.0, 2.0 ** -52], 6000)
+    x0 = 0.25 + k * w * (1.0 + d)
+    x0[0] = 0.25  # the origin itself
+    x1 = rng.random(6000) * 0.5
+    return np.ascontiguousarray(np.stack([x0, x1], 1)), eps
+
+
+def router_cases():
+    out = []
+    for name, n in (("c5", 70_001), ("c3k64", 50_021), ("c4k32", 20_011), ("c1", None)):
+        cfg = workloads.get_config(name)
+        cfg = cfg.scaled(n) if n else cfg
+        out.append((name, cfg.points(), cfg.eps))
+    pb, eb = boundary_points()
+    out.append(("boundaries", pb, eb))
+    return out
+
+
+@pytest.mark.parametrize("name,pts,eps", router_cases(), ids=[c[0] for c in router_cases()])
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_lib_router_equals_reference(name, pts, eps, world):
+    lib, ref = sjdist.LibRouter(), RefRouter()
+    dp = torch.from_numpy(pts).to(DEV)
+    cp = torch.from_numpy(pts)
+    ids = torch.from_numpy((np.arange(pts.shape[0]) * 7 + 3).astype(np.int32))
+    assert lib.bounds(dp) == ref.bounds(cp)
+    mn, mx = ref.bounds(cp)
+    ncol = lib.columns(mn[0], mx[0], eps)
+    assert ncol == ref.columns(mn[0], mx[0], eps)
+    h_lib = lib.histogram(dp, mn[0], eps, ncol)
+    h_ref = ref.histogram(cp, mn[0], eps, ncol)
+    np.testing.assert_array_equal(h_lib.cpu().numpy(), h_ref.numpy())
+    # a "global" histogram: this rank's, plus a second rank holding the same points shifted
+    got = lib.pack(dp, ids.to(DEV), mn[0], eps, h_lib, world)
+    want = ref.pack(cp, ids, mn[0], eps, h_ref, world)
+    for g, w_ in zip(got, want):
+        if isinstance(w_, list):
+            assert g == w_
+        else:
+            rows = int(w_.shape[0])
+            np.testing.assert_array_equal(g[:rows].cpu().numpy(), w_.numpy())
+
+
+def test_boundary_points_partition_like_the_build():
+    """The slab cut by libsj's columns never splits a cell of the build (sj_create_part rejects
+    a cell that mixes query and halo points), and the union of the slabs is the oracle's join."""
+    pts, eps = boundary_points()
+    want = oracle.grid_pairs(pts, eps)
+    lib = sjdist.LibRouter()
+    dp = torch.from_numpy(pts).to(DEV)
+    mn, mx = lib.bounds(dp)
+    ncol = lib.columns(mn[0], mx[0], eps)
+    hist = lib.histogram(dp, mn[0], eps, ncol)
+    world = 5
+    own_p, own_i, oc, halo_p, halo_i, hc = lib.pack(dp, None, mn[0], eps, hist, world)
+    parts, o0, h0 = [], 0, 0
+    for r in range(world):
+        p = torch.cat([own_p[o0:o0 + oc[r]], halo_p[h0:h0 + hc[r]]]).contiguous()
+        i = torch.cat([own_i[o0:o0 + oc[r]], halo_i[h0:h0 + hc[r]]]).contiguous()
+        o0 += oc[r]
+        h0 += hc[r]
+        if p.shape[0] == 0:
+            continue
+        with sj.Handle(p, eps, part=(i, oc[r], mn), k=8) as h:
+            parts.append(sj.self_join_pairs(h, DEV).cpu().numpy().view(np.uint32).reshape(-1, 2))
+    cat = np.concatenate(parts)
+    assert cat.shape == want.shape
+    np.testing.assert_array_equal(oracle.canonical(cat), want)
+
+
+def test_router_rejects_bad_input():
+    lib = sjdist.LibRouter()
+    dp = torch.tensor([[0.0, 1.0], [float("inf"), 2.0]], dtype=torch.float64, device=DEV)
+    with pytest.raises(sj.SJError):
+        lib.bounds(dp)
+    ok = torch.tensor([[0.0, 1.0], [3.0, 2.0]], dtype=torch.float64, device=DEV)
+    with pytest.raises(sj.SJError):  # a point beyond the last column
+        lib.histogram(ok, 0.0, 1.0, 2)
+    with pytest.raises(sj.SJError):  # below the origin
+        lib.histogram(ok, 1.0, 1.0, 8)
+    with pytest.raises(sj.SJError):
+        lib.columns(0.0, 1e12, 1e-6)  # >= 2^30 columns
