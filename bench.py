@@ -356,8 +356,10 @@ def main():
     torch.cuda.synchronize()
     l0 = sj.sj_kernel_launches()
     for i in range(args.steps):
+        # the flush is queued on this stream before the step's start event, and every libsj call
+        # waits for this stream first (include/sj.h, stream ordering): none of the step's GPU
+        # work can start before the flush ended or before the start event
         flush_buf.fill_(i & 0xFF)
-        torch.cuda.synchronize()  # the flush is complete before the step's start event
         evs[i][0].record(stream)
         rc, c, tot, st = step(out, cap)
         evs[i][1].record(stream)

@@ -103,10 +103,12 @@ __device__ void derive_geometry(const BBox *bb, int dim, const GeomArgs &ga) {
     }
     const double errq = __shfl_sync(0xffffffffu, q, errdim);
     GeomDev *g = ga.dev;
-    if (lane < dim) {
-        g->mins[lane] = mn;
-        g->nc[lane] = nc;
+    if (lane < SJ_MAX_DIM) {  // every entry written (the host copy reads all of them)
+        g->mins[lane] = lane < dim ? mn : 0.0;
+        g->nc[lane] = lane < dim ? nc : 1ull;
+        g->stride[lane] = 0;
     }
+    __syncwarp();
     unsigned long long ncd[SJ_MAX_DIM];  // every lane: the counts of all dimensions
 #pragma unroll
     for (int d = 0; d < SJ_MAX_DIM; ++d) ncd[d] = __shfl_sync(0xffffffffu, nc, d);
@@ -513,6 +515,10 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
                 summ += len;
             }
         }
+        // slot layout, 1-D..3-D: the cell's unused slots are cleared, so the join's fixed-size
+        // staging of a cell's first runs (flat / generic paths) never reads uninitialised memory
+        if (!FILL && runs && LPC == 1 && g.rows <= 5)
+            for (uint32_t e = out, end = (uint32_t)((r + 1) * (uint64_t)g.rows); e < end; ++e) runs[e] = make_uint2(0, 0);
         if (!FILL) {
             if (LPC == 32) {
 #pragma unroll

@@ -451,9 +451,18 @@ __device__ __forceinline__ unsigned group_sum(unsigned v) {
     return v;
 }
 
-// Home cell of one query: the balanced circulant half scan (reading c8) -- position rr
-// compares to rr+1 .. rr+floor((m-1)/2) (mod m), plus rr+m/2 when m is even and rr < m/2.
+// Home cell of one query (reading c8): position rr compares to rr+1, rr+2, ... (mod m), the
+// first home_count(m, rr) of them --
+//   * cells of <= 32 points (one WorkQueue chunk, one tile): the balanced circulant half scan,
+//     rr+1 .. rr+floor((m-1)/2) (mod m), plus rr+m/2 when m is even and rr < m/2;
+//   * larger cells (several chunks of 32 queries): the upper triangle rr+1 .. m-1, so a chunk
+//     at positions [32c, 32c+32) evaluates only the home tiles from its own on, unmasked but for
+//     the diagonal one (the circulant windows would mask half of every staged home tile).
+// Either way every in-cell pair is evaluated exactly once and the cell's mean per-point load is
+// ceil((m-1)/2) (a7's W, reading c9).
+constexpr unsigned kTriMin = 33;
 __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
+    if (m >= kTriMin) return m - 1u - rr;
     return (m - 1u) / 2u + (((m & 1u) == 0u && rr < m / 2u) ? 1u : 0u);
 }
 
@@ -693,10 +702,11 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
     return true;
 }
 
-// Evaluate one staged tile against every query of the chunk.  HOME: the tile holds home-cell
-// positions tb.. and a (query, slot) pair is inside the query's circulant half scan iff
-// (p - rr - 1) mod m < home_count(m, rr) (reading c8).
-template <int DIM, int K, int MODE, bool GCG, bool HOME>
+// Evaluate one staged tile against every query of the chunk.  HOME != 0: the tile holds
+// home-cell positions tb.. and a (query, slot) pair is inside the query's half scan (reading c8)
+// iff (p - rr - 1) mod m < home_count(m, rr) -- HOME = 1, the circulant windows of cells of
+// <= 32 points -- or iff p > rr -- HOME = 2, the upper triangle of larger cells.
+template <int DIM, int K, int MODE, bool GCG, int HOME>
 __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
                                             WarpSmem<DIM, MODE> &ws, int b, int &nbuf, unsigned long long &nhits,
                                             int lane, unsigned lt) {
@@ -735,10 +745,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             load_smem_point<DIM>(ws.qry + qi * PAD, qq);
             const unsigned oq = ws.qorig[qi];
             unsigned rr = 0, hl = 0;
-            if (HOME) {
-                rr = ws.qrr[qi];
-                hl = home_count(m, rr);
-            }
+            if (HOME) rr = ws.qrr[qi];
+            if (HOME == 1) hl = home_count(m, rr);
             unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
             const unsigned long long nh0 = nhits;
             flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.ctl);
@@ -752,10 +760,12 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             for (int s = 0; s < SPL; ++s) {
                 bool ok = qv & cv[s];
                 if (GCG) ok = ok & (co[s] != oq);  // GCG: skip (q, q)
-                if (HOME) {
+                if (HOME == 1) {
                     int d = (int)(tb + t + (unsigned)(K * s)) - (int)rr - 1;
                     if (d < 0) d += (int)m;
                     ok = ok & ((unsigned)d < hl);
+                } else if (HOME == 2) {
+                    ok = ok & (tb + t + (unsigned)(K * s) > rr);
                 }
                 emit<DIM, MODE, GCG>(close[s] & ok, oq, co[s], ws.buf, nbuf, nhits, lt, gbits, cur, a, lane);
             }
@@ -786,13 +796,16 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 oka = oka & (co != oqa);
                 okb = okb & (co != oqb);
             }
-            if (HOME) {
+            if (HOME == 1) {
                 const unsigned rra = ws.qrr[q0], rrb = ws.qrr[q1 & 31];
                 int da = dh - (int)rra, db = dh - (int)rrb;
                 if (da < 0) da += (int)m;
                 if (db < 0) db += (int)m;
                 oka = oka & ((unsigned)da < home_count(m, rra));
                 okb = okb & ((unsigned)db < home_count(m, rrb));
+            } else if (HOME == 2) {
+                oka = oka & (dh >= (int)ws.qrr[q0]);
+                okb = okb & (dh >= (int)ws.qrr[q1 & 31]);
             }
             const bool ha = ca & oka, hb = cb & okb;
             flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.ctl);
@@ -827,10 +840,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             load_smem_point<DIM>(ws.qry + qi * PAD, qq);
             const unsigned oq = ws.qorig[qi];
             unsigned rr = 0, hl = 0;
-            if (HOME) {
-                rr = ws.qrr[qi];
-                hl = home_count(m, rr);
-            }
+            if (HOME) rr = ws.qrr[qi];
+            if (HOME == 1) hl = home_count(m, rr);
             unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
             const unsigned long long nh0 = nhits;
 #pragma unroll 2
@@ -848,12 +859,15 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                     ok0 = ok0 & (tile_orig[j0 & 31] != oq);
                     ok1 = ok1 & (tile_orig[j1 & 31] != oq);
                 }
-                if (HOME) {
+                if (HOME == 1) {
                     int d0 = (int)(tb + j0) - (int)rr - 1, d1 = (int)(tb + j1) - (int)rr - 1;
                     if (d0 < 0) d0 += (int)m;
                     if (d1 < 0) d1 += (int)m;
                     ok0 = ok0 & ((unsigned)d0 < hl);
                     ok1 = ok1 & ((unsigned)d1 < hl);
+                } else if (HOME == 2) {
+                    ok0 = ok0 & (tb + j0 > rr);
+                    ok1 = ok1 & (tb + j1 > rr);
                 }
                 const bool hit0 = close0 & ok0, hit1 = close1 & ok1;
                 emit<DIM, MODE, GCG>(hit0, oq, hit0 ? tile_orig[j0 & 31] : 0u, ws.buf, nbuf, nhits, lt, gbits,
@@ -981,10 +995,11 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, MODE, GCG, false>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        tile_rounds<DIM, K, MODE, GCG, 0>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
         __syncwarp();
     }
-    // ---- home cell: balanced circulant half scan as a mask over staged home tiles
+    // ---- home cell: the half scan (reading c8) as a mask over staged home tiles; in the upper
+    // triangle of a large cell the tiles before the segment's first query hold no candidate
     auto stage_home = [&](int b, unsigned tb) {
         if (tb + (unsigned)lane < m) {
             const unsigned cidx = hb + tb + (unsigned)lane;
@@ -1000,7 +1015,14 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         }
         return;
     }
-    stage_home(0, 0);
+    unsigned tb0 = 0;
+    if (m >= kTriMin) {
+        // (re-read from shared memory: nothing of the segment's set-up stays live across the
+        // forward tiles, which would cost the 1-D..3-D kernels their 64-register budget)
+        const unsigned rmin = __reduce_min_sync(kFull, (unsigned)lane < nq ? ws.qrr[lane] : 0xFFFFFFFFu);
+        tb0 = ((rmin + 1u) / 32u) * 32u;
+    }
+    stage_home(0, tb0);
     if constexpr (SJ_HOMEWIN && !GCG && DIM <= 3 && K >= 4 && MODE != kRows && MODE != kDegree) {
         if (m <= 32u) {  // one tile: evaluate the circulant windows only
             cp_async_wait<0>();
@@ -1011,7 +1033,7 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         }
     }
     it = 0;
-    for (unsigned tb = 0; tb < m; tb += 32, ++it) {
+    for (unsigned tb = tb0; tb < m; tb += 32, ++it) {
         const bool more = tb + 32 < m;
         if (more) stage_home((it + 1) & 1, tb + 32);
         if (more)
@@ -1019,7 +1041,13 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, MODE, GCG, true>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        // (with the circulant windows of small cells evaluated above, only the triangle remains
+        // for the 1-D..3-D pair kernels; the others take either)
+        constexpr bool kOnlyTri = SJ_HOMEWIN && DIM <= 3 && K >= 4 && MODE != kRows && MODE != kDegree;
+        if (kOnlyTri || m >= kTriMin)
+            tile_rounds<DIM, K, MODE, GCG, 2>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        else
+            tile_rounds<DIM, K, MODE, GCG, 1>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
         __syncwarp();
     }
 }
