@@ -66,7 +66,9 @@ enum sj_option {
     SJ_OPT_BATCH_PAIRS = 2,    /* b_s, pairs per batch buffer; default 1e8                        */
     SJ_OPT_STREAMS = 3,        /* CUDA streams for batches, 1..8; default 3                       */
     SJ_OPT_SAMPLE_PPM = 4,     /* estimator sample of D' in parts per million; default 10000 = 1%*/
-    SJ_OPT_GRAB = 5,           /* WorkQueue chunks one warp dequeues per atomic (1..1024); default 1     */
+    SJ_OPT_GRAB = 5,           /* WorkQueue chunks one warp dequeues per atomic (1..1024); default 4 for
+                                  1-D..3-D (one same-address atomic per chunk congests its L2 slice,
+                                  measured), 1 for 4-D+ (heavy chunks: balance at the queue's end)   */
     SJ_OPT_COUNT_CALCS = 6,    /* 1 = instrument the join with a distance-calculation counter; default 0 */
     SJ_OPT_BLOCKS_PER_SM = 7,  /* persistent-grid CTAs per SM; 0 = occupancy maximum (default)           */
     SJ_OPT_FAST_PATH = 8,      /* 1 = device output written in place when it fits (default); 0 = always
@@ -77,7 +79,7 @@ enum sj_option {
                                   chunk at its own offset -- no estimator, no overflow retries, and the
                                   output ORDER is deterministic.  0 = the paper's 1% estimator (P:71,
                                   P:200) with atomic placement (default)                                 */
-    SJ_OPT_QUEUE = 10          /* 1 = WorkQueue: warps dequeue D' chunks with an atomic
+    SJ_OPT_QUEUE = 10,         /* 1 = WorkQueue: warps dequeue D' chunks with an atomic
                                   counter, batches are contiguous ranges of D', the estimator samples
                                   the first 1% of D' (default).  0 = SortByWL only
                                   (P:187-192): warp w statically takes chunks w, w + #warps, ... of D'
@@ -85,6 +87,12 @@ enum sj_option {
                                   v mod nbBatches = l} (Fig. 1) and the estimator samples
                                   every (1/1%)-th chunk of the whole queue.  The pair set is
                                   the same either way                                                    */
+    SJ_OPT_OUT_BLOCKS = 11     /* in-place output allocation: 0 = one atomic on the output counter per
+                                  warp flush; 1 = blocks of 4096 pairs per warp (one atomic per block),
+                                  the gaps the warps' last blocks leave closed by a compaction pass;
+                                  2 = blocks when the caller's buffer holds >= 1e9 pairs (default): a
+                                  single counter taking every flush of a large result congests its L2
+                                  slice and doubles the join (measured)                  */
 };
 
 /* Cell access patterns (sj_create_ex).  The paper's variants, Table II:

@@ -17,7 +17,7 @@ SJ_ORDER_WORKLOAD, SJ_ORDER_CELL, SJ_ORDER_INPUT = 0, 1, 2
 PATTERNS = {"lid_unicomp": SJ_PATTERN_LID_UNICOMP, "gcg": SJ_PATTERN_GCG, "unicomp": SJ_PATTERN_UNICOMP}
 ORDERS = {"workload": SJ_ORDER_WORKLOAD, "cell": SJ_ORDER_CELL, "input": SJ_ORDER_INPUT}
 (SJ_OPT_K, SJ_OPT_BATCH_PAIRS, SJ_OPT_STREAMS, SJ_OPT_SAMPLE_PPM, SJ_OPT_GRAB, SJ_OPT_COUNT_CALCS,
- SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH, SJ_OPT_EXACT, SJ_OPT_QUEUE) = range(1, 11)
+ SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH, SJ_OPT_EXACT, SJ_OPT_QUEUE, SJ_OPT_OUT_BLOCKS) = range(1, 12)
 _NAMES = {0: "SJ_OK", 1: "SJ_MORE", -1: "SJ_EINVAL", -2: "SJ_ENOMEM", -3: "SJ_ECUDA", -4: "SJ_EGRID",
           -5: "SJ_ESTATE"}
 
@@ -377,7 +377,7 @@ class Handle:
     _OPTS = {"k": SJ_OPT_K, "batch_pairs": SJ_OPT_BATCH_PAIRS, "streams": SJ_OPT_STREAMS,
              "sample_ppm": SJ_OPT_SAMPLE_PPM, "grab": SJ_OPT_GRAB, "count_calcs": SJ_OPT_COUNT_CALCS,
              "blocks_per_sm": SJ_OPT_BLOCKS_PER_SM, "fast_path": SJ_OPT_FAST_PATH, "exact": SJ_OPT_EXACT,
-             "queue": SJ_OPT_QUEUE}
+             "queue": SJ_OPT_QUEUE, "out_blocks": SJ_OPT_OUT_BLOCKS}
 
     def set_option(self, name, value) -> None:
         sj_set_option(self.h, self._OPTS[name] if isinstance(name, str) else name, int(value))

@@ -515,10 +515,12 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
                 summ += len;
             }
         }
-        // slot layout, 1-D..3-D: the cell's unused slots are cleared, so the join's fixed-size
-        // staging of a cell's first runs (flat / generic paths) never reads uninitialised memory
-        if (!FILL && runs && LPC == 1 && g.rows <= 5)
-            for (uint32_t e = out, end = (uint32_t)((r + 1) * (uint64_t)g.rows); e < end; ++e) runs[e] = make_uint2(0, 0);
+        // slot layout: the cell's unused slots among its first five are cleared, so the join's
+        // fixed-size staging of a cell's first runs (flat / generic paths, 1-D..3-D) never reads
+        // uninitialised memory
+        if (!FILL && runs && LPC == 1)
+            for (uint32_t e = out, end = (uint32_t)(r * (uint64_t)g.rows) + (uint32_t)min(g.rows, 5); e < end; ++e)
+                runs[e] = make_uint2(0, 0);
         if (!FILL) {
             if (LPC == 32) {
 #pragma unroll
@@ -598,6 +600,11 @@ __global__ void __launch_bounds__(kThreads) wl_keys_kernel(const uint32_t *wload
     if (r >= M) return;
     keys[r] = (idx && idx[cell_start[r]] >= nq) ? max_w + 1u : max_w - wload[r];
     vals[r] = (uint32_t)r;
+}
+
+// Empty chunks after the last one (kChunkPad): chunks[C + 1 + t] = the end of the queries.
+__global__ void __launch_bounds__(kThreads) chunk_pad_kernel(uint32_t *chunks, const uint32_t *d_nc, uint32_t end) {
+    chunks[*d_nc + 1u + blockIdx.x * kThreads + threadIdx.x] = end;
 }
 
 __global__ void __launch_bounds__(kThreads) queue_m_kernel(const uint32_t *qorder, const uint32_t *cell_start,
@@ -1324,7 +1331,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
 
     // ---- WorkQueue chunks over D'
     uint32_t *d_nc = ix.d_meta;
-    SJ_TRY(dev_alloc_t(&ix.chunks, n + 1, s));
+    SJ_TRY(dev_alloc_t(&ix.chunks, n + 1 + kChunkPad, s));
     // in input order a cell's points are scattered: no chunk may claim a cell
     const uint32_t big_min = ix.order == SJ_ORDER_INPUT ? 0xFFFFFFFFu : kBigCell;
     if (ix.order == SJ_ORDER_INPUT)
@@ -1333,6 +1340,9 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     else
         SJ_TRY(scan_fused(M, CellChunkLoad{ix.cellq, qb, big_min}, CellChunkStore{ix.cellq, qb, big_min, ix.chunks}, s,
                           ChunkDone{nq, ix.chunks, d_nc}, &tmp.ws));
+    chunk_pad_kernel<<<kChunkPad / kThreads, kThreads, 0, s>>>(ix.chunks, d_nc,
+                                                                ix.order == SJ_ORDER_INPUT ? (uint32_t)n : (uint32_t)nq);
+    note_launch();
     if (side) {
         SJ_CUDA_TRY(cudaStreamWaitEvent(s, side->eq, 0));  // points, ids and D' complete
         // the caller's points are read by the gather last: done before sj_create returns

@@ -49,6 +49,7 @@ KernelInfo join_pick<SJ_JOIN_DIM>(int mode, bool gcg, int k) {
     switch (mode) {
         case kCount: return gcg ? pick_k<D, kCount, true>(k) : pick_k<D, kCount, false>(k);
         case kPairs: return gcg ? pick_k<D, kPairs, true>(k) : pick_k<D, kPairs, false>(k);
+        case kPairsB: return gcg ? KernelInfo() : pick_k<D, kPairsB, false>(k);
         case kChunkCount: return gcg ? pick_k<D, kChunkCount, true>(k) : pick_k<D, kChunkCount, false>(k);
         case kExact: return gcg ? pick_k<D, kExact, true>(k) : pick_k<D, kExact, false>(k);
         case kRows: return gcg ? pick_k<D, kRows, true>(k) : KernelInfo();

@@ -78,7 +78,9 @@ struct PointPad {
 // are modes of their own so the default kernels carry none of their code.
 template <int MODE>
 struct Mode {
-    static constexpr bool pairs = MODE == kPairs || MODE == kExact;  // emits the pair list
+    static constexpr bool pairs = MODE == kPairs || MODE == kExact || MODE == kPairsB;  // emits the pair list
+    static constexpr bool inplace = MODE == kPairs || MODE == kPairsB;  // overflow stop, fused estimator
+    static constexpr bool blocked = MODE == kPairsB;                    // blocked output (JoinArgs::blk)
     static constexpr bool exact = MODE == kExact;                     // ... at chunk offsets
 };
 
@@ -126,6 +128,7 @@ struct WarpCtl {
     unsigned sclosed;
     unsigned long long sv1;  // end of the fused estimator's sample (virtual chunks [0, sv1))
     unsigned vcount;         // the batch's virtual chunks (in shared memory: no register in the loops)
+    unsigned long long ocur, oend;  // the warp's output block (blocked kPairs launches): [ocur, oend) free
 };
 
 template <int DIM, int MODE>
@@ -254,23 +257,51 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
 // (half patterns), or the single pair {q, c} (GCG, which meets every pair twice).
 // Exact sizing (kExact): the slots come from the chunk's own cursor instead, so the output
 // order is deterministic; the counter still totals the pairs.
-template <bool GCG, bool EXACT>
-__device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs &a, int lane,
-                                      WarpCtl *wc) {
+// Flush a warp's staged hits and return how many stay buffered (0, or the rest of a flush that
+// filled its output block).  The lanes write coalesced streaming stores: both mirrored pairs of a
+// hit as one 16-B store {q, c, c, q} (half patterns), or the single pair {q, c} (GCG, which
+// meets every pair twice).  The output slots:
+//   * default: ONE atomicAdd on the output counter per flush;
+//   * blocked output (JoinArgs::blk, half patterns, kPairs): from the CTA's current block, under
+//     the CTA's lock; a block is taken with ONE atomicAdd of blk per block and CTA.  A flush that
+//     does not fit in its block's rest fills the rest and keeps the other hits buffered (moved to
+//     the buffer's front) for the next flush, which starts a new block -- so every block but each
+//     CTA's last is full and the one write loop stays a single contiguous segment;
+//   * exact sizing (kExact): the chunk's own cursor, so the output order is deterministic; the
+//     counter still totals the pairs.
+// Positions from cap_e = out_cap & ~1 on go to the scratch buffer of a blocked launch
+// (compact_output moves them back), past it they are dropped and the warp stops (overflow).
+template <bool GCG, bool EXACT, bool BLOCKED>
+__device__ __forceinline__ int flush(uint2 *buf, int nbuf, const JoinArgs &a, int lane, WarpCtl *wc) {
     __syncwarp();
     constexpr unsigned long long kPer = GCG ? 1ull : 2ull;  // pairs per buffered hit
     unsigned long long base = 0;
+    unsigned take = (unsigned)nbuf;  // hits written by this flush
     if (lane == 0) {
-        base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)nbuf);
-        wc->wtot += (unsigned long long)nbuf;
+        if (BLOCKED && !GCG && !EXACT) {
+            // the warp's own output block (no lock): a new one (ONE atomicAdd of blk) when full
+            unsigned long long c = wc->ocur, e = wc->oend;
+            if (c == e) {
+                c = atomicAdd(a.emit_ctr, a.blk);
+                e = c + a.blk;
+                wc->oend = e;
+            }
+            take = min((unsigned)nbuf, (unsigned)((e - c) >> 1));
+            wc->ocur = c + 2ull * take;
+            base = c;
+        } else {
+            base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)nbuf);
+        }
+        wc->wtot += (unsigned long long)take;
         if (EXACT) {
             base = wc->wcur;
             wc->wcur = base + kPer * (unsigned long long)nbuf;
-        } else if (base + kPer * (unsigned long long)nbuf > a.out_cap) {
+        } else if (base + kPer * (unsigned long long)take > (a.out_cap & ~1ull) + a.scratch_cap) {
             wc->wcur = 1;  // overflow: stop dequeuing
         }
     }
     base = __shfl_sync(kFull, base, 0);
+    take = __shfl_sync(kFull, take, 0);
     uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
     if constexpr (GCG) {
         const bool fits = base + (unsigned long long)nbuf <= a.out_cap;
@@ -278,24 +309,37 @@ __device__ __forceinline__ void flush(const uint2 *buf, int nbuf, const JoinArgs
             if (fits || base + (unsigned long long)k < a.out_cap) __stcs(out2 + base + k, buf[k]);
     } else {
         uint4 *out4 = reinterpret_cast<uint4 *>(a.out) + (base >> 1);  // base is even
-        if (base + 2ull * (unsigned long long)nbuf <= a.out_cap) {
+        if (base + 2ull * (unsigned long long)take <= a.out_cap) {
 #pragma unroll 4
-            for (int k = lane; k < nbuf; k += 32) {
+            for (int k = lane; k < (int)take; k += 32) {
                 const uint2 v = buf[k];  // {orig q, orig c}
                 __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));  // (q,c) and (c,q)
             }
-        } else {  // overflow: keep what fits, the counter still reports the total
-            for (int k = lane; k < nbuf; k += 32) {
-                const unsigned long long slot = base + 2ull * (unsigned long long)k;
+        } else {  // past the buffer: the scratch of a blocked launch, else dropped (overflow)
+            const unsigned long long cap_e = a.out_cap & ~1ull;
+            for (int k = lane; k < (int)take; k += 32) {
+                const unsigned long long pos = base + 2ull * (unsigned long long)k;
                 const uint2 v = buf[k];
-                if (slot + 2 <= a.out_cap)
+                if (pos < cap_e)
                     __stcs(out4 + k, make_uint4(v.x, v.y, v.y, v.x));
-                else if (slot < a.out_cap)
-                    __stcs(out2 + slot, make_uint2(v.x, v.y));
+                else if (pos - cap_e < a.scratch_cap)
+                    __stcs(reinterpret_cast<uint4 *>(a.scratch) + ((pos - cap_e) >> 1), make_uint4(v.x, v.y, v.y, v.x));
             }
+        }
+        if (take < (unsigned)nbuf) {  // the rest to the buffer's front (forward copy: safe)
+            const unsigned rest = (unsigned)nbuf - take;
+            for (unsigned k0 = 0; k0 < rest; k0 += 32) {
+                const unsigned k = k0 + (unsigned)lane;
+                const uint2 v = k < rest ? buf[take + k] : make_uint2(0, 0);
+                __syncwarp();
+                if (k < rest) buf[k] = v;
+                __syncwarp();
+            }
+            return (int)rest;
         }
     }
     __syncwarp();
+    return 0;
 }
 
 // 1-D..3-D pair modes: COLUMN buffers.  Lane l appends its own hits to column l of the warp's
@@ -421,10 +465,31 @@ __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const 
         const unsigned lim = col_base(buf, lane) + 8u * kColPitch * (unsigned)(kColRows - room / 32);
         if (__any_sync(kFull, (unsigned)nbuf > lim)) flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
     } else if constexpr (Mode<MODE>::pairs) {
-        if (nbuf > CAP - room) {
-            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
-            nbuf = 0;
-        }
+        while (nbuf > CAP - room) nbuf = flush<GCG, Mode<MODE>::exact, Mode<MODE>::blocked>(buf, nbuf, a, lane, wc);
+    }
+}
+
+// Would a round adding up to `room` hits overflow the warp's buffer?  The tiled rounds return to
+// their caller to flush (flush_now): the hot loop's registers are dead there, and the flush's
+// own (the output reservation) do not add to them.
+template <int DIM, int MODE>
+__device__ __forceinline__ bool needs_flush(const uint2 *buf, int nbuf, int room, int lane) {
+    constexpr int CAP = BufCap<DIM>::value;
+    if constexpr (Cols<DIM, MODE>::value) {
+        const unsigned lim = col_base(buf, lane) + 8u * kColPitch * (unsigned)(kColRows - room / 32);
+        return __any_sync(kFull, (unsigned)nbuf > lim);
+    } else if constexpr (Mode<MODE>::pairs) {
+        return nbuf > CAP - room;
+    } else {
+        return false;
+    }
+}
+template <int DIM, int MODE, bool GCG>
+__device__ __forceinline__ void flush_now(uint2 *buf, int &nbuf, const JoinArgs &a, int lane, WarpCtl *wc) {
+    if constexpr (Cols<DIM, MODE>::value) {
+        flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
+    } else if constexpr (Mode<MODE>::pairs) {
+        nbuf = flush<GCG, Mode<MODE>::exact, Mode<MODE>::blocked>(buf, nbuf, a, lane, wc);
     }
 }
 
@@ -436,10 +501,7 @@ __device__ __forceinline__ void flush_all(uint2 *buf, int &nbuf, const JoinArgs 
         if (__any_sync(kFull, (unsigned)nbuf != col_base(buf, lane)))
             flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
     } else if constexpr (Mode<MODE>::pairs) {
-        if (nbuf > 0) {
-            flush<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
-            nbuf = 0;
-        }
+        while (nbuf > 0) nbuf = flush<GCG, Mode<MODE>::exact, Mode<MODE>::blocked>(buf, nbuf, a, lane, wc);
     }
 }
 
@@ -472,7 +534,7 @@ __device__ __forceinline__ unsigned home_count(unsigned m, unsigned rr) {
 template <int DIM, int K, int MODE, bool GCG>
 __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
                                               WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
-                                              unsigned long long &ncalcs, int lane, unsigned lt) {
+                                              unsigned &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     const int grp = lane / K;
@@ -614,7 +676,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
                                            WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
-                                           unsigned long long &ncalcs, int lane, unsigned lt) {
+                                           unsigned &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int FRS = Flat<DIM, MODE, GCG>::runs;
     constexpr int SR = StagedRuns<DIM>::value;
@@ -707,9 +769,9 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
 // iff (p - rr - 1) mod m < home_count(m, rr) -- HOME = 1, the circulant windows of cells of
 // <= 32 points -- or iff p > rr -- HOME = 2, the upper triangle of larger cells.
 template <int DIM, int K, int MODE, bool GCG, int HOME>
-__device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
-                                            WarpSmem<DIM, MODE> &ws, int b, int &nbuf, unsigned long long &nhits,
-                                            int lane, unsigned lt) {
+__device__ __forceinline__ unsigned tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
+                                                WarpSmem<DIM, MODE> &ws, int b, int &nbuf, unsigned long long &nhits,
+                                                int lane, unsigned lt, unsigned r_start) {
     const double *tile = ws.tile[b];
     const unsigned *tile_orig = ws.tile_orig[b];
     constexpr int PAD = PointPad<DIM>::value;
@@ -738,7 +800,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             load_smem_point<DIM>(tile + (j & 31) * PAD, cp[s]);
             co[s] = tile_orig[j & 31];
         }
-        for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+        for (unsigned r0 = r_start; r0 < nq; r0 += QPW) {
+            if (needs_flush<DIM, MODE>(ws.buf, nbuf, 32 * SPL, lane)) return r0;  // the caller flushes
             const unsigned qi = (r0 + grp) & 31;
             const bool qv = r0 + grp < nq;
             double qq[DIM];
@@ -749,7 +812,6 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             if (HOME == 1) hl = home_count(m, rr);
             unsigned long long cur = MODE == kRows ? ws.qcur[qi] : 0ull;
             const unsigned long long nh0 = nhits;
-            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * SPL, a, lane, &ws.ctl);
             // all SPL distances first (independent FP64 chains -> ILP), then the emissions;
             // evaluated unconditionally and masked after (invalid slots may hold stale or
             // uninitialised bits; FP64 arithmetic on them cannot trap)
@@ -782,7 +844,8 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
         load_smem_point<DIM>(tile + lane * PAD, cp);
         const unsigned co = tile_orig[lane];
         int dh = (int)(tb + (unsigned)lane) - 1;  // HOME: slot position - 1, minus rr below
-        for (unsigned q0 = 0; q0 < nq; q0 += 2) {
+        for (unsigned q0 = r_start; q0 < nq; q0 += 2) {
+            if (needs_flush<DIM, MODE>(ws.buf, nbuf, 64, lane)) return q0;  // the caller flushes
             const unsigned q1 = q0 + 1;
             const bool v1 = q1 < nq;
             double qa[DIM], qb[DIM];
@@ -808,7 +871,6 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
                 okb = okb & (dh >= (int)ws.qrr[q1 & 31]);
             }
             const bool ha = ca & oka, hb = cb & okb;
-            flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.ctl);
             unsigned long long cura = 0, curb = 0;
             if constexpr (MODE == kRows) {
                 cura = ws.qcur[q0];
@@ -833,7 +895,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             }
         }
     } else {  // tile slots read from shared memory each step (low dimensions, k < 8)
-        for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+        for (unsigned r0 = r_start; r0 < nq; r0 += QPW) {
             const unsigned qi = (r0 + grp) & 31;
             const bool qv = r0 + grp < nq;
             double qq[DIM];
@@ -878,6 +940,7 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
             round_end(qi, qv, cur, nh0);
         }
     }
+    return nq;
 }
 
 #ifndef SJ_HOMEWIN
@@ -888,8 +951,10 @@ __device__ __forceinline__ void tile_rounds(const JoinArgs &a, unsigned nq, unsi
 // a group evaluates only the query's circulant window (reading c8): window offsets i = t,
 // t+k, ... < home_count(m, rr) <= 16, slot (rr + 1 + i) mod m read from shared memory.
 template <int DIM, int K, int MODE, bool GCG>
-__device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned nq, unsigned m, WarpSmem<DIM, MODE> &ws,
-                                                   int b, int &nbuf, unsigned long long &nhits, int lane, unsigned lt) {
+__device__ __forceinline__ unsigned home_window_rounds(const JoinArgs &a, unsigned nq, unsigned m,
+                                                       WarpSmem<DIM, MODE> &ws, int b, int &nbuf,
+                                                       unsigned long long &nhits, int lane, unsigned lt,
+                                                       unsigned r_start) {
     constexpr int PAD = PointPad<DIM>::value;
     constexpr int QPW = 32 / K;
     constexpr int WS = (16 + K - 1) / K;  // window slots per lane
@@ -898,7 +963,8 @@ __device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned n
     const int grp = lane / K;
     const unsigned t = (unsigned)(lane % K);
     const unsigned gbits = K == 32 ? kFull : (((1u << K) - 1u) << (lane & ~(K - 1)));
-    for (unsigned r0 = 0; r0 < nq; r0 += QPW) {
+    for (unsigned r0 = r_start; r0 < nq; r0 += QPW) {
+        if (needs_flush<DIM, MODE>(ws.buf, nbuf, 32 * WS, lane)) return r0;  // the caller flushes
         const unsigned qi = (r0 + grp) & 31;
         const bool qv = r0 + grp < nq;
         double qq[DIM];
@@ -907,7 +973,6 @@ __device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned n
         const unsigned rr = ws.qrr[qi];
         const unsigned hl = home_count(m, rr);
         unsigned long long cur = 0;
-        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * WS, a, lane, &ws.ctl);
         double cp[WS][DIM];
         unsigned co[WS];
         bool ok[WS], close[WS];
@@ -927,6 +992,7 @@ __device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned n
         for (int s = 0; s < WS; ++s)
             emit<DIM, MODE, GCG>(close[s] & ok[s], oq, co[s], ws.buf, nbuf, nhits, lt, gbits, cur, a, lane);
     }
+    return nq;
 }
 
 // Tiled path: all nq queries of the chunk lie in one cell (hb, m, runs rb.., S forward
@@ -937,7 +1003,7 @@ __device__ __forceinline__ void home_window_rounds(const JoinArgs &a, unsigned n
 template <int DIM, int K, int MODE, bool GCG>
 __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsigned nq, uint2 qm_lane, uint4 ci,
                                             WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
-                                            unsigned long long &ncalcs, int lane, unsigned lt) {
+                                            unsigned &ncalcs, int lane, unsigned lt) {
     constexpr int PAD = PointPad<DIM>::value;
     const unsigned hb = ci.x, m = ci.y, S = ci.w;
     __syncwarp();
@@ -951,7 +1017,7 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         const unsigned rr = qm_lane.x - hb;
         ws.qrr[slot] = rr;
         // this query's distance calculations
-        ncalcs += GCG ? (unsigned long long)S - 1 : (unsigned long long)S + home_count(m, rr);
+        ncalcs += GCG ? S - 1u : S + home_count(m, rr);
     }
     // ---- forward runs (LID-UNICOMP): tiles staged with cp.async, double-buffered, so the
     // next tile's global loads overlap this tile's distance calculations
@@ -995,7 +1061,10 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
-        tile_rounds<DIM, K, MODE, GCG, 0>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        for (unsigned r = 0; r < nq;) {  // (the rounds return to flush the buffer)
+            r = tile_rounds<DIM, K, MODE, GCG, 0>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt, r);
+            if (r < nq) flush_now<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
+        }
         __syncwarp();
     }
     // ---- home cell: the half scan (reading c8) as a mask over staged home tiles; in the upper
@@ -1027,7 +1096,10 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         if (m <= 32u) {  // one tile: evaluate the circulant windows only
             cp_async_wait<0>();
             __syncwarp();
-            home_window_rounds<DIM, K, MODE, GCG>(a, nq, m, ws, 0, nbuf, nhits, lane, lt);
+            for (unsigned r = 0; r < nq;) {  // (the rounds return to flush the buffer)
+                r = home_window_rounds<DIM, K, MODE, GCG>(a, nq, m, ws, 0, nbuf, nhits, lane, lt, r);
+                if (r < nq) flush_now<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
+            }
             __syncwarp();
             return;
         }
@@ -1044,16 +1116,26 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         // (with the circulant windows of small cells evaluated above, only the triangle remains
         // for the 1-D..3-D pair kernels; the others take either)
         constexpr bool kOnlyTri = SJ_HOMEWIN && DIM <= 3 && K >= 4 && MODE != kRows && MODE != kDegree;
-        if (kOnlyTri || m >= kTriMin)
-            tile_rounds<DIM, K, MODE, GCG, 2>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
-        else
-            tile_rounds<DIM, K, MODE, GCG, 1>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt);
+        for (unsigned r = 0; r < nq;) {  // (the rounds return to flush the buffer)
+            if (kOnlyTri || m >= kTriMin)
+                r = tile_rounds<DIM, K, MODE, GCG, 2>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt, r);
+            else
+                r = tile_rounds<DIM, K, MODE, GCG, 1>(a, nq, min(32u, m - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt, r);
+            if (r < nq) flush_now<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
+        }
         __syncwarp();
     }
 }
 
+// 3-D kernels are held to three resident CTAs per SM (their shared-memory limit), i.e. up to 85
+// registers: ptxas' own choice otherwise drifts between 64 with spills and 80 with small changes.
+template <int DIM>
+struct MinBlocks {
+    static constexpr int value = DIM == 3 ? 3 : 0;
+};
+
 template <int DIM, int K, int MODE, bool GCG>
-__global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
+__global__ void __launch_bounds__(kJoinThreads, MinBlocks<DIM>::value) join_kernel(const JoinArgs a) {
     static_assert(32 % K == 0, "k must divide 32");
     constexpr int QPW = 32 / K;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -1063,7 +1145,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     WarpSmem<DIM, MODE> &ws = reinterpret_cast<WarpSmem<DIM, MODE> *>(smem_raw)[warp];
     int nbuf = Cols<DIM, MODE>::value ? (int)col_base(ws.buf, lane) : 0;  // column modes: see flush_cols
     unsigned long long nhits = 0;
-    unsigned long long ncalcs = 0;
+    unsigned ncalcs = 0;  // this lane's distance calculations (instrumented runs; 32 bits per lane)
     // The batch: virtual chunks v_begin, v_begin + v_stride, ... < v_end (contiguous, or the
     // strided D'_l of the SortByWL-only batches); i indexes them.  A device-sized
     // launch reads the build's chunk count here: V = the slice's chunks (rank, world).
@@ -1077,6 +1159,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
             if (a.sample_ppm) {  // the estimator's sample: the first ceil(V * ppm / 1e6) chunks
                 sv1 = (V * a.sample_ppm + 999999ull) / 1000000ull;
                 if (sv1 < 1) sv1 = 1;
+                sv1 = (sv1 + a.grab - 1) / a.grab * a.grab;  // whole dequeues (as the host rounds)
                 if (sv1 > V) sv1 = V;
             }
         }
@@ -1084,8 +1167,9 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         ws.ctl.sv1 = sv1;
         ws.ctl.wcur = ws.ctl.wtot = ws.ctl.samp = 0;
         ws.ctl.sclosed = 0;
+        ws.ctl.ocur = ws.ctl.oend = 0;
     }
-    __syncwarp();
+
     // a kernel parameter, not a register: the dequeue compares against the constant bank (a
     // register here costs the 1-D..3-D kernels 16 registers and a quarter of their occupancy)
     const unsigned vcount = a.v_count;
@@ -1097,7 +1181,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         // kPairs: a warp whose flush found the output full stops (the caller re-runs staged).
         unsigned ib = 0;
         if (lane == 0) {
-            if (MODE == kPairs && ws.ctl.wcur) {
+            if (Mode<MODE>::inplace && ws.ctl.wcur) {
                 ib = vcount;
             } else if (a.static_q) {
                 ib = ws.snext;
@@ -1107,9 +1191,9 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
             }
             // device-sized launch (a.v_count = ~0u): the bound the prologue read (grab 1)
             if (ib >= ws.ctl.vcount) ib = 0xFFFFFFFFu;
-            // fused estimator (a9; v_begin 0, stride 1, grab 1): on the first dequeue past the
-            // sample, this warp's hits so far all came from sample chunks
-            if (MODE == kPairs && !Cols<DIM, MODE>::value && !ws.ctl.sclosed && ib >= ws.ctl.sv1) {
+            // fused estimator (a9; v_begin 0, stride 1; the sample is whole dequeues): on the
+            // first dequeue past the sample, this warp's hits so far all came from sample chunks
+            if (Mode<MODE>::inplace && !Cols<DIM, MODE>::value && !ws.ctl.sclosed && ib >= ws.ctl.sv1) {
                 ws.ctl.samp = ws.ctl.wtot + (unsigned long long)nbuf;
                 ws.ctl.sclosed = 1;
             }
@@ -1120,6 +1204,8 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
         for (unsigned i = ib; i < iend; ++i) {
             const unsigned long long v = a.v_begin + (unsigned long long)i * a.v_stride;
             const unsigned long long c = v * a.world + a.rank;  // queue slice (multi-GPU)
+            // (a device-sized launch bounds this by 0xFFFFFFFF: its last dequeue may pass the
+            // build's chunk count by < grab * world chunks, which the build pads with empty ones)
             if (c >= a.n_chunks) break;
             if constexpr (MODE == kExact) {  // exact sizing: the chunk's pairs start at voff[v]
                 if (lane == 0) ws.ctl.wcur = __ldg(a.voff + v) - a.out_base;
@@ -1177,7 +1263,7 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     }
     if constexpr (Mode<MODE>::pairs) {
         flush_all<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
-        if (MODE == kPairs && a.sample_ctr && lane == 0) {
+        if (Mode<MODE>::inplace && a.sample_ctr && lane == 0) {
             const unsigned long long sh = ws.ctl.sclosed ? ws.ctl.samp : ws.ctl.wtot;
             if (sh) atomicAdd(a.sample_ctr, (GCG ? 1ull : 2ull) * sh);
         }
@@ -1188,8 +1274,14 @@ __global__ void __launch_bounds__(kJoinThreads) join_kernel(const JoinArgs a) {
     }
     if (a.calcs) {
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) ncalcs += __shfl_xor_sync(kFull, ncalcs, o);
-        if (lane == 0 && ncalcs) atomicAdd(a.calcs, ncalcs);
+        unsigned long long c = ncalcs;
+        for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
+        if (lane == 0 && c) atomicAdd(a.calcs, c);
+    }
+    if (Mode<MODE>::blocked && lane == 0) {  // the warp's last block: its unused rest is a gap
+        const unsigned gw = blockIdx.x * (unsigned)kWarps + (unsigned)warp;
+        a.gaps[2 * gw] = ws.ctl.ocur;
+        a.gaps[2 * gw + 1] = ws.ctl.oend - ws.ctl.ocur;
     }
 }
 

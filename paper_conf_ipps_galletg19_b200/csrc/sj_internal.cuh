@@ -17,6 +17,9 @@
 // WorkQueue chunk: at most kChunk D' positions; cells with at least kBigCell points get
 // chunks of their own.
 constexpr unsigned kChunk = 32;
+// Empty WorkQueue chunks written after the last one: a device-sized join (the host does not know
+// the chunk count yet) may dequeue past it by < grab * world chunks (the runtime checks the bound)
+constexpr unsigned kChunkPad = 4096;
 constexpr unsigned kBigCell = 8;
 
 namespace sj {
@@ -217,6 +220,16 @@ struct JoinArgs {
     unsigned long long *emit_ctr; // pairs emitted (may exceed out_cap -> overflow)
     unsigned long long out_cap;   // capacity of out in pairs
     unsigned long long *calcs;    // instrumented distance calculations, or nullptr
+    // kPairs, mirrored patterns: the output space is taken in BLOCKS of blk pairs, one atomic
+    // on emit_ctr per block and CTA (the warps of a CTA share its current block), instead of
+    // one per warp flush -- a single counter taking every flush congests its L2 slice and halves
+    // the join (measured).  Each CTA's last block stays partly empty: its gap {start, length}
+    // goes to gaps[blockIdx.x] and compact_output() closes the gaps afterwards.  Positions from
+    // out_cap & ~1 on go to scratch (scratch_cap pairs).  blk = 0: one atomic per flush.
+    unsigned long long blk;
+    unsigned long long *gaps;
+    uint32_t *scratch;
+    unsigned long long scratch_cap;
     // kPairs: the batch estimator fused into the join (a9): pairs of the virtual chunks
     // [v_begin, sample_v1) are added to *sample_ctr (sample_v1 = 0: off)
     unsigned long long *sample_ctr;
@@ -238,10 +251,18 @@ struct JoinArgs {
 
 // Join kernel modes: count pairs; emit the pair list; fill CSR rows; count CSR degrees;
 // count pairs per WorkQueue chunk (exact sizing pass 1); emit at chunk offsets (pass 2).
-enum JoinMode : int { kCount = 0, kPairs = 1, kRows = 2, kDegree = 3, kChunkCount = 4, kExact = 5 };
+// kPairsB: kPairs with the blocked output (JoinArgs::blk) -- a kernel of its own, so the default
+// one carries none of its code.
+enum JoinMode : int { kCount = 0, kPairs = 1, kRows = 2, kDegree = 3, kChunkCount = 4, kExact = 5, kPairsB = 6 };
 
 // Launch the join kernel for dim/k/mode (kRows / kDegree need the GCG pattern).
 int launch_join(const JoinArgs &a, int dim, int k, int mode, int blocks, cudaStream_t s);
+// After a blocked kPairs launch (JoinArgs::blk): move the pairs past the total into the CTAs'
+// gaps so the output is [0, total) again; total -> *d_total.  ws: device workspace of
+// compact_ws_bytes(blocks) bytes.  Two launches on s, no host round trip.
+size_t compact_ws_bytes(int blocks);
+constexpr int kCompactMaxWarps = 8192;  // warps (gaps) compact_output handles
+int compact_output(const JoinArgs &a, int blocks, unsigned long long *d_total, void *ws, cudaStream_t s);
 // Max resident CTAs per SM of the join kernel configuration.
 int join_occupancy(int dim, int k, int mode, bool gcg, int *blocks_per_sm);
 constexpr int kJoinThreads = 256;

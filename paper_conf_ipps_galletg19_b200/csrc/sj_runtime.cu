@@ -151,6 +151,21 @@ using namespace sj;
 namespace {
 
 constexpr int kMaxStreams = 8;
+// Device counters of a join: [0] pairs emitted (one atomic per output flush), [kHead] the
+// WorkQueue head (one atomic per dequeue), [2] distance calculations, [4] the fused estimator's
+// sample pairs, [kHead + 2] a separate estimator's queue head.  The two hot atomics live in
+// different 128-byte lines: in one line they serialise on one L2 slice, and the join then falls
+// into a congested mode (C5: 0.95 -> 1.8 ms, C5 eps 0.2: 3.1 -> 6.1 ms, measured).
+constexpr int kHead = 16;
+constexpr int kTotal = 8;  // a blocked in-place join's pair total (compact_output)
+constexpr int kCtrWords = 24;
+// Blocked in-place output (JoinArgs::blk): pairs per CTA block.  One atomic per block and CTA
+// instead of one per warp flush; the CTAs' last blocks leave gaps that compact_output closes
+// (at most blocks * kOutBlk pairs to move, from a scratch of the same size past the buffer).
+constexpr unsigned long long kOutBlk = 4096;
+// pinned mailbox layout (uint64 words): [0, kCtrWords) counters; [48, 50) the build's tail;
+// [64 + 4 s, 64 + 4 s + 3) staged slot s's counters
+constexpr int kMailSlots = 64;
 
 struct Job {
     uint64_t v0, v1;  // virtual chunks v0, v0 + stride, ... < v1 of this handle's slice
@@ -191,7 +206,7 @@ struct sj_handle {
     uint64_t batch_pairs = 100000000ull;
     int streams = 3;
     uint32_t sample_ppm = 10000;
-    uint32_t grab = 1;
+    uint32_t grab = 4;  // WorkQueue chunks per dequeue (fewer same-address atomics, measured)
     int count_calcs = 0;
     int blocks_per_sm = 0;
     int fast_path = 1;
@@ -201,6 +216,9 @@ struct sj_handle {
 
     uint64_t *d_voff = nullptr;  // exact sizing: per-chunk pairs -> offsets, [V+1]
     uint64_t voff_cap = 0;
+    char *outws = nullptr;       // blocked in-place output: gaps, compaction workspace, scratch
+    size_t outws_bytes = 0;
+    int out_blocks = 2;          // SJ_OPT_OUT_BLOCKS
 
     unsigned long long *d_ctr = nullptr;  // [0]=emit [1]=head [2]=calcs [3..] spare
     uint64_t *mail = nullptr;             // pinned host mailbox [64]
@@ -294,7 +312,7 @@ int handle_init_common(sj_handle *h) {
     SJ_CUDA_TRY(cudaEventCreateWithFlags(&h->side.ej, cudaEventDisableTiming));
     h->mail = static_cast<uint64_t *>(pinned_acquire());
     if (!h->mail) return SJ_ENOMEM;
-    SJ_TRY(dev_alloc_t(&h->d_ctr, 8, h->s_main));
+    SJ_TRY(dev_alloc_t(&h->d_ctr, kCtrWords, h->s_main));
     return SJ_OK;
 }
 
@@ -340,7 +358,7 @@ int slot_init(sj_handle *h, int i) {
     SJ_CUDA_TRY(cudaEventCreate(&s.ev_start));
     SJ_CUDA_TRY(cudaEventCreate(&s.ev_stop));
     SJ_CUDA_TRY(cudaEventCreateWithFlags(&s.ev_done, cudaEventDisableTiming));
-    SJ_TRY(dev_alloc_t(&s.d_ctr, 4, s.stream));
+    SJ_TRY(dev_alloc_t(&s.d_ctr, kCtrWords, s.stream));
     return SJ_OK;
 }
 
@@ -478,9 +496,9 @@ int join_blocks(const sj_handle *h, int mode, int *blocks) {
 int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *ms, uint64_t *vcount = nullptr,
                 uint64_t stride = 1) {
     cudaStream_t s = h->s_main;
-    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
     JoinArgs a = base_args(h);
-    a.head = h->d_ctr + 1;  // zeroed above
+    a.head = h->d_ctr + kHead;  // zeroed above
     a.v_begin = v0;
     a.v_end = v1;
     a.v_stride = (uint32_t)stride;
@@ -496,7 +514,7 @@ int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *
     if (v1 > v0) SJ_TRY(launch_join(a, h->ix.dim, h->k, mode, blocks, s));
     if (vcount) SJ_TRY(scan_exclusive_u64(vcount + v0, vcount + v0, v1 - v0, vcount + v1, s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, kCtrWords * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
     *pairs = h->mail[0];
     if (h->count_calcs) h->st.calcs_measured = h->mail[2];
@@ -508,9 +526,9 @@ int count_range(sj_handle *h, uint64_t v0, uint64_t v1, uint64_t *pairs, float *
 int launch_job(sj_handle *h, Job &j, int slot_idx) {
     Slot &s = h->slots[slot_idx];
     SJ_TRY(slot_buffer(h, s, j.expect != UINT64_MAX ? std::max<uint64_t>(h->batch_pairs, j.expect) : h->batch_pairs));
-    SJ_CUDA_TRY(cudaMemsetAsync(s.d_ctr, 0, 4 * sizeof(unsigned long long), s.stream));
+    SJ_CUDA_TRY(cudaMemsetAsync(s.d_ctr, 0, kCtrWords * sizeof(unsigned long long), s.stream));
     JoinArgs a = base_args(h);
-    a.head = s.d_ctr + 1;  // zeroed above
+    a.head = s.d_ctr + kHead;  // zeroed above
     a.v_begin = j.v0;
     a.v_end = j.v1;
     a.v_stride = (uint32_t)j.stride;
@@ -528,7 +546,7 @@ int launch_job(sj_handle *h, Job &j, int slot_idx) {
     SJ_CUDA_TRY(cudaEventRecord(s.ev_start, s.stream));
     SJ_TRY(launch_join(a, h->ix.dim, h->k, exact ? kExact : kPairs, blocks, s.stream));
     SJ_CUDA_TRY(cudaEventRecord(s.ev_stop, s.stream));
-    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail + 8 + 4 * slot_idx, s.d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost,
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail + kMailSlots + 4 * slot_idx, s.d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost,
                                 s.stream));
     SJ_CUDA_TRY(cudaEventRecord(s.ev_done, s.stream));
     j.slot = slot_idx;
@@ -568,7 +586,7 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
         Slot &s = h->slots[j.slot];
         if (!j.complete) {
             SJ_CUDA_TRY(cudaEventSynchronize(s.ev_done));
-            const uint64_t *m = h->mail + 8 + 4 * j.slot;
+            const uint64_t *m = h->mail + kMailSlots + 4 * j.slot;
             j.cnt = m[0];
             if (h->count_calcs) h->st.calcs_measured += m[2];
             float ms = 0;
@@ -658,9 +676,9 @@ int continue_staged(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) 
 int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_t v1, bool exact,
                  uint64_t *emitted) {
     cudaStream_t s = h->s_main;
-    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
     JoinArgs a = base_args(h);
-    a.head = h->d_ctr + 1;  // zeroed above
+    a.head = h->d_ctr + kHead;  // zeroed above
     a.v_begin = v0;
     a.v_end = v1;
     a.out = out;
@@ -677,7 +695,7 @@ int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_
     SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
     if (v1 > v0) SJ_TRY(launch_join(a, h->ix.dim, h->k, mode, blocks, s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, kCtrWords * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
     float ms = 0;
     SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_c, h->ev_d));
@@ -703,15 +721,48 @@ int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_
 // 3 ms on C5 eps=0.2, where estimator and join fight over the same heaviest head of D'.)
 // *spairs = the sample's pairs, *total = all pairs emitted (> cap: overflow, only the first
 // cap were written).
+// Blocked output for an in-place kPairs launch of `blocks` CTAs (JoinArgs::blk, mode kPairsB):
+// the gaps array, the compaction workspace and the scratch, from one per-handle allocation.  Half
+// patterns only (GCG emits single pairs).  SJ_OPT_OUT_BLOCKS: 1 on, 0 off, 2 (default) on when
+// the caller's buffer holds at least kBlockedMinCap pairs (a large result: the output counter's
+// congestion doubles the join, measured on C5 eps 0.2; below it the compaction's fixed cost
+// outweighs it).
+constexpr uint64_t kBlockedMinCap = 1000000000ull;
+int blocked_out(sj_handle *h, JoinArgs &a, int blocks, uint64_t cap, bool *on) {
+    *on = h->out_blocks == 1 || (h->out_blocks == 2 && cap >= kBlockedMinCap);
+    *on = *on && h->ix.pattern != SJ_PATTERN_GCG && blocks * (kJoinThreads / 32) <= kCompactMaxWarps;
+    if (!*on) return SJ_OK;
+    const size_t gbytes = ((size_t)blocks * kJoinThreads / 32 * 16 + 255) & ~(size_t)255;  // a gap per warp
+    const size_t wbytes = (compact_ws_bytes(blocks) + 255) & ~(size_t)255;
+    const size_t sbytes = (size_t)blocks * kJoinThreads / 32 * kOutBlk * 8;
+    const size_t need = gbytes + wbytes + sbytes;
+    if (h->outws_bytes < need) {
+        dev_free(h->outws, h->s_main);
+        h->outws = nullptr;
+        h->outws_bytes = 0;
+        SJ_TRY(dev_alloc(reinterpret_cast<void **>(&h->outws), need, h->s_main));
+        h->outws_bytes = need;
+    }
+    a.blk = kOutBlk;
+    a.gaps = reinterpret_cast<unsigned long long *>(h->outws);
+    a.scratch = reinterpret_cast<uint32_t *>(h->outws + gbytes + wbytes);
+    a.scratch_cap = (unsigned long long)blocks * kJoinThreads / 32 * kOutBlk;
+    return SJ_OK;
+}
+
+void *blocked_ws(sj_handle *h, int blocks) {
+    return h->outws + (((size_t)blocks * kJoinThreads / 32 * 16 + 255) & ~(size_t)255);
+}
+
 int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, uint64_t sv1, uint64_t sstride,
                      uint64_t V, uint64_t *spairs, uint64_t *total) {
     cudaStream_t s = h->s_main;
-    const bool fused = sstride == 1 && h->queue && h->grab == 1 && sch && !getenv("SJ_SEPARATE_EST");
-    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    const bool fused = sstride == 1 && h->queue && sch && !getenv("SJ_SEPARATE_EST");
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
     if (!fused) {
         JoinArgs e = base_args(h);
-        e.head = h->d_ctr + 5;
+        e.head = h->d_ctr + kHead + 2;
         e.emit_ctr = h->d_ctr + 4;
         e.v_begin = 0;
         e.v_end = sv1;  // the sample: chunks 0, sstride, ... < sv1 (sch of them)
@@ -726,7 +777,7 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
     a.emit_ctr = h->d_ctr;
     a.out_cap = cap;
     a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
-    a.head = h->d_ctr + 1;
+    a.head = h->d_ctr + kHead;
     a.v_begin = 0;
     a.v_end = V;
     if (fused) {
@@ -735,10 +786,14 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
     }
     int blocks;
     SJ_TRY(join_blocks(h, kPairs, &blocks));
-    if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, kPairs, blocks, s));
+    bool blocked = false;
+    SJ_TRY(blocked_out(h, a, blocks, cap, &blocked));
+    if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, blocked ? kPairsB : kPairs, blocks, s));
+    if (V && blocked) SJ_TRY(compact_output(a, blocks, h->d_ctr + kTotal, blocked_ws(h, blocks), s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 5 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, kCtrWords * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    if (blocked) h->mail[0] = h->mail[kTotal];  // pairs emitted (the counter itself counts blocks)
     float ms_est = 0, ms = 0;
     SJ_CUDA_TRY(cudaEventElapsedTime(&ms_est, h->ev_c, h->ev_e));
     SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_e, h->ev_d));
@@ -749,7 +804,7 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
     h->st.est_fused = fused ? 1u : 0u;
     *spairs = h->mail[4];
     *total = h->mail[0];
-    if (fused && h->mail[1] < sv1) {  // overflowed before the sample was handed out: count it apart
+    if (fused && h->mail[kHead] < sv1) {  // overflowed before the sample was handed out: count it apart
         const uint64_t emitted = *total;
         const uint64_t calcs = h->mail[2];
         float ms_c = 0;
@@ -768,7 +823,7 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
 // into the join.  *spairs = the sample's pairs, *total = all pairs emitted.
 int run_in_place_lazy(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *spairs, uint64_t *total) {
     cudaStream_t s = h->s_main;
-    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_e, s));
     JoinArgs a = base_args(h);
     a.n_chunks = 0xFFFFFFFFu;      // bounded by the device-side V instead
@@ -780,15 +835,19 @@ int run_in_place_lazy(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *spair
     a.emit_ctr = h->d_ctr;
     a.out_cap = cap;
     a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
-    a.head = h->d_ctr + 1;
+    a.head = h->d_ctr + kHead;
     a.v_begin = 0;
     a.v_end = 0xFFFFFFFFull;  // v_count = ~0u: the kernel bounds the queue by the device-side V
     int blocks;
     SJ_TRY(join_blocks(h, kPairs, &blocks));
-    SJ_TRY(launch_join(a, h->ix.dim, h->k, kPairs, blocks, s));
+    bool blocked = false;
+    SJ_TRY(blocked_out(h, a, blocks, cap, &blocked));
+    SJ_TRY(launch_join(a, h->ix.dim, h->k, blocked ? kPairsB : kPairs, blocks, s));
+    if (blocked) SJ_TRY(compact_output(a, blocks, h->d_ctr + kTotal, blocked_ws(h, blocks), s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
-    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 5 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, kCtrWords * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
     SJ_CUDA_TRY(cudaStreamSynchronize(s));
+    if (blocked) h->mail[0] = h->mail[kTotal];  // pairs emitted (the counter itself counts blocks)
     SJ_TRY(ix_ready(h));
     float ms = 0;
     SJ_CUDA_TRY(cudaEventElapsedTime(&ms, h->ev_e, h->ev_d));
@@ -899,7 +958,8 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     const bool dev_out = out && is_device_ptr(out, h->device);
     // right after sj_create, the in-place WorkQueue join needs nothing from the build on the
     // host (run_in_place_lazy); every other path reads the build's tail first
-    const bool lazy = h->pending && dev_out && h->fast_path && !h->exact && h->queue && h->grab == 1 &&
+    const bool lazy = h->pending && dev_out && h->fast_path && !h->exact && h->queue &&
+                      (uint64_t)h->grab * (uint64_t)h->world <= kChunkPad &&
                       !getenv("SJ_DEBUG_VRANGE") && !getenv("SJ_SEPARATE_EST") &&
                       !(reinterpret_cast<uintptr_t>(out) & 15u);
     uint64_t lazy_spairs = 0, lazy_total = 0;
@@ -941,6 +1001,9 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
     // dataset"; P:200 contrasts the two)
     uint64_t sch = (nch * (uint64_t)h->sample_ppm + 999999ull) / 1000000ull;
     if (sch < 1) sch = 1;
+    // whole dequeues (a WorkQueue dequeue takes `grab` consecutive chunks): the fused estimator's
+    // sample then ends where a dequeue ends (the join kernel rounds the same way)
+    if (h->queue) sch = (sch + h->grab - 1) / h->grab * h->grab;
     if (sch > nch) sch = nch;
     uint64_t sstride = 1, sv1 = sch;
     if (!h->queue && nch) {
@@ -960,7 +1023,7 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
         if (lazy) {  // already ran; the sample is complete unless the output overflowed early
             spairs = lazy_spairs;
             total = lazy_total;
-            if (h->mail[1] < sv1) {
+            if (h->mail[kHead] < sv1) {
                 const uint64_t calcs = h->mail[2];
                 float ms_c = 0;
                 SJ_TRY(count_range(h, 0, sv1, &spairs, &ms_c));
@@ -1064,14 +1127,14 @@ int neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, 
     }
     // pass 1: degrees
     JoinArgs a = base_args(h);
-    a.head = h->d_ctr + 1;
+    a.head = h->d_ctr + kHead;
     a.emit_ctr = h->d_ctr;
     a.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
     a.v_begin = 0;
     a.v_end = V;
     a.qdeg = d_deg;
     rc = [&]() -> int {
-        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
         SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
         if (V) SJ_TRY(launch_join(a, h->ix.dim, h->k, kDegree, blocks, s));
         SJ_TRY(scan_exclusive_u32_to_u64(d_deg, d_off, n, d_off + n, s));
@@ -1117,7 +1180,7 @@ int neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, 
     }
     rc = [&]() -> int {
         JoinArgs b = base_args(h);
-        b.head = h->d_ctr + 1;
+        b.head = h->d_ctr + kHead;
         b.emit_ctr = h->d_ctr;
         b.calcs = h->count_calcs ? h->d_ctr + 2 : nullptr;
         b.v_begin = 0;
@@ -1126,11 +1189,11 @@ int neighbor_csr(sj_handle *h, uint64_t *row_off, uint32_t *nbrs, uint64_t cap, 
         b.nbrs = d_nbrs;
         int fb;
         SJ_TRY(join_blocks(h, kRows, &fb));
-        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, 8 * sizeof(unsigned long long), s));
+        SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
         SJ_CUDA_TRY(cudaEventRecord(h->ev_c, s));
         if (V) SJ_TRY(launch_join(b, h->ix.dim, h->k, kRows, fb, s));
         SJ_CUDA_TRY(cudaEventRecord(h->ev_d, s));
-        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        SJ_CUDA_TRY(cudaMemcpyAsync(h->mail, h->d_ctr, kCtrWords * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
         if (!nb_dev && tot)
             SJ_CUDA_TRY(cudaMemcpyAsync(nbrs, d_nbrs, tot * sizeof(uint32_t), cudaMemcpyDefault, s));
         SJ_CUDA_TRY(cudaStreamSynchronize(s));
@@ -1288,6 +1351,7 @@ static sj_handle *create_impl(const double *points, uint64_t n, int dim, double 
         snprintf(g_err, sizeof g_err, "%s", keep.c_str());
         return nullptr;
     }
+    if (dim >= 4) h->grab = 1;  // 4-D+: every chunk is heavy; one per dequeue keeps the end balanced
     if (sync_build) {
         fill_static_stats(h);
         h->st.ms_build = ms;
@@ -1344,6 +1408,7 @@ void sj_destroy(sj_handle *h) {
     cudaSetDevice(h->device);
     slots_release(h);
     if (h->s_main) dev_free(h->d_voff, h->s_main);
+    if (h->s_main) dev_free(h->outws, h->s_main);
     if (h->s_main && h->owns_index) free_index(h->ix, h->s_main);  // stream-ordered frees
     if (!core_release(h)) {
         if (h->s_main) {
@@ -1414,6 +1479,10 @@ int sj_set_option(sj_handle *h, int opt, int64_t v) {
         case SJ_OPT_QUEUE:
             if (v != 0 && v != 1) break;
             h->queue = (int)v;
+            return SJ_OK;
+        case SJ_OPT_OUT_BLOCKS:
+            if (v < 0 || v > 2) break;
+            h->out_blocks = (int)v;
             return SJ_OK;
 
     }
@@ -1628,6 +1697,7 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
         sj_destroy(h);
         return nullptr;
     }
+    if (ix.dim >= 4) h->grab = 1;
     fill_static_stats(h);
     return h;
 }

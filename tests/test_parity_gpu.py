@@ -268,3 +268,41 @@ def test_index_blob_roundtrip():
         assert h3.count() == want.shape[0]
 
 # (full BASELINE sizes: tests/test_fullsize_gpu.py, element by element)
+
+
+# ------------------------------------------------------------------ blocked in-place output
+
+@pytest.mark.parametrize("name,n", [("c2k64", 150_001), ("c3k64", 150_013), ("c5", 200_003), ("c4k32", 40_009)])
+@pytest.mark.parametrize("slack", [0, 1, 777_777])
+def test_blocked_output_elementwise(name, n, slack):
+    """SJ_OPT_OUT_BLOCKS=1: every warp takes output blocks of 4096 pairs (one atomic per block);
+    the warps' last blocks leave gaps that the compaction pass closes, positions past the caller's
+    buffer go to the scratch and are moved back.  Exactly sized, odd-sized (+1) and large buffers."""
+    cfg = workloads.get_config(name).scaled(n)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    p = torch.from_numpy(pts).to(DEV)
+    cap = want.shape[0] + slack
+    out = torch.full((cap, 2), -1, dtype=torch.int32, device=DEV)
+    with sj.Handle(p, cfg.eps, k=cfg.k, out_blocks=1, count_calcs=1) as h:
+        rc, c = h.self_join(out, cap)
+        st = h.stats()
+    assert rc == sj.SJ_OK and c == want.shape[0] and st["fast_path"] == 1
+    got = out[:c].cpu().numpy().view(np.uint32)
+    np.testing.assert_array_equal(canon(got), want)
+    assert st["calcs_measured"] == st["dist_calcs"]
+
+
+def test_blocked_output_overflow_falls_back():
+    cfg = workloads.get_config("c5").scaled(120_007)
+    pts = cfg.points()
+    want = oracle.grid_pairs(pts, cfg.eps)
+    p = torch.from_numpy(pts).to(DEV)
+    cap = want.shape[0] // 2 + 1
+    with sj.Handle(p, cfg.eps, k=8, out_blocks=1) as h:
+        buf = torch.empty((cap, 2), dtype=torch.int32, device=DEV)
+        parts, rc = [], sj.SJ_MORE
+        while rc == sj.SJ_MORE:
+            rc, c = h.self_join(buf, cap)
+            parts.append(buf[:c].cpu().numpy().view(np.uint32).copy())
+    np.testing.assert_array_equal(canon(np.concatenate(parts)), want)
