@@ -45,6 +45,9 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--batched-steps", type=int, default=5)
+    ap.add_argument("--mp", default="replicated", choices=["replicated", "broadcast"],
+                    help="N > 1: every rank builds the index (replicated input), or rank 0 builds and "
+                         "NCCL-broadcasts it (zero-copy views on the other ranks)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-stride", type=int, default=0, help="oracle sample: every s-th query (0 = auto)")
     ap.add_argument("--json-out", default=None)
@@ -315,10 +318,13 @@ def main():
         if world == 1:
             h = sj.Handle(d_pts, cfg.eps, k=k)
             return h
-        h = sj.Handle(d_pts, cfg.eps, k=k) if rank == 0 else None
-        h, _ = sjdist.replicate_index(h, 0, group, dev)
-        if rank != 0:
-            h.set_option("k", k)
+        if args.mp == "replicated":  # every rank builds from its own copy
+            h = sj.Handle(d_pts, cfg.eps, k=k)
+        else:  # rank 0 builds; NCCL broadcast of the index blob; zero-copy views elsewhere
+            h = sj.Handle(d_pts, cfg.eps, k=k) if rank == 0 else None
+            h, _ = sjdist.replicate_index(h, 0, group, dev)
+            if rank != 0:
+                h.set_option("k", k)
         h.set_slice(rank, world)
         return h
 
@@ -466,6 +472,9 @@ def main():
         def step_host():
             if world == 1:
                 h = sj.Handle(h_pts, cfg.eps, k=k)
+            elif args.mp == "replicated":
+                h = sj.Handle(h_pts, cfg.eps, k=k)
+                h.set_slice(rank, world)
             else:
                 h = sj.Handle(h_pts, cfg.eps, k=k) if rank == 0 else None
                 h, _ = sjdist.replicate_index(h, 0, group, dev)
@@ -521,7 +530,7 @@ def main():
             "data": "synthetic, seeded (workloads/, SURVEY.md §8.0 recipe)",
             "config": {"workload": f"{cfg.name}: {cfg.note}", "n": cfg.n, "dim": cfg.dim, "eps": cfg.eps, "k": k,
                        "pairs": tot_pairs, "dist_calcs": d_alg, "n_cells": st0["n_cells"],
-                       "fwd_runs": st0["fwd_runs"], "parallelism": f"replicas+queue slices x{world}",
+                       "fwd_runs": st0["fwd_runs"], "parallelism": f"{args.mp} index + queue slices x{world}" if world > 1 else "1 GPU",
                        "l2": "flushed before every step (256 MiB write, outside the step events)",
                        "output": "HBM-resident pairs (uint32 x2), written in place"},
             "self_join_s": total_ms / args.steps / 1e3,

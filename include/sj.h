@@ -253,6 +253,12 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes);
  * torch's current stream before every call. */
 void sj_set_stream(void *stream);
 
+/* Zero-copy variant of sj_create_from_index for a blob in device memory of the current device
+ * (256-byte aligned, e.g. the output of an NCCL broadcast): the handle's index arrays ARE the
+ * blob's -- nothing is allocated or copied -- so the caller keeps the blob alive and unchanged
+ * until sj_destroy.  The blob is validated as in sj_create_from_index.  NULL on error. */
+sj_handle *sj_create_from_index_view(const void *blob, uint64_t bytes);
+
 /* ABI version (SJ_ABI_VERSION). */
 int sj_abi_version(void);
 

@@ -15,7 +15,7 @@ from ._lib import (  # noqa: F401
     SJ_OPT_K, SJ_OPT_BATCH_PAIRS, SJ_OPT_STREAMS, SJ_OPT_SAMPLE_PPM, SJ_OPT_GRAB,
     SJ_OPT_COUNT_CALCS, SJ_OPT_BLOCKS_PER_SM, SJ_OPT_FAST_PATH, SJ_OPT_EXACT, SJ_OPT_QUEUE,
     SJError, SJStats, lib_path, header_functions,
-    sj_abi_version, sj_kernel_launches, sj_last_error, sj_create, sj_create_ex, sj_create_part, sj_create_from_index, sj_self_join, sj_destroy,
+    sj_abi_version, sj_kernel_launches, sj_last_error, sj_create, sj_create_ex, sj_create_part, sj_create_from_index, sj_create_from_index_view, sj_self_join, sj_destroy,
     sj_set_option, sj_set_slice, sj_get_stats, sj_export_index, sj_forward_offsets,
     sj_slice_chunks, sj_batch_chunks, sj_measure_fp64, sj_measure_atomics, sj_neighbor_csr, sj_set_stream,
     sj_part_bounds, sj_part_columns, sj_part_histogram, sj_part_pack,

@@ -67,6 +67,7 @@ _sig = {
     "sj_get_stats": (_int, [_vp, ctypes.POINTER(SJStats)]),
     "sj_export_index": (_int, [_vp, _vp, _u64, ctypes.POINTER(_u64)]),
     "sj_create_from_index": (_vp, [_vp, _u64]),
+    "sj_create_from_index_view": (_vp, [_vp, _u64]),
     "sj_create_part": (_vp, [_vp, _vp, _u64, _u64, _int, _dbl, _vp]),
     "sj_forward_offsets": (_int, [_int, _vp, _u64]),
     "sj_slice_chunks": (_i64, [_u64, _int, _int, _vp, _u64]),
@@ -204,6 +205,15 @@ def sj_create_part(points, ids, n_query: int, eps: float, origin) -> int:
 def sj_create_from_index(blob, nbytes: int) -> int:
     _order_after_torch()
     h = _lib.sj_create_from_index(_ptr(blob), int(nbytes))
+    if not h:
+        raise SJError(SJ_EINVAL, sj_last_error())
+    return h
+
+
+def sj_create_from_index_view(blob, nbytes: int) -> int:
+    """Zero copy: the handle's index arrays alias the (device) blob, which must outlive it."""
+    _order_after_torch()
+    h = _lib.sj_create_from_index_view(_ptr(blob), int(nbytes))
     if not h:
         raise SJError(SJ_EINVAL, sj_last_error())
     return h
@@ -371,7 +381,14 @@ class Handle:
             self.set_option(k, v)
 
     @classmethod
-    def from_index(cls, blob, nbytes: int) -> "Handle":
+    def from_index(cls, blob, nbytes: int, view: bool = False) -> "Handle":
+        """A handle from an exported index blob; view=True aliases a device blob (zero copy: the
+        blob must stay alive and unchanged while the handle exists -- the handle keeps a
+        reference to the object passed)."""
+        if view:
+            h = cls(raw=sj_create_from_index_view(blob, nbytes))
+            h._blob = blob
+            return h
         return cls(raw=sj_create_from_index(blob, nbytes))
 
     _OPTS = {"k": SJ_OPT_K, "batch_pairs": SJ_OPT_BATCH_PAIRS, "streams": SJ_OPT_STREAMS,

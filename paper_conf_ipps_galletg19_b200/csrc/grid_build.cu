@@ -218,28 +218,43 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
 // contraction flags (reading c1): c_d = floor( (x_d - min_d) / w ).
 // The geometry comes from device memory (bbox_kernel's last block); keys are 32-bit when the
 // grid has at most 2^32 cells, else 64-bit (the host picks the buffer once it reads key_bits).
-__global__ void __launch_bounds__(kThreads) cell_id_kernel(const double *raw, uint64_t n,
+// One block per radix tile (kRadixTileKeys points): it also counts the tile's low 8-bit digits,
+// the first pass of the point sort (a4) -- its histogram kernel is not launched.
+constexpr int kCellIdThreads = 1024;  // 2 points per thread: the 6-D divisions need the parallelism
+__global__ void __launch_bounds__(kCellIdThreads) cell_id_kernel(const double *raw, uint64_t n,
                                                            const GeomDev *__restrict__ gp, uint32_t *keys32,
-                                                           unsigned long long *keys64, uint32_t *vals, GeomArgs ga) {
-    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i == 0 && ga.host) publish_geometry(gp, ga);
-    if (i >= n || gp->err) return;
+                                                           unsigned long long *keys64, uint32_t *vals, GeomArgs ga,
+                                                           uint32_t *hist0, uint32_t ntiles) {
+    __shared__ uint32_t h[256];
+    if (threadIdx.x < 256) h[threadIdx.x] = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0 && ga.host) publish_geometry(gp, ga);
+    __syncthreads();
     const int dim = gp->dim;
     const double w = gp->w;
-    unsigned long long lid = 0;
+    const bool ok = !gp->err, narrow = gp->key_bits <= 32;
+    const uint64_t base = (uint64_t)blockIdx.x * kRadixTileKeys;
 #pragma unroll
-    for (int d = 0; d < SJ_MAX_DIM; ++d) {
-        if (d < dim) {
-            double q = __ddiv_rn(__dsub_rn(raw[i * dim + d], gp->mins[d]), w);
-            unsigned long long c = __double2ull_rd(q);
-            lid += c * gp->stride[d];
+    for (int it = 0; it < kRadixTileKeys / kCellIdThreads; ++it) {
+        const uint64_t i = base + (uint64_t)it * kCellIdThreads + threadIdx.x;
+        if (i >= n || !ok) continue;
+        unsigned long long lid = 0;
+#pragma unroll
+        for (int d = 0; d < SJ_MAX_DIM; ++d) {
+            if (d < dim) {
+                double q = __ddiv_rn(__dsub_rn(raw[i * dim + d], gp->mins[d]), w);
+                unsigned long long c = __double2ull_rd(q);
+                lid += c * gp->stride[d];
+            }
         }
+        if (narrow)
+            keys32[i] = (uint32_t)lid;
+        else
+            keys64[i] = lid;
+        vals[i] = (uint32_t)i;
+        atomicAdd(&h[(uint32_t)lid & 0xFFu], 1u);
     }
-    if (gp->key_bits <= 32)
-        keys32[i] = (uint32_t)lid;
-    else
-        keys64[i] = lid;
-    vals[i] = (uint32_t)i;
+    __syncthreads();
+    if (threadIdx.x < 256) hist0[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
 }
 
 // a5: run-length compaction of the sorted ids, fused into one single-pass scan:
@@ -255,10 +270,12 @@ struct RleStore {
     uint32_t *cellof;
     unsigned long long *cell_lid;
     uint32_t *cell_start;
+    uint32_t *dense;  // a6's dense lid -> cell table (pre-filled with ~0), or null (hashed lookup)
     __device__ void operator()(uint64_t p, unsigned ex, unsigned flag) const {
         if (flag) {
             cell_lid[ex] = (unsigned long long)ks[p];
             cell_start[ex] = (uint32_t)p;
+            if (dense) dense[ks[p]] = ex;
         }
         cellof[p] = flag ? ex : ex - 1;  // point (sorted position) -> cell rank
     }
@@ -299,13 +316,6 @@ __device__ __forceinline__ uint32_t lookup_cell(const Lookup &L, unsigned long l
         if (k == ~0ull) return 0xFFFFFFFFu;
         h = (h + 1) & L.hmask;
     }
-}
-
-__global__ void __launch_bounds__(kThreads) dense_fill_kernel(const unsigned long long *cell_lid, const uint64_t *d_M,
-                                                              uint32_t *dense) {
-    uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= *d_M) return;
-    dense[cell_lid[r]] = (uint32_t)r;
 }
 
 __global__ void __launch_bounds__(kThreads) hash_insert_kernel(const unsigned long long *cell_lid, const uint64_t *d_M,
@@ -926,22 +936,22 @@ struct Temps {
 
 template <class K>
 static int sort_points(Temps &tmp, K *ka, uint32_t *va, uint64_t n, int bits, cudaStream_t s, K **keys_sorted,
-                       uint32_t **idx_sorted) {
+                       uint32_t **idx_sorted, uint32_t *hist0) {
     K *kb;
     uint32_t *vb;
     SJ_TRY(tmp.alloc(&kb, n));
     SJ_TRY(tmp.alloc(&vb, n));
     if constexpr (sizeof(K) == 4)
-        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws));
+        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws, hist0));
     else
-        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws));
+        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws, hist0));
     return SJ_OK;
 }
 
 template <class K>
 static int rle(const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *cell_lid, uint32_t *cell_start,
-               uint64_t *d_M, cudaStream_t s, Workspace *ws) {  // d_M: zero-filled
-    return scan_fused(n, RleLoad<K>{ks}, RleStore<K>{ks, cellof, cell_lid, cell_start}, s,
+               uint64_t *d_M, cudaStream_t s, Workspace *ws, uint32_t *dense) {  // d_M: zero-filled
+    return scan_fused(n, RleLoad<K>{ks}, RleStore<K>{ks, cellof, cell_lid, cell_start, dense}, s,
                       RleDone{n, cell_start, d_M}, ws);
 }
 
@@ -1030,7 +1040,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&keys32, n));
     SJ_TRY(tmp.alloc(&keys64, n));
     SJ_TRY(tmp.alloc(&vals0, n));
-    cell_id_kernel<<<grid_for(n), kThreads, 0, s>>>(d_raw, n, d_geo, keys32, keys64, vals0, ga);
+    const uint32_t ntiles = (uint32_t)((n + kRadixTileKeys - 1) / kRadixTileKeys);
+    uint32_t *hist0;  // the point sort's first-pass tile histogram, counted by the cell-id kernel
+    SJ_TRY(tmp.alloc(&hist0, (uint64_t)256 * ntiles));
+    cell_id_kernel<<<ntiles, kCellIdThreads, 0, s>>>(d_raw, n, d_geo, keys32, keys64, vals0, ga, hist0, ntiles);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     if (zero_copy) {
@@ -1080,15 +1093,33 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     Lookup L{};
     const bool dense = ncells_total <= (1ull << 27) && ncells_total <= 64ull * n + 4096;
     ix.lookup_hash = dense ? 0 : 1;
+    // the dense table is cleared on the side stream while the points sort, and filled by the
+    // compaction's store (a5) -- no kernel of its own
+    uint32_t *tab = nullptr;
+    if (dense) {
+        SJ_TRY(tmp.alloc(&tab, ncells_total));
+        cudaStream_t st = side ? side->s2 : s;
+        if (side) {
+            SJ_CUDA_TRY(cudaEventRecord(side->ea, s));
+            SJ_CUDA_TRY(cudaStreamWaitEvent(st, side->ea, 0));
+        }
+        SJ_CUDA_TRY(cudaMemsetAsync(tab, 0xFF, ncells_total * sizeof(uint32_t), st));
+        if (side) {
+            SJ_CUDA_TRY(cudaEventRecord(side->eq, st));
+        }
+        L.dense = tab;
+    }
     if (ix.key_bits <= 32) {
         uint32_t *ks;
-        SJ_TRY(sort_points<uint32_t>(tmp, keys32, vals0, n, ix.key_bits, s, &ks, &idx_sorted));
-        SJ_TRY(rle<uint32_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
+        SJ_TRY(sort_points<uint32_t>(tmp, keys32, vals0, n, ix.key_bits, s, &ks, &idx_sorted, hist0));
+        if (dense && side) SJ_CUDA_TRY(cudaStreamWaitEvent(s, side->eq, 0));
+        SJ_TRY(rle<uint32_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws, tab));
     } else {
         uint64_t *ks;
         SJ_TRY(sort_points<uint64_t>(tmp, reinterpret_cast<uint64_t *>(keys64), vals0, n, ix.key_bits, s, &ks,
-                                     &idx_sorted));
-        SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws));
+                                     &idx_sorted, hist0));
+        if (dense && side) SJ_CUDA_TRY(cudaStreamWaitEvent(s, side->eq, 0));
+        SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws, tab));
     }
     // the gather of the points into cell order needs only the point sort: side stream
     SJ_TRY(dev_alloc_t(&ix.pts, n * ix.pad, s));
@@ -1102,14 +1133,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
                                                      part ? part->d_ids : nullptr);
     note_launch();
     if (side) SJ_CUDA_TRY(cudaEventRecord(side->eg, sg));
-    if (dense) {
-        uint32_t *tab;
-        SJ_TRY(tmp.alloc(&tab, ncells_total));
-        SJ_CUDA_TRY(cudaMemsetAsync(tab, 0xFF, ncells_total * sizeof(uint32_t), s));
-        dense_fill_kernel<<<grid_for(n), kThreads, 0, s>>>(cell_lid, d_M, tab);
-        note_launch();
-        L.dense = tab;
-    } else {
+    if (!dense) {
         unsigned long long cap = 1024;
         while (cap < 2 * n) cap <<= 1;
         unsigned long long *hk;

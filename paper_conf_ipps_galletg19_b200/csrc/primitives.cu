@@ -58,6 +58,7 @@ constexpr int kRadixThreads = 256;
 constexpr int kRadixWarps = kRadixThreads / 32;
 constexpr int kRadixItems = 8;  // per lane
 constexpr int kRadixTile = kRadixThreads * kRadixItems;
+static_assert(kRadixTile == kRadixTileKeys, "the cell-id kernel counts the first pass per tile of this size");
 constexpr int kRadixBins = 256;
 
 // Per-tile digit counts, digit-major: hist[d * ntiles + tile].
@@ -164,7 +165,7 @@ __global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *k
 
 template <class K>
 int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_t n, int bits, K **keys_out,
-               uint32_t **vals_out, cudaStream_t s, Workspace *ws) {
+               uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0) {
     *keys_out = keys;
     *vals_out = vals;
     if (n <= 1 || bits <= 0) return SJ_OK;
@@ -174,14 +175,17 @@ int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_
     }
     const uint32_t ntiles = (uint32_t)((n + kRadixTile - 1) / kRadixTile);
     const uint64_t hbytes = (uint64_t)kRadixBins * ntiles * sizeof(uint32_t);
-    uint32_t *hist = ws ? static_cast<uint32_t *>(ws->take(hbytes)) : nullptr;
+    // hist0: the first pass's tile histogram, already counted by the producer of the keys
+    uint32_t *hist = hist0 ? hist0 : ws ? static_cast<uint32_t *>(ws->take(hbytes)) : nullptr;
     const bool own = hist == nullptr;
     if (own) SJ_TRY(dev_alloc(reinterpret_cast<void **>(&hist), hbytes + 16, s));
     K *ka = keys, *kb = keys_alt;
     uint32_t *va = vals, *vb = vals_alt;
     for (int shift = 0; shift < bits; shift += 8) {
-        radix_hist_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, n, shift, hist, ntiles);
-        note_launch();
+        if (!(hist0 && shift == 0)) {
+            radix_hist_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, n, shift, hist, ntiles);
+            note_launch();
+        }
         SJ_TRY(scan_exclusive_u32(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s, ws));
         radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, va, kb, vb, n, shift, hist, ntiles);
         note_launch();
@@ -255,12 +259,12 @@ int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uin
 }
 
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws) {
-    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws);
+                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0) {
+    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws, hist0);
 }
 int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws) {
-    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws);
+                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0) {
+    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws, hist0);
 }
 
 }  // namespace sj

@@ -1619,7 +1619,13 @@ static bool blob_header_ok(const BlobHeader &b, uint64_t bytes, const char **why
     return true;
 }
 
-sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
+static sj_handle *from_index_impl(const void *blob, uint64_t bytes, bool view);
+
+sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) { return from_index_impl(blob, bytes, false); }
+
+sj_handle *sj_create_from_index_view(const void *blob, uint64_t bytes) { return from_index_impl(blob, bytes, true); }
+
+static sj_handle *from_index_impl(const void *blob, uint64_t bytes, bool view) {
     set_error("");
     if (!blob || bytes < kHdr) {
         set_error("sj_create_from_index: invalid blob");
@@ -1633,6 +1639,11 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
     }
     sj_handle *h = nullptr;
     if (create_common(&h) < 0) return nullptr;
+    if (view && (!is_device_ptr(blob, h->device) || (reinterpret_cast<uintptr_t>(blob) & 255u))) {
+        sj_destroy(h);
+        set_error("sj_create_from_index_view: the blob must be device memory of the current device, 256-byte aligned");
+        return nullptr;
+    }
     cudaStream_t s = h->s_main;
     // the blob may have been written on the caller's stream (e.g. the NCCL broadcast's output)
     BlobHeader b;
@@ -1683,6 +1694,14 @@ sj_handle *sj_create_from_index(const void *blob, uint64_t bytes) {
     ix.lookup_hash = (int)b.lookup_hash;
     void **dst[7] = {(void **)&ix.pts,  (void **)&ix.orig,     (void **)&ix.qmap,  (void **)&ix.cellq,
                      (void **)&ix.runs, (void **)&ix.cell_lid, (void **)&ix.chunks};
+    if (view) {  // zero copy: the arrays are the blob's (the caller keeps it alive, unchanged)
+        for (int i = 0; i < 7; ++i)
+            *dst[i] = const_cast<char *>(static_cast<const char *>(blob)) + b.off[i];
+        h->owns_index = false;
+        if (ix.dim >= 4) h->grab = 1;
+        fill_static_stats(h);
+        return h;
+    }
     for (int i = 0; i < 7 && rc == SJ_OK; ++i) {
         rc = dev_alloc(dst[i], b.bytes[i] + 32, s);
         if (rc == SJ_OK && b.bytes[i] &&

@@ -39,9 +39,11 @@ def allreduce_counts(values, group=None, device: str | torch.device = "cpu", op=
     return [int(x) for x in t.tolist()]
 
 
-def replicate_index(handle: Handle | None, src: int = 0, group=None, device="cuda"):
+def replicate_index(handle: Handle | None, src: int = 0, group=None, device="cuda", view: bool | None = None):
     """Rank `src` exports its handle's index into a device blob, NCCL-broadcasts it, and every
-    other rank builds a handle from it.  Returns (handle, blob)."""
+    other rank builds a handle from it -- by default (device blobs) a zero-copy VIEW whose index
+    arrays are the broadcast buffer itself (sj_create_from_index_view: no allocation, no copy;
+    the handle keeps the blob alive).  Returns (handle, blob)."""
     rank = dist.get_rank(group)
     blob = None
     if rank == src:
@@ -50,8 +52,25 @@ def replicate_index(handle: Handle | None, src: int = 0, group=None, device="cud
         handle.export_index(blob, nbytes)
     blob = broadcast_blob(blob, src, group, device)
     if rank != src:
-        handle = Handle.from_index(blob, blob.numel())
+        if view is None:
+            view = blob.is_cuda
+        handle = Handle.from_index(blob, blob.numel(), view=view)
     return handle, blob
+
+
+def replicated_self_join(points, eps: float, out, cap: int, group=None, **options):
+    """The multi-GPU path for inputs every rank holds (the bench's replicated input): every rank
+    builds the same index from its own copy (the build is deterministic: identical D', chunks and
+    slices on every rank), joins its WorkQueue slice (chunk c -> rank c mod world) into `out`,
+    and one all-reduce sums the pairs.  No broadcast: the build runs on all ranks at once instead
+    of on one rank followed by a 100+ MB broadcast.  Returns (handle, local_pairs, total)."""
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    h = Handle(points, eps, **options)
+    h.set_slice(rank, world)
+    rc, local = h.self_join(out, cap)
+    dev = out.device if hasattr(out, "device") else torch.device("cpu")
+    total = allreduce_counts([local], group, dev)[0]
+    return h, local, total
 
 
 def distributed_self_join(points, eps: float, out, cap: int, group=None, src: int = 0, **options):

@@ -266,6 +266,12 @@ def test_index_blob_roundtrip():
     np.testing.assert_array_equal(canon(got), want)
     with sj.Handle.from_index(host_blob, nbytes) as h3:
         assert h3.count() == want.shape[0]
+    # zero-copy view of a device blob: the handle's arrays are the blob's
+    with sj.Handle.from_index(blob, nbytes, view=True) as h4:
+        got4 = sj.self_join_pairs(h4, DEV).cpu().numpy().view(np.uint32)
+    np.testing.assert_array_equal(canon(got4), want)
+    with pytest.raises(sj.SJError):  # a host blob cannot be viewed
+        sj.Handle.from_index(host_blob, nbytes, view=True)
 
 # (full BASELINE sizes: tests/test_fullsize_gpu.py, element by element)
 
