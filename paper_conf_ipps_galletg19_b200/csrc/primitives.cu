@@ -62,27 +62,41 @@ static_assert(kRadixTile == kRadixTileKeys, "the cell-id kernel counts the first
 constexpr int kRadixBins = 256;
 
 // Per-tile digit counts, digit-major: hist[d * ntiles + tile].
+// (warp-private counters: the 256 bins of one shared histogram serialise a warp's atomics on
+// the frequent digits of clustered keys; the keys are loaded first, then counted)
 template <class K>
 __global__ void __launch_bounds__(kRadixThreads) radix_hist_kernel(const K *keys, uint64_t n, int shift,
                                                                    uint32_t *hist, uint32_t ntiles) {
-    __shared__ uint32_t h[kRadixBins];
-    h[threadIdx.x] = 0;
+    __shared__ uint32_t h[kRadixWarps][kRadixBins];
+#pragma unroll
+    for (int w = 0; w < kRadixWarps; ++w) h[w][threadIdx.x] = 0;
     __syncthreads();
+    const int warp = threadIdx.x >> 5;
     const uint64_t base = (uint64_t)blockIdx.x * kRadixTile;
+    uint32_t d[kRadixItems];
 #pragma unroll
     for (int it = 0; it < kRadixItems; ++it) {
-        uint64_t i = base + (uint64_t)it * kRadixThreads + threadIdx.x;
-        if (i < n) atomicAdd(&h[(uint32_t)(keys[i] >> shift) & 0xFFu], 1u);
+        const uint64_t i = base + (uint64_t)it * kRadixThreads + threadIdx.x;
+        d[it] = i < n ? (uint32_t)(keys[i] >> shift) & 0xFFu : kRadixBins;
     }
+#pragma unroll
+    for (int it = 0; it < kRadixItems; ++it)
+        if (d[it] < kRadixBins) atomicAdd(&h[warp][d[it]], 1u);
     __syncthreads();
-    hist[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
+    uint32_t t = 0;
+#pragma unroll
+    for (int w = 0; w < kRadixWarps; ++w) t += h[w][threadIdx.x];
+    hist[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = t;
 }
 
 // Stable scatter of one tile: per-warp ranks with __match_any_sync, a block-wide prefix
 // over warps and digits, global starts from the scanned digit-major histogram, and a
 // shared-memory reorder so each digit's run is written contiguously.
+#ifndef SJ_SCATTER_MINB
+#define SJ_SCATTER_MINB 4
+#endif
 template <class K>
-__global__ void __launch_bounds__(kRadixThreads) radix_scatter_kernel(const K *keys_in, const uint32_t *vals_in,
+__global__ void __launch_bounds__(kRadixThreads, SJ_SCATTER_MINB) radix_scatter_kernel(const K *keys_in, const uint32_t *vals_in,
                                                                       K *keys_out, uint32_t *vals_out, uint64_t n,
                                                                       int shift, const uint32_t *hist_scanned,
                                                                       uint32_t ntiles) {
