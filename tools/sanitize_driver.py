@@ -60,6 +60,19 @@ for cfg in cases:
             rc, c = h.self_join(small_out, small_out.shape[0])
             parts.append(small_out[:c].cpu().numpy().view(np.uint32).copy())
     assert np.array_equal(canon(np.concatenate(parts)), want), "overflow"
+    # 5b. blocked in-place output (per-warp output blocks + compaction), exact and larger buffers
+    for slack in (0, 999):
+        ob = torch.full((want.shape[0] + slack, 2), -1, dtype=torch.int32, device="cuda")
+        with sj.Handle(d, cfg.eps, k=8, out_blocks=1) as h:
+            rc, c = h.self_join(ob, want.shape[0] + slack)
+        assert rc == sj.SJ_OK and np.array_equal(canon(ob[:c]), want), "blocked"
+    # 5c. zero-copy index view
+    with sj.Handle(d, cfg.eps, k=8) as h:
+        nb = h.export_index()
+        blob = torch.empty(nb, dtype=torch.uint8, device="cuda")
+        h.export_index(blob, nb)
+    with sj.Handle.from_index(blob, nb, view=True) as h:
+        assert np.array_equal(canon(sj.self_join_pairs(h, "cuda")), want), "view"
     # 6. device CSR on the GCG pattern
     with sj.Handle(d, cfg.eps, pattern="gcg", k=8) as h:
         off, nb = h.neighbor_csr()
