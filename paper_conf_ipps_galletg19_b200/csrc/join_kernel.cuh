@@ -84,9 +84,12 @@ struct Mode {
     static constexpr bool exact = MODE == kExact;                     // ... at chunk offsets
 };
 
+#ifndef SJ_BUF3
+#define SJ_BUF3 512
+#endif
 template <int DIM>
 struct BufCap {
-    static constexpr int value = DIM <= 3 ? kBufHits : kBufHitsHi;
+    static constexpr int value = DIM <= 2 ? kBufHits : DIM == 3 ? SJ_BUF3 : kBufHitsHi;
 };
 
 // Per-warp shared memory: emission buffer, the chunk's queries, one candidate tile.
@@ -149,7 +152,7 @@ struct WarpSmem {
         };
         struct {
             uint2 gruns[32 * StagedRuns<DIM>::value];  // generic (3-D) / flat: the queries' first runs
-            unsigned wpre[32];                         // flat: exclusive prefix of the list lengths
+            unsigned char neq[32];                     // flat: lanes of the non-empty lists, in order
             uint4 fq[32];                              // flat: per query {home begin, m, rr, S}
         };
     };
@@ -670,9 +673,10 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
 // so their candidate loads are in flight together.  The k-lane rounds of generic_chunk instead
 // walk 32/k queries per round with a dependent global load chain each round, which is what the
 // sparse tail's time is made of (it is latency-bound, not issue-bound).  The queries' points,
-// ids and forward runs are staged in shared memory first; the query of pair f is found by a
-// binary search over the prefix sums of the list lengths.  Returns false (nothing evaluated)
-// when a list is longer than SJ_FLAT_W or a cell has more runs than are staged (UNICOMP).
+// ids and forward runs are staged in shared memory first; the query of pair f is the r-th
+// non-empty list, r counted with a ballot and an OR-reduction of the lists' start bits.
+// Returns false (nothing evaluated) when a list is longer than SJ_FLAT_W or a cell has more runs
+// than are staged (UNICOMP).
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, uint2 qm_lane, uint4 ci_lane,
                                            WarpSmem<DIM, MODE> &ws, int &nbuf, unsigned long long &nhits,
@@ -699,7 +703,9 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
         if (lane >= o) incl += v;
     }
     const unsigned T = __shfl_sync(kFull, incl, 31);
-    ws.wpre[lane] = incl - W;
+    const unsigned start = incl - W;  // the lane's first pair number
+    const unsigned nem = __ballot_sync(kFull, W > 0u);
+    if (W > 0u) ws.neq[__popc(nem & lt)] = (unsigned char)lane;
     ws.fq[lane] = make_uint4(ci_lane.x, ci_lane.y, rr_l, ci_lane.w);
     cp_async_commit();
     cp_async_wait<0>();
@@ -722,13 +728,17 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
         bool ok[2];
 #pragma unroll
         for (int u = 0; u < 2; ++u) {
-            const unsigned f = f0 + (unsigned)(u * 32 + lane);
+            const unsigned fb = f0 + (unsigned)(u * 32), f = fb + (unsigned)lane;
             ok[u] = f < T;
-            unsigned q = 0;  // the last query whose prefix is <= f (zero-length lists are skipped)
-#pragma unroll
-            for (unsigned st = 16; st > 0; st >>= 1)
-                if (ws.wpre[q + st] <= f) q += st;
-            unsigned j = f - ws.wpre[q];
+            // the query of pair f: the r-th non-empty list, r = the non-empty lists starting at
+            // or before f (the starts of non-empty lists are distinct) -- those before the
+            // window, plus the window's start bits up to f
+            const unsigned rel = start - fb;
+            const unsigned before = __ballot_sync(kFull, W > 0u && start < fb);
+            const unsigned win = __reduce_or_sync(kFull, (W > 0u && rel < 32u) ? 1u << rel : 0u);
+            const int r = __popc(before) + __popc(win & ((2u << lane) - 1u));  // >= 1: the first list starts at 0
+            const unsigned q = ws.neq[r - 1];
+            unsigned j = f - __shfl_sync(kFull, start, q);
             const uint4 d = ws.fq[q];  // {home begin, m, rr, S}
             unsigned idx;
             if (j < d.w) {  // forward runs, in order
@@ -783,6 +793,7 @@ __device__ __forceinline__ unsigned tile_rounds(const JoinArgs &a, unsigned nq, 
     // kRows / kDegree: the round's query cursor (count) lives in ws.qcur between rounds
     auto round_end = [&](unsigned qi, bool qv, unsigned long long cur, unsigned long long nh0) {
         if constexpr (MODE == kRows) {
+            __syncwarp();  // every lane of the group read the cursor before it is advanced (racecheck)
             if (t == 0 && qv) ws.qcur[qi] = cur;
         } else if constexpr (MODE == kDegree) {
             const unsigned d = group_sum<K>((unsigned)(nhits - nh0));
@@ -1129,9 +1140,12 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
 
 // 3-D kernels are held to three resident CTAs per SM (their shared-memory limit), i.e. up to 85
 // registers: ptxas' own choice otherwise drifts between 64 with spills and 80 with small changes.
+#ifndef SJ_MINB3
+#define SJ_MINB3 3
+#endif
 template <int DIM>
 struct MinBlocks {
-    static constexpr int value = DIM == 3 ? 3 : 0;
+    static constexpr int value = DIM == 3 ? SJ_MINB3 : 0;
 };
 
 template <int DIM, int K, int MODE, bool GCG>
