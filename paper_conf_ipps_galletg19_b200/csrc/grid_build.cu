@@ -219,11 +219,12 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
 // The geometry comes from device memory (bbox_kernel's last block); keys are 32-bit when the
 // grid has at most 2^32 cells, else 64-bit (the host picks the buffer once it reads key_bits).
 // One block per radix tile (kRadixTileKeys points): it also counts the tile's low 8-bit digits,
-// the first pass of the point sort (a4) -- its histogram kernel is not launched.
+// the first pass of the point sort (a4) -- its histogram kernel is not launched.  The sort's
+// values (input ids) are the identity, generated by its first scatter: not written here.
 constexpr int kCellIdThreads = 1024;  // 2 points per thread: the 6-D divisions need the parallelism
 __global__ void __launch_bounds__(kCellIdThreads) cell_id_kernel(const double *raw, uint64_t n,
                                                            const GeomDev *__restrict__ gp, uint32_t *keys32,
-                                                           unsigned long long *keys64, uint32_t *vals, GeomArgs ga,
+                                                           unsigned long long *keys64, GeomArgs ga,
                                                            uint32_t *hist0, uint32_t ntiles) {
     __shared__ uint32_t h[256];
     if (threadIdx.x < 256) h[threadIdx.x] = 0;
@@ -250,7 +251,6 @@ __global__ void __launch_bounds__(kCellIdThreads) cell_id_kernel(const double *r
             keys32[i] = (uint32_t)lid;
         else
             keys64[i] = lid;
-        vals[i] = (uint32_t)i;
         atomicAdd(&h[(uint32_t)lid & 0xFFu], 1u);
     }
     __syncthreads();
@@ -483,7 +483,8 @@ template <bool FILL, int LPC>
 __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
                                                         const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *rcnt,
                                                         uint32_t *wload, const uint32_t *rbegin, uint2 *runs,
-                                                        BuildTotals *tot, TotalsPub pub) {
+                                                        BuildTotals *tot, TotalsPub pub, uint32_t *wkey,
+                                                        uint32_t *wval) {
     // grid-stride over the cells (M is only known on the device): a bounded grid, so the block
     // reduction below runs once per resident block, not once per n-sized block
     const uint64_t M = *d_M;
@@ -553,6 +554,12 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
                     calcs += (unsigned long long)m * (m - 1) / 2 + (unsigned long long)m * summ;
                 }
                 wload[r] = wr;
+                // a8's SortByWL keys (the counting pass writes them: no key kernel): sorted on their
+                // low bits_for(max W) bits, ~W ascending is W non-increasing, ties in lid order (the
+                // value r); a partitioned index sorts on bits_for(max W + 1) bits, its query cells
+                // keyed ~(W + 1) and its halo cells ~0, after every query cell
+                wkey[r] = g.idx ? (qcell ? ~(wr + 1u) : ~0u) : ~wr;
+                wval[r] = (uint32_t)r;
                 w = max(w, wr);
             }
         }
@@ -600,57 +607,48 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
     }
 }
 
-// a8 (SortByWL): key = max_w - W so an ascending stable sort gives non-increasing W
-// (partitioned index: halo cells get max_w + 1, so they sort after every query cell and the
-// queries occupy D' positions [0, nq))
-__global__ void __launch_bounds__(kThreads) wl_keys_kernel(const uint32_t *wload, uint64_t M, uint32_t max_w,
-                                                           uint32_t *keys, uint32_t *vals, const uint32_t *cell_start,
-                                                           const uint32_t *idx, uint32_t nq) {
-    uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= M) return;
-    keys[r] = (idx && idx[cell_start[r]] >= nq) ? max_w + 1u : max_w - wload[r];
-    vals[r] = (uint32_t)r;
-}
-
 // Empty chunks after the last one (kChunkPad): chunks[C + 1 + t] = the end of the queries.
 __global__ void __launch_bounds__(kThreads) chunk_pad_kernel(uint32_t *chunks, const uint32_t *d_nc, uint32_t end) {
     chunks[*d_nc + 1u + blockIdx.x * kThreads + threadIdx.x] = end;
 }
 
-__global__ void __launch_bounds__(kThreads) queue_m_kernel(const uint32_t *qorder, const uint32_t *cell_start,
-                                                           uint64_t M, uint32_t *mq) {
-    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= M) return;
-    uint32_t r = qorder[i];
-    mq[i] = cell_start[r + 1] - cell_start[r];
-}
-
-__global__ void __launch_bounds__(kThreads) cells_finalize_kernel(const uint32_t *qorder, const uint32_t *qb,
-                                                                  const uint32_t *cell_start, const uint32_t *rbegin,
-                                                                  uint32_t slot_rows,
-                                                                  const uint32_t *wload,
-                                                                  const unsigned long long *cell_lid, uint64_t M,
-                                                                  int full, uint4 *cellq, uint32_t *r2q, uint32_t *qbr,
-                                                                  uint64_t *lid_q, const uint32_t *idx, uint32_t nq) {
-    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= M) return;
-    uint32_t r = qorder[i];
-    uint32_t m = cell_start[r + 1] - cell_start[r];
-    const uint32_t rb = rbegin ? rbegin[r] : r * slot_rows;  // first forward run
-    if (idx && idx[cell_start[r]] >= nq) {  // halo cell: never queued (m = 0 in its record)
-        cellq[i] = make_uint4(cell_start[r], 0u, rb, 0u);
-        r2q[r] = (uint32_t)i;
-        qbr[r] = qb[i];
-        lid_q[i] = cell_lid[r];
-        return;
+// a8's queue cells, one fused scan (no count kernel, no separate finalize): load(i) = m of the
+// i-th cell of the queue order, store(i, qb) = its record at queue position i, qb = its first D'
+// position (the exclusive prefix of the counts).
+struct QueueLoad {
+    const uint32_t *qorder, *cell_start;
+    __device__ unsigned operator()(uint64_t i) const {
+        const uint32_t r = qorder[i];
+        return cell_start[r + 1] - cell_start[r];
     }
-    // {begin in the lid-ordered storage, m, first run, S = sum of the runs' lengths}
-    // (half patterns: W = floor(m/2) + S; GCG: W = S - 1, the query itself excluded)
-    cellq[i] = make_uint4(cell_start[r], m, rb, full ? wload[r] + 1 : wload[r] - m / 2);
-    r2q[r] = (uint32_t)i;
-    qbr[r] = qb[i];
-    lid_q[i] = cell_lid[r];
-}
+};
+struct QueueStore {
+    const uint32_t *qorder, *cell_start, *rbegin;
+    uint32_t slot_rows;
+    const uint32_t *wload;
+    const unsigned long long *cell_lid;
+    int full;
+    uint4 *cellq;
+    uint32_t *r2q, *qbr, *qb;
+    uint64_t *lid_q;
+    const uint32_t *idx;
+    uint32_t nq;
+    __device__ void operator()(uint64_t i, unsigned ex, unsigned m) const {
+        const uint32_t r = qorder[i];
+        const uint32_t rb = rbegin ? rbegin[r] : r * slot_rows;  // first forward run
+        qb[i] = ex;
+        r2q[r] = (uint32_t)i;
+        qbr[r] = ex;
+        lid_q[i] = cell_lid[r];
+        if (idx && idx[cell_start[r]] >= nq) {  // halo cell: never queued (m = 0 in its record)
+            cellq[i] = make_uint4(cell_start[r], 0u, rb, 0u);
+            return;
+        }
+        // {begin in the lid-ordered storage, m, first run, S = sum of the runs' lengths}
+        // (half patterns: W = floor(m/2) + S; GCG: W = S - 1, the query itself excluded)
+        cellq[i] = make_uint4(cell_start[r], m, rb, full ? wload[r] + 1 : wload[r] - m / 2);
+    }
+};
 
 // Points gathered into lid (spatial) order, padded AoS, plus D' = the queue as an index
 // array: qmap[D' position] = {lid-storage position, queue-order cell}.  With
@@ -942,9 +940,9 @@ static int sort_points(Temps &tmp, K *ka, uint32_t *va, uint64_t n, int bits, cu
     SJ_TRY(tmp.alloc(&kb, n));
     SJ_TRY(tmp.alloc(&vb, n));
     if constexpr (sizeof(K) == 4)
-        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws, hist0));
+        SJ_TRY(radix_sort_u32(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws, hist0, true));
     else
-        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws, hist0));
+        SJ_TRY(radix_sort_u64(ka, va, kb, vb, n, bits, keys_sorted, idx_sorted, s, &tmp.ws, hist0, true));
     return SJ_OK;
 }
 
@@ -1043,7 +1041,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     const uint32_t ntiles = (uint32_t)((n + kRadixTileKeys - 1) / kRadixTileKeys);
     uint32_t *hist0;  // the point sort's first-pass tile histogram, counted by the cell-id kernel
     SJ_TRY(tmp.alloc(&hist0, (uint64_t)256 * ntiles));
-    cell_id_kernel<<<ntiles, kCellIdThreads, 0, s>>>(d_raw, n, d_geo, keys32, keys64, vals0, ga, hist0, ntiles);
+    cell_id_kernel<<<ntiles, kCellIdThreads, 0, s>>>(d_raw, n, d_geo, keys32, keys64, ga, hist0, ntiles);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     if (zero_copy) {
@@ -1223,12 +1221,18 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         pub.epoch = next_epoch();
         h_pub[5] = 0;
     }
+    // a8's SortByWL keys and values, written by the counting pass (M <= n cells)
+    uint32_t *wk, *wv;
+    SJ_TRY(tmp.alloc(&wk, n));
+    SJ_TRY(tmp.alloc(&wv, n));
     if (wide)
         runs_kernel<false, 32><<<runs_grid(n, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                    nullptr, slots ? ix.runs : nullptr, d_tot, pub);
+                                                                    nullptr, slots ? ix.runs : nullptr, d_tot, pub,
+                                                                    wk, wv);
     else
         runs_kernel<false, 1><<<runs_grid(n, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                  nullptr, slots ? ix.runs : nullptr, d_tot, pub);
+                                                                  nullptr, slots ? ix.runs : nullptr, d_tot, pub,
+                                                                  wk, wv);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin = nullptr;
@@ -1296,22 +1300,18 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         // (the counting pass wrote them)
     } else if (wide)
         runs_kernel<true, 32><<<runs_grid(M, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
-                                                                    rbegin, ix.runs, nullptr, TotalsPub{});
+                                                                    rbegin, ix.runs, nullptr, TotalsPub{}, nullptr,
+                                                                    nullptr);
     else
         runs_kernel<true, 1><<<runs_grid(M, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
-                                                              rbegin, ix.runs, nullptr, TotalsPub{});
+                                                              rbegin, ix.runs, nullptr, TotalsPub{}, nullptr, nullptr);
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
 
     // ---- a8: SortByWL over cells -> D' (queue of points in non-increasing W)
-    uint32_t *wk, *wv, *wk2, *wv2, *qorder_keys, *qorder;
-    SJ_TRY(tmp.alloc(&wk, M));
-    SJ_TRY(tmp.alloc(&wv, M));
+    uint32_t *wk2, *wv2, *qorder_keys, *qorder;
     SJ_TRY(tmp.alloc(&wk2, M));
     SJ_TRY(tmp.alloc(&wv2, M));
-    wl_keys_kernel<<<grid_for(M), kThreads, 0, s>>>(wload, M, ix.max_w, wk, wv, cell_start, part ? idx_sorted : nullptr,
-                                                    (uint32_t)nq);
-    note_launch();
     if (ix.order == SJ_ORDER_WORKLOAD) {
         SJ_TRY(radix_sort_u32(wk, wv, wk2, wv2, M, bits_for(part ? ix.max_w + 1ull : ix.max_w), &qorder_keys, &qorder,
                               s, &tmp.ws));
@@ -1319,12 +1319,8 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         qorder_keys = wk;
         qorder = wv;
     }
-    uint32_t *mq, *qb;
-    SJ_TRY(tmp.alloc(&mq, M));
+    uint32_t *qb;
     SJ_TRY(tmp.alloc(&qb, M));
-    queue_m_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, cell_start, M, mq);
-    note_launch();
-    SJ_TRY(scan_exclusive_u32(mq, qb, M, nullptr, s, &tmp.ws));
 
     // ---- final arrays
     SJ_TRY(dev_alloc_t(&ix.cellq, M, s));
@@ -1333,11 +1329,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     uint32_t *r2q, *qbr;
     SJ_TRY(tmp.alloc(&r2q, M));
     SJ_TRY(tmp.alloc(&qbr, M));
-    cells_finalize_kernel<<<grid_for(M), kThreads, 0, s>>>(qorder, qb, cell_start, rbegin, (uint32_t)R, wload,
-                                                           cell_lid, M,
-                                                           fg.full, ix.cellq, r2q, qbr, ix.cell_lid,
-                                                           part ? idx_sorted : nullptr, (uint32_t)nq);
-    note_launch();
+    SJ_TRY(scan_fused(M, QueueLoad{qorder, cell_start},
+                      QueueStore{qorder, cell_start, rbegin, (uint32_t)R, wload, cell_lid, fg.full, ix.cellq, r2q, qbr,
+                                 qb, ix.cell_lid, part ? idx_sorted : nullptr, (uint32_t)nq},
+                      s, NoDone(), &tmp.ws));
     // D' (qmap): after the cells' queue positions; on the side stream too (the chunk scan below
     // needs it only in input order), the main stream waits for it before the build ends
     if (side) {

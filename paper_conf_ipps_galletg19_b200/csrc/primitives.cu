@@ -5,7 +5,7 @@
 // cells by workload for SortByWL.  Per 8-bit pass:
 //   1. tile histogram (2048 keys per CTA, shared-memory counters), digit-major,
 //   2. single-pass exclusive scan (decoupled look-back) of the [256 x tiles] histogram,
-//   3. stable scatter: per-warp ranks with __match_any_sync, a block-wide prefix over
+//   3. stable scatter: per-warp ranks from ballots over the digit bits, a block-wide prefix over
 //      warps and digits, a shared-memory reorder of the tile so the global writes of one
 //      digit run are contiguous (coalesced).
 #include <cstdio>
@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(kRadixThreads) radix_hist_kernel(const K *keys
     hist[(uint64_t)threadIdx.x * ntiles + blockIdx.x] = t;
 }
 
-// Stable scatter of one tile: per-warp ranks with __match_any_sync, a block-wide prefix
+// Stable scatter of one tile: per-warp ranks from 8 ballots over the digit bits, a block-wide prefix
 // over warps and digits, global starts from the scanned digit-major histogram, and a
 // shared-memory reorder so each digit's run is written contiguously.
 #ifndef SJ_SCATTER_MINB
@@ -122,7 +122,7 @@ __global__ void __launch_bounds__(kRadixThreads, SJ_SCATTER_MINB) radix_scatter_
         uint64_t i = wbase + (uint64_t)it * 32 + lane;
         if (i < n) {
             key[it] = keys_in[i];
-            val[it] = vals_in[i];
+            val[it] = vals_in ? vals_in[i] : (uint32_t)i;  // null: the identity (first pass of the point sort)
             dig[it] = (uint32_t)(key[it] >> shift) & 0xFFu;
         } else {
             key[it] = 0;
@@ -131,10 +131,20 @@ __global__ void __launch_bounds__(kRadixThreads, SJ_SCATTER_MINB) radix_scatter_
         }
     }
     __syncthreads();
+    // (only the last tile has empty slots: their sentinel digit matches no key's below)
+    const bool full_tile = base + (uint64_t)kRadixTile <= n;
 #pragma unroll
     for (int it = 0; it < kRadixItems; ++it) {
         const uint32_t d = dig[it];
-        const uint32_t peers = __match_any_sync(0xffffffffu, d);
+        // the lanes of this item with the same digit, from 8 ballots over the digit's bits
+        // (__match_any_sync runs on the ADU pipe at ~70 cycles a warp: it bound this kernel)
+        uint32_t peers = full_tile ? 0xffffffffu : __ballot_sync(0xffffffffu, d < kRadixBins);
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+            const uint32_t bit = (d >> b) & 1u;
+            const uint32_t bb = __ballot_sync(0xffffffffu, bit);
+            peers &= bit ? bb : ~bb;
+        }
         uint32_t before = 0;
         if (d < kRadixBins) before = cnt[warp][d];
         rank[it] = before + __popc(peers & lt);
@@ -177,12 +187,26 @@ __global__ void __launch_bounds__(kRadixThreads, SJ_SCATTER_MINB) radix_scatter_
     }
 }
 
+__global__ void __launch_bounds__(kRadixThreads) iota_kernel(uint32_t *v, uint64_t n) {
+    const uint64_t i = (uint64_t)blockIdx.x * kRadixThreads + threadIdx.x;
+    if (i < n) v[i] = (uint32_t)i;
+}
+
+// vals_identity: `vals` holds no values yet -- they are the identity 0..n-1, generated by the
+// first pass's scatter (the point sort: no kernel writes the input ids), and `vals` is scratch.
 template <class K>
 int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_t n, int bits, K **keys_out,
-               uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0) {
+               uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0, bool vals_identity) {
     *keys_out = keys;
     *vals_out = vals;
-    if (n <= 1 || bits <= 0) return SJ_OK;
+    if (n <= 1 || bits <= 0) {
+        if (vals_identity && n) {
+            iota_kernel<<<(unsigned)((n + kRadixThreads - 1) / kRadixThreads), kRadixThreads, 0, s>>>(vals, n);
+            note_launch();
+            SJ_CUDA_TRY(cudaGetLastError());
+        }
+        return SJ_OK;
+    }
     if (n >= (1ull << 32)) {
         set_error("radix_sort: n >= 2^32");
         return SJ_EINVAL;
@@ -201,7 +225,8 @@ int radix_sort(K *keys, uint32_t *vals, K *keys_alt, uint32_t *vals_alt, uint64_
             note_launch();
         }
         SJ_TRY(scan_exclusive_u32(hist, hist, (uint64_t)kRadixBins * ntiles, nullptr, s, ws));
-        radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, va, kb, vb, n, shift, hist, ntiles);
+        radix_scatter_kernel<K><<<ntiles, kRadixThreads, 0, s>>>(ka, (vals_identity && shift == 0) ? nullptr : va, kb,
+                                                                 vb, n, shift, hist, ntiles);
         note_launch();
         SJ_CUDA_TRY(cudaGetLastError());
         K *tk = ka; ka = kb; kb = tk;
@@ -273,12 +298,16 @@ int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uin
 }
 
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0) {
-    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws, hist0);
+                   uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0,
+                   bool vals_identity) {
+    return radix_sort<uint32_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws, hist0,
+                                vals_identity);
 }
 int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
-                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0) {
-    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws, hist0);
+                   uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws, uint32_t *hist0,
+                   bool vals_identity) {
+    return radix_sort<uint64_t>(keys, vals, keys_alt, vals_alt, n, bits, keys_out, vals_out, s, ws, hist0,
+                                vals_identity);
 }
 
 }  // namespace sj

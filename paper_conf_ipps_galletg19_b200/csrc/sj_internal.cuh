@@ -124,13 +124,15 @@ int scan_exclusive_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, uin
 // or the alternates).
 // hist0 (optional): the first pass's tile histogram (digit-major [256][tiles of 2048 keys]),
 // already counted by the kernel that produced the keys; it also serves as the histogram buffer.
+// vals_identity: the values are the identity 0..n-1, generated by the first pass (`vals` is then
+// uninitialised scratch of n entries).
 constexpr int kRadixTileKeys = 2048;
 int radix_sort_u32(uint32_t *keys, uint32_t *vals, uint32_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
                    uint32_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws = nullptr,
-                   uint32_t *hist0 = nullptr);
+                   uint32_t *hist0 = nullptr, bool vals_identity = false);
 int radix_sort_u64(uint64_t *keys, uint32_t *vals, uint64_t *keys_alt, uint32_t *vals_alt, uint64_t n, int bits,
                    uint64_t **keys_out, uint32_t **vals_out, cudaStream_t s, Workspace *ws = nullptr,
-                   uint32_t *hist0 = nullptr);
+                   uint32_t *hist0 = nullptr, bool vals_identity = false);
 
 // --------------------------------------------------------------------------- index
 // The index I in its B200 layout, DESIGN.md §4.  Points are stored in the
