@@ -90,7 +90,7 @@ enum sj_option {
     SJ_OPT_OUT_BLOCKS = 11     /* in-place output allocation: 0 = one atomic on the output counter per
                                   warp flush; 1 = blocks of 4096 pairs per warp (one atomic per block),
                                   the gaps the warps' last blocks leave closed by a compaction pass;
-                                  2 = blocks when the caller's buffer holds >= 1e9 pairs (default): a
+                                  2 = blocks when the caller's buffer holds >= 3e8 pairs (default): a
                                   single counter taking every flush of a large result congests its L2
                                   slice and doubles the join (measured)                  */
 };

@@ -3,10 +3,11 @@
 // A blocked join hands out the output in blocks of blk pairs, one atomic per block and warp;
 // every block is filled completely except each warp's last one, whose unused rest is a gap.  So
 // after the join the pairs are [0, A) minus at most one gap per warp (A = the allocation
-// counter), positions from cap_e = out_cap & ~1 on in the scratch buffer.  With G = the gaps' total, the join produced T = A - G pairs.  This moves
-// the pairs lying at or past T into the gaps below T (both add up to the same count), so the
-// output is [0, T) again: the k-th pair past T (in position order, gaps skipped) goes to the
-// k-th hole below T.  Holes and sources are disjoint, so one parallel copy does it.
+// counter), positions from cap_e = out_cap & ~1 on in the scratch buffer.  With G = the gaps'
+// total, the join produced T = A - G pairs.  This moves the pairs lying at or past T into the
+// gaps below T (both add up to the same count), so the output is [0, T) again: the k-th pair past
+// T (in position order, gaps skipped) goes to the k-th hole below T (holes in warp order).  Holes
+// and sources are disjoint, so one parallel copy does it.
 #include <algorithm>
 
 #include "sj_internal.cuh"
@@ -15,8 +16,7 @@ namespace sj {
 
 namespace {
 
-constexpr int kMaxGaps = kCompactMaxWarps;  // >= the blocked join's warps (the runtime checks)
-static_assert(kMaxGaps == 8192, "the sort keys carry a 13-bit gap index");
+constexpr int kMaxGaps = kCompactMaxGaps;  // >= the blocked join's warps (the runtime checks)
 constexpr int kPrepThreads = 1024;
 
 struct CompactWs {
@@ -27,111 +27,96 @@ struct CompactWs {
 };
 
 // Exclusive scan of v[0, n) in shared memory (one block of kPrepThreads; n <= kMaxGaps + 2):
-// thread t scans its contiguous run of entries; returns the total.
+// thread t scans its contiguous run of entries, the runs' sums by warp shuffles; returns the total.
 __device__ unsigned long long block_scan(unsigned long long *v, int n, unsigned long long *part) {
-    const int t = threadIdx.x;
+    const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
     const int per = (n + kPrepThreads - 1) / kPrepThreads;
     const int lo = min(n, t * per), hi = min(n, lo + per);
     unsigned long long sum = 0;
     for (int i = lo; i < hi; ++i) sum += v[i];
-    part[t] = sum;
+    unsigned long long x = sum;  // inclusive scan of the runs' sums within the warp
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) part[wid] = x;
     __syncthreads();
-    for (int o = 1; o < kPrepThreads; o <<= 1) {  // Hillis-Steele inclusive scan of the runs' sums
-        const unsigned long long x = t >= o ? part[t - o] : 0ull;
-        __syncthreads();
-        part[t] += x;
-        __syncthreads();
+    if (wid == 0) {  // the warps' totals (kPrepThreads / 32 = 32 of them)
+        unsigned long long z = part[lane];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long y = __shfl_up_sync(0xffffffffu, z, o);
+            if (lane >= o) z += y;
+        }
+        part[lane] = z;
     }
-    unsigned long long run = part[t] - sum;
+    __syncthreads();
+    unsigned long long run = (wid ? part[wid - 1] : 0ull) + x - sum;
     for (int i = lo; i < hi; ++i) {
-        const unsigned long long x = v[i];
+        const unsigned long long y = v[i];
         v[i] = run;
-        run += x;
+        run += y;
     }
-    const unsigned long long total = part[kPrepThreads - 1];
+    const unsigned long long total = part[kPrepThreads / 32 - 1];
     __syncthreads();
     return total;
 }
 
-// One block: sort the gaps by start, T, the holes below T and the source segments past it, with
-// their prefix sums.  Dynamic shared memory: three arrays of kMaxGaps + 2 words (192 KB).
+// One block, no sort.  The allocation counter hands out blocks of blk pairs in order, so [0, A) is
+// blocks 0 .. A/blk - 1, every one full except each warp's LAST block, which holds the gap at its
+// end (gaps[2w] = its start, gaps[2w+1] = its length).  With T = A - sum of the gaps:
+//   holes   = the gaps' parts below T, listed in warp order;
+//   sources = the filled parts of the blocks b >= T / blk, clipped to >= T, in block order: a
+//             block is full unless it is some warp's last block (then filled up to its gap);
+//             there are at most (A - T) / blk + 1 <= warps + 1 such blocks.
+// The k-th source pair goes to the k-th hole pair (any pairing of equal totals closes the gaps).
+// Dynamic shared memory: two arrays of kMaxGaps + 2 words.
 __global__ void __launch_bounds__(kPrepThreads) compact_prep_kernel(const unsigned long long *gaps, int ngap,
                                                                    const unsigned long long *d_alloc,
-                                                                   unsigned long long cap_e, CompactWs *w,
-                                                                   unsigned long long *d_total) {
+                                                                   unsigned long long blk, unsigned long long cap_e,
+                                                                   CompactWs *w, unsigned long long *d_total) {
     extern __shared__ unsigned long long smem[];
-    unsigned long long *key = smem, *ln = smem + (kMaxGaps + 2), *tmp = smem + 2 * (kMaxGaps + 2);
-    __shared__ unsigned long long part[kPrepThreads];
-    __shared__ int s_m;
+    unsigned long long *hv = smem, *sv = smem + (kMaxGaps + 2);
+    __shared__ unsigned long long part[kPrepThreads / 32];
     const int t = threadIdx.x;
-    int np = 2;  // the sort's size: a power of two >= ngap
-    while (np < ngap) np <<= 1;
-    // keys (start / 2) << 13 | gap index: starts are even and distinct (the gaps are disjoint),
-    // gap index < kMaxGaps = 2^13; empty gaps sort last
-    for (int i = t; i < np; i += kPrepThreads) {
-        const bool ok = i < ngap && gaps[2 * i + 1] > 0;
-        key[i] = ok ? ((gaps[2 * i] >> 1) << 13) | (unsigned long long)i : ~0ull;
-    }
-    if (t == 0) s_m = 0;
+    // G = the gaps' total (the lengths through hv, scanned in place)
+    for (int i = t; i < ngap; i += kPrepThreads) hv[i] = gaps[2 * i + 1];
     __syncthreads();
-    for (int k = 2; k <= np; k <<= 1)  // bitonic sort
-        for (int j = k >> 1; j > 0; j >>= 1) {
-            for (int i = t; i < np; i += kPrepThreads) {
-                const int p = i ^ j;
-                if (p > i) {
-                    const bool up = (i & k) == 0;
-                    const unsigned long long x = key[i], y = key[p];
-                    if ((x > y) == up) {
-                        key[i] = y;
-                        key[p] = x;
-                    }
-                }
-            }
-            __syncthreads();
-        }
-    // the sorted gaps: key[i] becomes the start, ln[i] the length
-    int mine = 0;
-    for (int i = t; i < np; i += kPrepThreads) {
-        const unsigned long long kk = key[i];
-        const bool ok = kk != ~0ull;
-        const int g = (int)(kk & 8191ull);
-        key[i] = ok ? gaps[2 * g] : ~0ull;
-        ln[i] = ok ? gaps[2 * g + 1] : 0ull;
-        tmp[i] = ln[i];
-        mine += ok ? 1 : 0;
-    }
-    atomicAdd(&s_m, mine);
-    __syncthreads();
-    const int m = s_m;
-    unsigned long long *st = key;
-    const unsigned long long G = block_scan(tmp, np, part);
+    const unsigned long long G = block_scan(hv, ngap, part);
     const unsigned long long A = *d_alloc;
     const unsigned long long T = A - G;
-    // holes: the gaps' parts below T
-    for (int i = t; i < m; i += kPrepThreads) {
-        w->h_start[i] = st[i];
-        tmp[i] = st[i] < T ? min(st[i] + ln[i], T) - st[i] : 0ull;
+    const unsigned long long b0 = T / blk, b1 = (A + blk - 1) / blk;  // source blocks [b0, b1)
+    const int nb = (int)(b1 - b0);  // <= ngap + 1 (A - T = G < ngap * blk)
+    // holes below T, in warp order; the source blocks' fill (blk unless a warp's last block)
+    for (int i = t; i < ngap; i += kPrepThreads) {
+        const unsigned long long st = gaps[2 * i], ln = gaps[2 * i + 1];
+        w->h_start[i] = st;
+        hv[i] = (ln > 0 && st < T) ? min(st + ln, T) - st : 0ull;
+    }
+    for (int i = t; i < nb; i += kPrepThreads) sv[i] = blk;
+    __syncthreads();
+    for (int i = t; i < ngap; i += kPrepThreads) {
+        const unsigned long long st = gaps[2 * i], ln = gaps[2 * i + 1];
+        const unsigned long long b = st / blk;  // the gap's block (a gap never spans two)
+        if (ln > 0 && b >= b0 && b < b1) sv[b - b0] = st - b * blk;
     }
     __syncthreads();
-    const unsigned long long H = block_scan(tmp, m, part);
-    for (int i = t; i < m; i += kPrepThreads) w->h_pre[i] = tmp[i];
-    __syncthreads();
-    // sources: [T, A) outside the gaps -- the segments between consecutive gaps, clipped to >= T
-    for (int i = t; i <= m; i += kPrepThreads) {
-        const unsigned long long lo0 = i == 0 ? 0ull : st[i - 1] + ln[i - 1];
-        const unsigned long long hi = i == m ? A : st[i];
-        const unsigned long long lo = max(lo0, T);
+    for (int i = t; i < nb; i += kPrepThreads) {
+        const unsigned long long bs = (b0 + (unsigned long long)i) * blk, lo = max(bs, T), hi = bs + sv[i];
         w->s_start[i] = lo;
-        tmp[i] = hi > lo ? hi - lo : 0ull;
+        sv[i] = hi > lo ? hi - lo : 0ull;
     }
     __syncthreads();
-    const unsigned long long S = block_scan(tmp, m + 1, part);
-    for (int i = t; i <= m; i += kPrepThreads) w->s_pre[i] = tmp[i];
+    const unsigned long long H = block_scan(hv, ngap, part);
+    const unsigned long long S = block_scan(sv, nb, part);
+    for (int i = t; i < ngap; i += kPrepThreads) w->h_pre[i] = hv[i];
+    for (int i = t; i < nb; i += kPrepThreads) w->s_pre[i] = sv[i];
     if (t == 0) {
-        w->h_pre[m] = H;
-        w->s_pre[m + 1] = S;
-        w->nh = (unsigned long long)m;
-        w->ns = (unsigned long long)m + 1;
+        w->h_pre[ngap] = H;
+        w->s_pre[nb] = S;
+        w->nh = (unsigned long long)ngap;
+        w->ns = (unsigned long long)nb;
         // (H == S by construction; T > cap_e: the output overflowed, the caller re-runs staged)
         w->moved = (T <= cap_e && H == S) ? H : 0ull;
         *d_total = T;
@@ -151,17 +136,19 @@ __device__ __forceinline__ unsigned long long seg_of(const unsigned long long *p
 
 __global__ void __launch_bounds__(256) compact_copy_kernel(uint4 *out, const uint4 *scratch, unsigned long long cap_e,
                                                            const CompactWs *w) {
-    // each thread moves a contiguous run of records (2 pairs each: every gap and segment is
-    // even), locating its first hole and source once and walking the segments from there
+    // each warp moves a contiguous run of records (2 pairs each: every gap and segment is even),
+    // its lanes 32 consecutive records per step (coalesced 16-B loads and stores); a lane locates
+    // its first hole and source once and walks the segments from there
     const unsigned long long recs = w->moved / 2;
-    const unsigned long long nth = (unsigned long long)gridDim.x * blockDim.x;
-    const unsigned long long per = (recs + nth - 1) / nth;
-    const unsigned long long r0 = ((unsigned long long)blockIdx.x * blockDim.x + threadIdx.x) * per;
-    const unsigned long long r1 = min(recs, r0 + per);
+    const unsigned long long nw = (unsigned long long)gridDim.x * blockDim.x / 32;
+    const unsigned long long per = ((recs + nw - 1) / nw + 31) / 32 * 32;
+    const unsigned long long gw = ((unsigned long long)blockIdx.x * blockDim.x + threadIdx.x) / 32;
+    const unsigned long long r0 = gw * per + (threadIdx.x & 31);
+    const unsigned long long r1 = min(recs, gw * per + per);
     if (r0 >= r1) return;
     const unsigned long long nh = w->nh, ns = w->ns;
     unsigned long long hj = seg_of(w->h_pre, nh, 2 * r0), sj_ = seg_of(w->s_pre, ns, 2 * r0);
-    for (unsigned long long r = r0; r < r1; ++r) {
+    for (unsigned long long r = r0; r < r1; r += 32) {
         const unsigned long long p = 2 * r;
         while (w->h_pre[hj + 1] <= p) ++hj;  // next non-empty hole / source
         while (w->s_pre[sj_ + 1] <= p) ++sj_;
@@ -190,11 +177,11 @@ int compact_output(const JoinArgs &a, int blocks, unsigned long long *d_total, v
     static bool attr = false;
     if (!attr) {
         SJ_CUDA_TRY(cudaFuncSetAttribute(compact_prep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         3 * (kMaxGaps + 2) * (int)sizeof(unsigned long long)));
+                                         2 * (kMaxGaps + 2) * (int)sizeof(unsigned long long)));
         attr = true;
     }
-    compact_prep_kernel<<<1, kPrepThreads, 3 * (kMaxGaps + 2) * sizeof(unsigned long long), s>>>(
-        a.gaps, nwarps, a.emit_ctr, cap_e, w, d_total);
+    compact_prep_kernel<<<1, kPrepThreads, 2 * (kMaxGaps + 2) * sizeof(unsigned long long), s>>>(
+        a.gaps, nwarps, a.emit_ctr, a.blk, cap_e, w, d_total);
     note_launch();
     compact_copy_kernel<<<148 * 4, 256, 0, s>>>(reinterpret_cast<uint4 *>(a.out),
                                                reinterpret_cast<const uint4 *>(a.scratch), cap_e, w);

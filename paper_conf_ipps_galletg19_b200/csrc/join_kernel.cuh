@@ -255,21 +255,16 @@ __device__ __forceinline__ double sqdist(const double (&q)[DIM], const double (&
     return s;
 }
 
-// Flush a warp's staged hits: ONE atomicAdd reserves the output slots, then the lanes write
-// coalesced streaming stores: both mirrored pairs of a hit as one 16-B store {q, c, c, q}
-// (half patterns), or the single pair {q, c} (GCG, which meets every pair twice).
-// Exact sizing (kExact): the slots come from the chunk's own cursor instead, so the output
-// order is deterministic; the counter still totals the pairs.
 // Flush a warp's staged hits and return how many stay buffered (0, or the rest of a flush that
 // filled its output block).  The lanes write coalesced streaming stores: both mirrored pairs of a
 // hit as one 16-B store {q, c, c, q} (half patterns), or the single pair {q, c} (GCG, which
 // meets every pair twice).  The output slots:
 //   * default: ONE atomicAdd on the output counter per flush;
-//   * blocked output (JoinArgs::blk, half patterns, kPairs): from the CTA's current block, under
-//     the CTA's lock; a block is taken with ONE atomicAdd of blk per block and CTA.  A flush that
-//     does not fit in its block's rest fills the rest and keeps the other hits buffered (moved to
-//     the buffer's front) for the next flush, which starts a new block -- so every block but each
-//     CTA's last is full and the one write loop stays a single contiguous segment;
+//   * blocked output (JoinArgs::blk, half patterns, kPairs): from the warp's current block; a
+//     block is taken with ONE atomicAdd of blk per block and warp.  A flush that does not fit in
+//     its block's rest fills the rest and keeps the other hits buffered (moved to the buffer's
+//     front) for the next flush, which starts a new block -- so every block but each warp's last
+//     is full and the one write loop stays a single contiguous segment;
 //   * exact sizing (kExact): the chunk's own cursor, so the output order is deterministic; the
 //     counter still totals the pairs.
 // Positions from cap_e = out_cap & ~1 on go to the scratch buffer of a blocked launch
@@ -778,7 +773,9 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
 // home-cell positions tb.. and a (query, slot) pair is inside the query's half scan (reading c8)
 // iff (p - rr - 1) mod m < home_count(m, rr) -- HOME = 1, the circulant windows of cells of
 // <= 32 points -- or iff p > rr -- HOME = 2, the upper triangle of larger cells.
-template <int DIM, int K, int MODE, bool GCG, int HOME>
+// FULL (1-D..3-D register path): the tile holds 32 candidates and every round 32/k queries, so
+// no slot or query validity is tested (the dense cells' common case).
+template <int DIM, int K, int MODE, bool GCG, int HOME, bool FULL = false>
 __device__ __forceinline__ unsigned tile_rounds(const JoinArgs &a, unsigned nq, unsigned nt, unsigned tb, unsigned m,
                                                 WarpSmem<DIM, MODE> &ws, int b, int &nbuf, unsigned long long &nhits,
                                                 int lane, unsigned lt, unsigned r_start) {
@@ -807,14 +804,14 @@ __device__ __forceinline__ unsigned tile_rounds(const JoinArgs &a, unsigned nq, 
 #pragma unroll
         for (int s = 0; s < SPL; ++s) {
             const unsigned j = t + (unsigned)(K * s);
-            cv[s] = j < nt;
+            cv[s] = FULL || j < nt;
             load_smem_point<DIM>(tile + (j & 31) * PAD, cp[s]);
             co[s] = tile_orig[j & 31];
         }
         for (unsigned r0 = r_start; r0 < nq; r0 += QPW) {
             if (needs_flush<DIM, MODE>(ws.buf, nbuf, 32 * SPL, lane)) return r0;  // the caller flushes
             const unsigned qi = (r0 + grp) & 31;
-            const bool qv = r0 + grp < nq;
+            const bool qv = FULL || r0 + grp < nq;
             double qq[DIM];
             load_smem_point<DIM>(ws.qry + qi * PAD, qq);
             const unsigned oq = ws.qorig[qi];
@@ -1072,8 +1069,13 @@ __device__ __forceinline__ void tiled_chunk(const JoinArgs &a, unsigned s0, unsi
         else
             cp_async_wait<0>();
         __syncwarp();
+        const unsigned nt = min(32u, S - tb);
+        const bool full = DIM <= 3 && nt == 32u && nq % (32u / K) == 0u;
         for (unsigned r = 0; r < nq;) {  // (the rounds return to flush the buffer)
-            r = tile_rounds<DIM, K, MODE, GCG, 0>(a, nq, min(32u, S - tb), tb, m, ws, it & 1, nbuf, nhits, lane, lt, r);
+            if (full)
+                r = tile_rounds<DIM, K, MODE, GCG, 0, true>(a, nq, nt, tb, m, ws, it & 1, nbuf, nhits, lane, lt, r);
+            else
+                r = tile_rounds<DIM, K, MODE, GCG, 0>(a, nq, nt, tb, m, ws, it & 1, nbuf, nhits, lane, lt, r);
             if (r < nq) flush_now<DIM, MODE, GCG>(ws.buf, nbuf, a, lane, &ws.ctl);
         }
         __syncwarp();

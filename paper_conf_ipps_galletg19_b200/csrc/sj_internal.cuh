@@ -228,10 +228,10 @@ struct JoinArgs {
     unsigned long long out_cap;   // capacity of out in pairs
     unsigned long long *calcs;    // instrumented distance calculations, or nullptr
     // kPairs, mirrored patterns: the output space is taken in BLOCKS of blk pairs, one atomic
-    // on emit_ctr per block and CTA (the warps of a CTA share its current block), instead of
-    // one per warp flush -- a single counter taking every flush congests its L2 slice and halves
-    // the join (measured).  Each CTA's last block stays partly empty: its gap {start, length}
-    // goes to gaps[blockIdx.x] and compact_output() closes the gaps afterwards.  Positions from
+    // on emit_ctr per block and warp, instead of one per warp flush -- a single counter taking
+    // every flush congests its L2 slice and halves the join (measured).  Each warp's last block
+    // stays partly empty: its gap {start, length} goes to gaps[global warp index] and
+    // compact_output() closes the gaps afterwards.  Positions from
     // out_cap & ~1 on go to scratch (scratch_cap pairs).  blk = 0: one atomic per flush.
     unsigned long long blk;
     unsigned long long *gaps;
@@ -264,11 +264,11 @@ enum JoinMode : int { kCount = 0, kPairs = 1, kRows = 2, kDegree = 3, kChunkCoun
 
 // Launch the join kernel for dim/k/mode (kRows / kDegree need the GCG pattern).
 int launch_join(const JoinArgs &a, int dim, int k, int mode, int blocks, cudaStream_t s);
-// After a blocked kPairs launch (JoinArgs::blk): move the pairs past the total into the CTAs'
+// After a blocked kPairs launch (JoinArgs::blk): move the pairs past the total into the warps'
 // gaps so the output is [0, total) again; total -> *d_total.  ws: device workspace of
 // compact_ws_bytes(blocks) bytes.  Two launches on s, no host round trip.
 size_t compact_ws_bytes(int blocks);
-constexpr int kCompactMaxWarps = 8192;  // warps (gaps) compact_output handles
+constexpr int kCompactMaxGaps = 8192;  // warps (gaps) compact_output handles
 int compact_output(const JoinArgs &a, int blocks, unsigned long long *d_total, void *ws, cudaStream_t s);
 // Max resident CTAs per SM of the join kernel configuration.
 int join_occupancy(int dim, int k, int mode, bool gcg, int *blocks_per_sm);

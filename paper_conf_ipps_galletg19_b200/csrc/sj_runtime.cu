@@ -159,10 +159,21 @@ constexpr int kMaxStreams = 8;
 constexpr int kHead = 16;
 constexpr int kTotal = 8;  // a blocked in-place join's pair total (compact_output)
 constexpr int kCtrWords = 24;
-// Blocked in-place output (JoinArgs::blk): pairs per CTA block.  One atomic per block and CTA
-// instead of one per warp flush; the CTAs' last blocks leave gaps that compact_output closes
-// (at most blocks * kOutBlk pairs to move, from a scratch of the same size past the buffer).
-constexpr unsigned long long kOutBlk = 4096;
+// Blocked in-place output (JoinArgs::blk): pairs per warp block.  One atomic per block and warp
+// instead of one per warp flush (~900 pairs); the warps' last blocks leave gaps that
+// compact_output closes (on average half a block per warp to move, from a scratch of one block
+// per warp past the buffer).  SJ_OUT_BLK (environment, even) overrides it for measurements.
+// (Blocks shared by the warps of a CTA -- a packed {block, offset} word in shared memory, one
+// shared atomic per flush -- were measured slower: C5 join 0.93 -> 1.06 ms.)
+constexpr unsigned long long kOutBlkDefault = 4096;
+static unsigned long long out_blk() {
+    static const unsigned long long v = [] {
+        const char *e = getenv("SJ_OUT_BLK");
+        const unsigned long long x = e ? strtoull(e, nullptr, 10) : 0ull;
+        return (x >= 1024 && x <= (1ull << 22) && x % 2 == 0) ? x : kOutBlkDefault;
+    }();
+    return v;
+}
 // pinned mailbox layout (uint64 words): [0, kCtrWords) counters; [48, 50) the build's tail;
 // [64 + 4 s, 64 + 4 s + 3) staged slot s's counters
 constexpr int kMailSlots = 64;
@@ -725,16 +736,17 @@ int run_in_place(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t v0, uint64_
 // the gaps array, the compaction workspace and the scratch, from one per-handle allocation.  Half
 // patterns only (GCG emits single pairs).  SJ_OPT_OUT_BLOCKS: 1 on, 0 off, 2 (default) on when
 // the caller's buffer holds at least kBlockedMinCap pairs (a large result: the output counter's
-// congestion doubles the join, measured on C5 eps 0.2; below it the compaction's fixed cost
-// outweighs it).
-constexpr uint64_t kBlockedMinCap = 1000000000ull;
+// congestion doubles the join, measured on C5 eps 0.2 every time and on C5 on some boxes -- 0.88
+// vs 1.3-1.4 ms, with blocks 0.93 on every box; below it the compaction's fixed cost (a prep
+// launch, ~15 us, and a copy of half a block per warp) outweighs the risk: C2 K64 0.28 vs 0.34).
+constexpr uint64_t kBlockedMinCap = 300000000ull;
 int blocked_out(sj_handle *h, JoinArgs &a, int blocks, uint64_t cap, bool *on) {
     *on = h->out_blocks == 1 || (h->out_blocks == 2 && cap >= kBlockedMinCap);
-    *on = *on && h->ix.pattern != SJ_PATTERN_GCG && blocks * (kJoinThreads / 32) <= kCompactMaxWarps;
+    *on = *on && h->ix.pattern != SJ_PATTERN_GCG && blocks * (kJoinThreads / 32) <= kCompactMaxGaps;
     if (!*on) return SJ_OK;
     const size_t gbytes = ((size_t)blocks * kJoinThreads / 32 * 16 + 255) & ~(size_t)255;  // a gap per warp
     const size_t wbytes = (compact_ws_bytes(blocks) + 255) & ~(size_t)255;
-    const size_t sbytes = (size_t)blocks * kJoinThreads / 32 * kOutBlk * 8;
+    const size_t sbytes = (size_t)blocks * kJoinThreads / 32 * out_blk() * 8;
     const size_t need = gbytes + wbytes + sbytes;
     if (h->outws_bytes < need) {
         dev_free(h->outws, h->s_main);
@@ -743,10 +755,10 @@ int blocked_out(sj_handle *h, JoinArgs &a, int blocks, uint64_t cap, bool *on) {
         SJ_TRY(dev_alloc(reinterpret_cast<void **>(&h->outws), need, h->s_main));
         h->outws_bytes = need;
     }
-    a.blk = kOutBlk;
+    a.blk = out_blk();
     a.gaps = reinterpret_cast<unsigned long long *>(h->outws);
     a.scratch = reinterpret_cast<uint32_t *>(h->outws + gbytes + wbytes);
-    a.scratch_cap = (unsigned long long)blocks * kJoinThreads / 32 * kOutBlk;
+    a.scratch_cap = (unsigned long long)blocks * kJoinThreads / 32 * out_blk();
     return SJ_OK;
 }
 

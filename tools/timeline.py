@@ -16,8 +16,12 @@ sys.path.insert(0, '.')
 import paper_conf_ipps_galletg19_b200 as sj  # noqa: E402
 import workloads  # noqa: E402
 
+import os  # noqa: E402
+
 cfg = workloads.get_config(sys.argv[1] if len(sys.argv) > 1 else 'c5')
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
+# extra Handle options for the timed steps, e.g. TL_KW="out_blocks=1"
+kw = {k: int(v) for k, v in (x.split('=') for x in os.environ.get('TL_KW', '').split(',') if x)}
 pts = cfg.points()
 d = torch.from_numpy(pts).cuda()
 h = sj.Handle(d, cfg.eps, k=cfg.k)
@@ -27,7 +31,7 @@ out = torch.empty((n, 2), dtype=torch.int32, device='cuda')
 
 
 def step():
-    hh = sj.Handle(d, cfg.eps, k=cfg.k)
+    hh = sj.Handle(d, cfg.eps, k=cfg.k, **kw)
     hh.self_join(out, n)
     st = hh.stats()
     hh.close()
