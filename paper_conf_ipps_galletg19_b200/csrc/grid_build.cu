@@ -162,16 +162,24 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
     unsigned bad = 0;
     const double2 *r2 = reinterpret_cast<const double2 *>(raw);
     const uint64_t pairs = total / 2;
-#pragma unroll 4
-    for (uint64_t e = t; e < pairs; e += T) {
-        const double2 v = __ldg(r2 + e);
+    auto take = [&](const double2 v) {
         bad |= !isfinite(v.x) | !isfinite(v.y);
         const unsigned long long k0 = ordered_key(v.x), k1 = ordered_key(v.y);
         mn0 = min(mn0, k0);
         mx0 = max(mx0, k0);
         mn1 = min(mn1, k1);
         mx1 = max(mx1, k1);
+    };
+    // four independent 16-B loads in flight per thread (a stride of T keeps the dimensions)
+    uint64_t e = t;
+    for (; e + 3 * T < pairs; e += 4 * T) {
+        const double2 v0 = __ldg(r2 + e), v1 = __ldg(r2 + e + T), v2 = __ldg(r2 + e + 2 * T), v3 = __ldg(r2 + e + 3 * T);
+        take(v0);
+        take(v1);
+        take(v2);
+        take(v3);
     }
+    for (; e < pairs; e += T) take(__ldg(r2 + e));
     if ((total & 1) && t == 0) {  // odd element count: the last double (dimension dim-1)
         const double x = raw[total - 1];
         bad |= !isfinite(x);
@@ -221,31 +229,49 @@ __global__ void __launch_bounds__(kThreads) bbox_kernel(const double *raw, uint6
 // One block per radix tile (kRadixTileKeys points): it also counts the tile's low 8-bit digits,
 // the first pass of the point sort (a4) -- its histogram kernel is not launched.  The sort's
 // values (input ids) are the identity, generated by its first scatter: not written here.
-constexpr int kCellIdThreads = 1024;  // 2 points per thread: the 6-D divisions need the parallelism
-__global__ void __launch_bounds__(kCellIdThreads) cell_id_kernel(const double *raw, uint64_t n,
+// threads per block: 1-D..3-D 512 (4 points per thread, loaded before any division), 4-D+ 1024
+// (2 points: their coordinates fill the registers, and the divisions need the parallelism)
+template <int DIM>
+struct CellIdThreads {
+    static constexpr int value = DIM <= 3 ? 512 : 1024;
+};
+template <int DIM>
+__global__ void __launch_bounds__(CellIdThreads<DIM>::value) cell_id_kernel(const double *raw, uint64_t n,
                                                            const GeomDev *__restrict__ gp, uint32_t *keys32,
                                                            unsigned long long *keys64, GeomArgs ga,
                                                            uint32_t *hist0, uint32_t ntiles) {
+    constexpr int kCellIdThreads = CellIdThreads<DIM>::value;
+    constexpr int PPT = kRadixTileKeys / kCellIdThreads;
     __shared__ uint32_t h[256];
     if (threadIdx.x < 256) h[threadIdx.x] = 0;
     if (blockIdx.x == 0 && threadIdx.x == 0 && ga.host) publish_geometry(gp, ga);
     __syncthreads();
-    const int dim = gp->dim;
     const double w = gp->w;
     const bool ok = !gp->err, narrow = gp->key_bits <= 32;
-    const uint64_t base = (uint64_t)blockIdx.x * kRadixTileKeys;
+    double mins[DIM];
+    unsigned long long stride[DIM];
 #pragma unroll
-    for (int it = 0; it < kRadixTileKeys / kCellIdThreads; ++it) {
+    for (int d = 0; d < DIM; ++d) {
+        mins[d] = gp->mins[d];
+        stride[d] = gp->stride[d];
+    }
+    const uint64_t base = (uint64_t)blockIdx.x * kRadixTileKeys;
+    double x[PPT][DIM];
+#pragma unroll
+    for (int it = 0; it < PPT; ++it) {
+        const uint64_t i = base + (uint64_t)it * kCellIdThreads + threadIdx.x;
+#pragma unroll
+        for (int d = 0; d < DIM; ++d) x[it][d] = (i < n && ok) ? __ldg(raw + i * DIM + d) : 0.0;
+    }
+#pragma unroll
+    for (int it = 0; it < PPT; ++it) {
         const uint64_t i = base + (uint64_t)it * kCellIdThreads + threadIdx.x;
         if (i >= n || !ok) continue;
         unsigned long long lid = 0;
 #pragma unroll
-        for (int d = 0; d < SJ_MAX_DIM; ++d) {
-            if (d < dim) {
-                double q = __ddiv_rn(__dsub_rn(raw[i * dim + d], gp->mins[d]), w);
-                unsigned long long c = __double2ull_rd(q);
-                lid += c * gp->stride[d];
-            }
+        for (int d = 0; d < DIM; ++d) {
+            const double q = __ddiv_rn(__dsub_rn(x[it][d], mins[d]), w);
+            lid += __double2ull_rd(q) * stride[d];
         }
         if (narrow)
             keys32[i] = (uint32_t)lid;
@@ -1041,7 +1067,15 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     const uint32_t ntiles = (uint32_t)((n + kRadixTileKeys - 1) / kRadixTileKeys);
     uint32_t *hist0;  // the point sort's first-pass tile histogram, counted by the cell-id kernel
     SJ_TRY(tmp.alloc(&hist0, (uint64_t)256 * ntiles));
-    cell_id_kernel<<<ntiles, kCellIdThreads, 0, s>>>(d_raw, n, d_geo, keys32, keys64, ga, hist0, ntiles);
+    switch (dim) {
+#define SJ_CELL_ID(D)                                                                                          \
+    case D:                                                                                                    \
+        cell_id_kernel<D><<<ntiles, CellIdThreads<D>::value, 0, s>>>(d_raw, n, d_geo, keys32, keys64, ga, hist0, \
+                                                                     ntiles);                              \
+        break;
+        SJ_CELL_ID(1) SJ_CELL_ID(2) SJ_CELL_ID(3) SJ_CELL_ID(4) SJ_CELL_ID(5) SJ_CELL_ID(6) SJ_CELL_ID(7) SJ_CELL_ID(8)
+#undef SJ_CELL_ID
+    }
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     if (zero_copy) {
