@@ -15,7 +15,7 @@ for c in ${CFGS:-c5 c2k64 c3k64 c4k32 c5e02 c1 c2k16 c2k256 c3k256}; do
   timeout 300 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none --csv --log-file $OUT/ncu_${c}_build_metrics_all.csv python tools/step.py $c 1 > /dev/null 2>&1
   python tools/last_step_kernels.py $OUT/ncu_${c}_build_metrics_all.csv > $OUT/ncu_${c}_build_metrics.csv 2>/dev/null
 done
-python tools/r02_facts.py $OUT r02 > $OUT/facts.json 2>&1; cp profiles/ncu_facts.json $OUT/ncu_facts.json
+python tools/r02_facts.py $OUT r02/ev${EVTAG:-} > $OUT/facts.json 2>&1; cp profiles/ncu_facts.json $OUT/ncu_facts.json
 timeout 900 python bench.py --json-out $OUT/bench.jsonl 2>$OUT/bench.err | tail -1
 for c in ${BCFGS:-c2k64 c3k64 c4k32 c5e02 c1 c2k16 c2k256 c3k256}; do
   timeout 600 python bench.py --config $c --steps 30 --warmup 3 --e2e-steps 1 --batched-steps 2 --no-cpu-baseline --json-out $OUT/bench.jsonl 2>>$OUT/bench.err | tail -c 300
