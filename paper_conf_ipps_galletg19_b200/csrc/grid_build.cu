@@ -405,17 +405,20 @@ struct TotalsPub {
 //   D_alg = sum_A C(m_A, 2) + m_A * sum_{B in fwd(A)} m_B
 // Cell coordinates from a row-major linear id (c_0 most significant): n-1 divisions,
 // 32-bit when the whole grid has < 2^32 cells.
+// (DIM: the grid's dimensionality, a template parameter so each dimensionality's kernels carry
+// only their own loops)
+template <int DIM>
 __device__ __forceinline__ void decode_lid(unsigned long long lid, const FwdGeom &g, long long (&c)[SJ_MAX_DIM]) {
     if (g.small) {
         unsigned rem = (unsigned)lid;
 #pragma unroll
         for (int d = 0; d < SJ_MAX_DIM; ++d) {
-            if (d < g.dim - 1) {
+            if (d < DIM - 1) {
                 const unsigned st = (unsigned)g.stride[d];
                 const unsigned q = rem / st;
                 c[d] = q;
                 rem -= q * st;
-            } else if (d == g.dim - 1) {
+            } else if (d == DIM - 1) {
                 c[d] = rem;
             }
         }
@@ -423,11 +426,11 @@ __device__ __forceinline__ void decode_lid(unsigned long long lid, const FwdGeom
         unsigned long long rem = lid;
 #pragma unroll
         for (int d = 0; d < SJ_MAX_DIM; ++d) {
-            if (d < g.dim - 1) {
+            if (d < DIM - 1) {
                 const unsigned long long q = rem / g.stride[d];
                 c[d] = (long long)q;
                 rem -= q * g.stride[d];
-            } else if (d == g.dim - 1) {
+            } else if (d == DIM - 1) {
                 c[d] = (long long)rem;
             }
         }
@@ -450,21 +453,22 @@ struct CellPos {
     unsigned lo_mask, hi_mask, odd_mask;  // c_d == 0 / c_d == nc_d - 1 (d < last); c_d odd (all d)
 };
 
+template <int DIM>
 __device__ __forceinline__ CellPos cell_pos(unsigned long long lid, const FwdGeom &g) {
     long long c[SJ_MAX_DIM];
-    decode_lid(lid, g, c);
+    decode_lid<DIM>(lid, g, c);
     CellPos p;
     p.lid = lid;
     p.lo_mask = p.hi_mask = p.odd_mask = 0;
     p.clast = 0;
 #pragma unroll
     for (int d = 0; d < SJ_MAX_DIM; ++d) {
-        if (d < g.dim - 1) {
+        if (d < DIM - 1) {
             p.lo_mask |= (c[d] == 0 ? 1u : 0u) << d;
             p.hi_mask |= (c[d] == (long long)g.nc[d] - 1 ? 1u : 0u) << d;
         }
-        if (d < g.dim) p.odd_mask |= (unsigned)(c[d] & 1) << d;
-        if (d == g.dim - 1) p.clast = c[d];
+        if (d < DIM) p.odd_mask |= (unsigned)(c[d] & 1) << d;
+        if (d == DIM - 1) p.clast = c[d];
     }
     return p;
 }
@@ -472,6 +476,7 @@ __device__ __forceinline__ CellPos cell_pos(unsigned long long lid, const FwdGeo
 // The non-empty cells among the row's <= 3 cells (consecutive along the last dimension) have
 // consecutive ranks, so their points are one run [b, b+len) of the lid-ordered storage.  The
 // <= 3 lookups are issued together.
+template <int DIM>
 __device__ __forceinline__ bool eval_row(int j, const CellPos &cp, const FwdGeom &g, const Lookup &L,
                                          const uint32_t *cell_start, uint32_t &b, uint32_t &len) {
     const RowEnt e = g.rows_ent[j];
@@ -481,7 +486,7 @@ __device__ __forceinline__ bool eval_row(int j, const CellPos &cp, const FwdGeom
     const int lo = (int)(e.meta & 3u) - 1, hi = (int)((e.meta >> 2) & 3u) - 1;
     const long long x0 = cp.clast + lo;
     const int nx = hi - lo + 1;
-    const long long ncl = (long long)g.nc[g.dim - 1];
+    const long long ncl = (long long)g.nc[DIM - 1];
     const unsigned long long base = cp.lid + (unsigned long long)e.delta;
     uint32_t nb[3];
 #pragma unroll
@@ -505,7 +510,7 @@ __device__ __forceinline__ bool eval_row(int j, const CellPos &cp, const FwdGeom
 
 // a6 + a7 over the forward rows; LPC lanes per cell (1, or 32 when there are many rows:
 // 6-D has 122) so the independent lookups of a cell run in parallel.
-template <bool FILL, int LPC>
+template <int DIM, bool FILL, int LPC>
 __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long *cell_lid, const uint32_t *cell_start,
                                                         const uint64_t *d_M, FwdGeom g, Lookup L, uint32_t *rcnt,
                                                         uint32_t *wload, const uint32_t *rbegin, uint2 *runs,
@@ -522,7 +527,7 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
     uint32_t w = 0;
     if (!FILL && gt == 0) rcnt[M] = 0;  // the scan runs over M + 1 entries
     for (uint64_t r = gt / LPC; r < M; r += cstride) {  // uniform across the LPC lanes of a cell
-        const CellPos cp = cell_pos(cell_lid[r], g);
+        const CellPos cp = cell_pos<DIM>(cell_lid[r], g);
         const uint32_t m = cell_start[r + 1] - cell_start[r];
         // FILL: the compacted layout (rbegin = scan of the counts); counting with `runs` set: the
         // slot layout, cell r's runs at r * rows (no second pass, no scan)
@@ -537,7 +542,7 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
         for (int jb = 0; jb < g.rows; jb += LPC) {
             const int j = jb + (int)sub;
             uint32_t b = 0, len = 0;
-            const bool found = qcell && j < g.rows && eval_row(j, cp, g, L, cell_start, b, len);
+            const bool found = qcell && j < g.rows && eval_row<DIM>(j, cp, g, L, cell_start, b, len);
             if (FILL || runs) {
                 if (LPC == 1) {
                     if (found) runs[out++] = make_uint2(b, len);
@@ -1259,14 +1264,22 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     uint32_t *wk, *wv;
     SJ_TRY(tmp.alloc(&wk, n));
     SJ_TRY(tmp.alloc(&wv, n));
-    if (wide)
-        runs_kernel<false, 32><<<runs_grid(n, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                    nullptr, slots ? ix.runs : nullptr, d_tot, pub,
-                                                                    wk, wv);
-    else
-        runs_kernel<false, 1><<<runs_grid(n, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt, wload,
-                                                                  nullptr, slots ? ix.runs : nullptr, d_tot, pub,
-                                                                  wk, wv);
+    // (per dimensionality: the counting pass's per-cell loops are the build's ALU work)
+#define SJ_RUNS_COUNT(D, LPC)                                                                                  \
+    runs_kernel<D, false, LPC><<<runs_grid(n, LPC), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, rcnt,     \
+                                                                      wload, nullptr, slots ? ix.runs : nullptr, \
+                                                                      d_tot, pub, wk, wv)
+#define SJ_RUNS_COUNT_D(D)         \
+    case D:                        \
+        if (wide)                  \
+            SJ_RUNS_COUNT(D, 32);  \
+        else                       \
+            SJ_RUNS_COUNT(D, 1);   \
+        break;
+    switch (dim) { SJ_RUNS_COUNT_D(1) SJ_RUNS_COUNT_D(2) SJ_RUNS_COUNT_D(3) SJ_RUNS_COUNT_D(4) SJ_RUNS_COUNT_D(5)
+                   SJ_RUNS_COUNT_D(6) SJ_RUNS_COUNT_D(7) SJ_RUNS_COUNT_D(8) }
+#undef SJ_RUNS_COUNT_D
+#undef SJ_RUNS_COUNT
     note_launch();
     SJ_CUDA_TRY(cudaGetLastError());
     uint32_t *rbegin = nullptr;
@@ -1332,14 +1345,24 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     }
     if (slots) {
         // (the counting pass wrote them)
-    } else if (wide)
-        runs_kernel<true, 32><<<runs_grid(M, 32), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
-                                                                    rbegin, ix.runs, nullptr, TotalsPub{}, nullptr,
-                                                                    nullptr);
-    else
-        runs_kernel<true, 1><<<runs_grid(M, 1), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr, nullptr,
-                                                              rbegin, ix.runs, nullptr, TotalsPub{}, nullptr, nullptr);
-    note_launch();
+    } else {
+#define SJ_RUNS_FILL(D, LPC)                                                                                   \
+    runs_kernel<D, true, LPC><<<runs_grid(M, LPC), kThreads, 0, s>>>(cell_lid, cell_start, d_M, fg, L, nullptr,  \
+                                                                     nullptr, rbegin, ix.runs, nullptr,        \
+                                                                     TotalsPub{}, nullptr, nullptr)
+#define SJ_RUNS_FILL_D(D)         \
+    case D:                       \
+        if (wide)                 \
+            SJ_RUNS_FILL(D, 32);  \
+        else                      \
+            SJ_RUNS_FILL(D, 1);   \
+        break;
+        switch (dim) { SJ_RUNS_FILL_D(1) SJ_RUNS_FILL_D(2) SJ_RUNS_FILL_D(3) SJ_RUNS_FILL_D(4) SJ_RUNS_FILL_D(5)
+                       SJ_RUNS_FILL_D(6) SJ_RUNS_FILL_D(7) SJ_RUNS_FILL_D(8) }
+#undef SJ_RUNS_FILL_D
+#undef SJ_RUNS_FILL
+        note_launch();
+    }
     SJ_CUDA_TRY(cudaGetLastError());
 
     // ---- a8: SortByWL over cells -> D' (queue of points in non-increasing W)
