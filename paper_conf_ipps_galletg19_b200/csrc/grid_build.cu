@@ -829,15 +829,22 @@ int forward_offsets_public(int dim, int8_t *out, uint64_t cap) {
 }
 
 void free_index(Index &ix, cudaStream_t s) {
-    dev_free(ix.d_meta, s);
+    if (ix.block) {  // one allocation holds every array but (possibly) the runs
+        dev_free(ix.block, s);
+        if (ix.runs_own) dev_free(ix.runs, s);
+    } else {
+        dev_free(ix.d_meta, s);
+        dev_free(ix.pts, s);
+        dev_free(ix.orig, s);
+        dev_free(ix.qmap, s);
+        dev_free(ix.cellq, s);
+        dev_free(ix.runs, s);
+        dev_free(ix.cell_lid, s);
+        dev_free(ix.chunks, s);
+    }
+    ix.block = nullptr;
+    ix.runs_own = true;
     ix.d_meta = nullptr;
-    dev_free(ix.pts, s);
-    dev_free(ix.orig, s);
-    dev_free(ix.qmap, s);
-    dev_free(ix.cellq, s);
-    dev_free(ix.runs, s);
-    dev_free(ix.cell_lid, s);
-    dev_free(ix.chunks, s);
     ix.chunks = nullptr;
     ix.pts = nullptr;
     ix.orig = nullptr;
@@ -1159,8 +1166,42 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         SJ_TRY(rle<uint64_t>(ks, n, cellof, cell_lid, cell_start, d_M, s, &tmp.ws, tab));
     }
     // the gather of the points into cell order needs only the point sort: side stream
-    SJ_TRY(dev_alloc_t(&ix.pts, n * ix.pad, s));
-    SJ_TRY(dev_alloc_t(&ix.orig, n, s));
+    // the index arrays: one allocation, each array at its bound (M <= n cells); the slot-layout
+    // runs (n * rows entries, up to 4 GB) join it when they fit the slot bound
+    std::vector<uint64_t> rows;
+    const int R = pattern_rows(dim, ix.pattern, rows);
+    const bool slots = (uint64_t)n * R * sizeof(uint2) <= (4ull << 30);
+    {
+        auto al = [](size_t b) { return (b + 255) & ~(size_t)255; };
+        const size_t b_pts = al(n * ix.pad * sizeof(double)), b_orig = al(n * sizeof(uint32_t)),
+                     b_qmap = al(n * sizeof(uint2)), b_cellq = al(n * sizeof(uint4)),
+                     b_lid = al(n * sizeof(uint64_t)), b_chunks = al((n + 1 + kChunkPad) * sizeof(uint32_t)),
+                     b_meta = al(4 * sizeof(uint32_t)),
+                     b_runs = slots ? al(((uint64_t)n * R + 2) * sizeof(uint2)) : 0;
+        char *blk = nullptr;
+        SJ_TRY(dev_alloc(reinterpret_cast<void **>(&blk),
+                         b_pts + b_orig + b_qmap + b_cellq + b_lid + b_chunks + b_meta + b_runs, s));
+        ix.block = blk;
+        ix.pts = reinterpret_cast<double *>(blk);
+        blk += b_pts;
+        ix.orig = reinterpret_cast<uint32_t *>(blk);
+        blk += b_orig;
+        ix.qmap = reinterpret_cast<uint2 *>(blk);
+        blk += b_qmap;
+        ix.cellq = reinterpret_cast<uint4 *>(blk);
+        blk += b_cellq;
+        ix.cell_lid = reinterpret_cast<uint64_t *>(blk);
+        blk += b_lid;
+        ix.chunks = reinterpret_cast<uint32_t *>(blk);
+        blk += b_chunks;
+        ix.d_meta = reinterpret_cast<uint32_t *>(blk);
+        blk += b_meta;
+        if (slots) {
+            ix.runs = reinterpret_cast<uint2 *>(blk);
+            ix.runs_cap = (uint64_t)n * R + 2;
+            ix.runs_own = false;
+        }
+    }
     cudaStream_t sg = side ? side->s2 : s;
     if (side) {
         SJ_CUDA_TRY(cudaEventRecord(side->ea, s));
@@ -1186,9 +1227,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     }
     SJ_CUDA_TRY(cudaGetLastError());
 
-    // ---- a6 + a7: forward runs, workload, D_alg
-    std::vector<uint64_t> rows;
-    const int R = pattern_rows(dim, ix.pattern, rows);
+    // ---- a6 + a7: forward runs, workload, D_alg (rows R: above)
     // the rows resolved against this grid: linear-id delta, edge masks, meta (eval_row)
     std::vector<RowEnt> ents(R);
     for (int j = 0; j < R; ++j) {
@@ -1239,11 +1278,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     // Slot layout: cell r's runs at r * R, written by the counting pass itself -- no scan, no
     // second pass, no third host round trip; the array is sized by n >= M before M is known
     // (up to 4 GB of the 180 GB: every configuration, 6-D at 2M points included: 1.95 GB).
-    const bool slots = (uint64_t)n * R * sizeof(uint2) <= (4ull << 30);
-    if (slots) {
-        ix.runs_cap = (uint64_t)n * R + 2;
-        SJ_TRY(dev_alloc_t(&ix.runs, ix.runs_cap, s));
-    }
+    // (slots: the runs are part of the index block, allocated above)
     // grid-stride kernels (M is on the device): at most 8 resident blocks per SM
     int nsm = 148;
     {
@@ -1318,7 +1353,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     ix.max_w = bt.max_w;
     // persistent device words {n_chunks, E}: the join reads the chunk count from here (a
     // device-sized launch needs no host round trip after the build)
-    SJ_TRY(dev_alloc_t(&ix.d_meta, 4, s));
+    // (d_meta: part of the index block)
     uint32_t *d_E32 = ix.d_meta + 1;
     if (!slots) SJ_TRY(scan_exclusive_u32(rcnt, rbegin, M + 1, d_E32, s, &tmp.ws));
     // The runs array is allocated at its bound M * rows when that is small (every 1-D..4-D
@@ -1380,9 +1415,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     SJ_TRY(tmp.alloc(&qb, M));
 
     // ---- final arrays
-    SJ_TRY(dev_alloc_t(&ix.cellq, M, s));
-    SJ_TRY(dev_alloc_t(&ix.cell_lid, M, s));
-    SJ_TRY(dev_alloc_t(&ix.qmap, n, s));
+    // (cellq, cell_lid, qmap: part of the index block)
     uint32_t *r2q, *qbr;
     SJ_TRY(tmp.alloc(&r2q, M));
     SJ_TRY(tmp.alloc(&qbr, M));
@@ -1407,7 +1440,7 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
 
     // ---- WorkQueue chunks over D'
     uint32_t *d_nc = ix.d_meta;
-    SJ_TRY(dev_alloc_t(&ix.chunks, n + 1 + kChunkPad, s));
+    // (chunks: part of the index block)
     // in input order a cell's points are scattered: no chunk may claim a cell
     const uint32_t big_min = ix.order == SJ_ORDER_INPUT ? 0xFFFFFFFFu : kBigCell;
     if (ix.order == SJ_ORDER_INPUT)

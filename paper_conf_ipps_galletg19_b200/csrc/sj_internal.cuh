@@ -167,6 +167,10 @@ struct Index {
     uint64_t runs_cap = 0;      // entries allocated for runs (>= E + 2)
     uint64_t runs_len = 0;      // entries the cells' run indices span: M * rows in the slot
                                 // layout (cell r's runs at r * rows), 0 = compact (E)
+    // the build's arrays carved from ONE stream-ordered allocation (bounds from n: M <= n), so a
+    // build and a destroy cost one allocation call each; runs are outside it when runs_own
+    void *block = nullptr;
+    bool runs_own = true;
 };
 inline uint64_t runs_entries(const Index &ix) { return ix.runs_len ? ix.runs_len : ix.n_runs; }
 

@@ -273,6 +273,8 @@ struct Core {
     sj::BuildSide side;
     unsigned long long *d_ctr;
     uint64_t *mail;
+    char *outws;  // the blocked output's workspace (gaps, compaction, scratch), kept with the core
+    size_t outws_bytes;
 };
 std::mutex g_core_mu;
 std::vector<Core> g_core_cache;
@@ -298,6 +300,8 @@ int handle_init_common(sj_handle *h) {
                 h->side = c.side;
                 h->d_ctr = c.d_ctr;
                 h->mail = c.mail;
+                h->outws = c.outws;
+                h->outws_bytes = c.outws_bytes;
                 return SJ_OK;
             }
     }
@@ -343,7 +347,9 @@ bool core_release(sj_handle *h) {
     std::lock_guard<std::mutex> lk(g_core_mu);
     if (g_core_cache.size() >= 64) return false;
     g_core_cache.push_back(Core{h->device, h->num_sms, h->s_main, {h->ev_a, h->ev_b, h->ev_c, h->ev_d, h->ev_e, h->ev_ba, h->ev_bb, h->ev_in}, h->side, h->d_ctr,
-                                h->mail});
+                                h->mail, h->outws, h->outws_bytes});
+    h->outws = nullptr;
+    h->outws_bytes = 0;
     return true;
 }
 
@@ -1420,10 +1426,10 @@ void sj_destroy(sj_handle *h) {
     cudaSetDevice(h->device);
     slots_release(h);
     if (h->s_main) dev_free(h->d_voff, h->s_main);
-    if (h->s_main) dev_free(h->outws, h->s_main);
     if (h->s_main && h->owns_index) free_index(h->ix, h->s_main);  // stream-ordered frees
-    if (!core_release(h)) {
+    if (!core_release(h)) {  // (a released core keeps the blocked output's workspace)
         if (h->s_main) {
+            dev_free(h->outws, h->s_main);
             cudaStreamSynchronize(h->s_main);
             dev_free(h->d_ctr, h->s_main);
             cudaStreamSynchronize(h->s_main);
