@@ -60,14 +60,6 @@ constexpr int kBufHitsHi = SJ_BUF_HI;
 // A cell segment of >= 2 queries is tiled when its forward list has at least this many
 // candidates (6-D: ~1300 per cell of ~4 points), so staging pays for itself.
 constexpr unsigned kTileMinCand = 128;
-// Column emission buffers (1-D..3-D pair modes, see flush_cols): kColRows hits per lane,
-// rows kColPitch = 33 entries apart so that reading one column down its rows (the flush)
-// walks the shared-memory banks instead of hitting one bank pair 32 times.
-constexpr int kColRows = 16;
-constexpr int kColPitch = 33;
-#ifndef SJ_COLS
-#define SJ_COLS 0  // measured slower than the ballot-ranked buffer on B200 (C5 join +40 %)
-#endif
 
 template <int DIM>
 struct PointPad {
@@ -165,7 +157,7 @@ struct WarpSmem {
     uint2 runs_s[(DIM >= 4 && DIM <= 6) ? 128 : 1];
     // hits buffered before a flush: fewer in high dimensions (few hits per calculation,
     // and the smaller footprint buys occupancy)
-    alignas(16) uint2 buf[Mode<MODE>::pairs ? ((SJ_COLS && DIM <= 3) ? kColRows * kColPitch : BufCap<DIM>::value) : 2];
+    alignas(16) uint2 buf[Mode<MODE>::pairs ? BufCap<DIM>::value : 2];
     WarpCtl ctl;
     unsigned snext;  // SortByWL only (static assignment): this warp's next chunk index
     // kRows: the segment's per-query row cursors; kDegree: their running neighbour counts
@@ -340,87 +332,6 @@ __device__ __forceinline__ int flush(uint2 *buf, int nbuf, const JoinArgs &a, in
     return 0;
 }
 
-// 1-D..3-D pair modes: COLUMN buffers.  Lane l appends its own hits to column l of the warp's
-// buffer (hit r of lane l at buf[r*kColPitch + l]) with one predicated shared store, so an evaluation
-// step costs no warp vote; a flush ranks the columns with one warp scan, reserves the output
-// slots with ONE atomicAdd and writes coalesced 16-byte streaming stores -- output position o
-// finds its column by a 5-step binary search over the columns' exclusive offsets.  (In 4-D+
-// hits are rare (~2 % of the calculations) and the ballot-ranked buffer below skips hit-free
-// steps with one vote; there the column fill would force frequent flushes.)
-template <int DIM, int MODE>
-struct Cols {
-    static constexpr bool value = SJ_COLS && Mode<MODE>::pairs && DIM <= 3;
-};
-
-//
-// In the column modes the per-lane `nbuf` is the shared-memory ADDRESS of the lane's next
-// column slot (column base + kColPitch * 8 B per buffered hit), so appending a hit is one predicated
-// st.shared plus one add.
-__device__ __forceinline__ unsigned col_base(const uint2 *buf, int lane) {
-    return (unsigned)__cvta_generic_to_shared(buf) + 8u * (unsigned)lane;
-}
-
-template <bool GCG, bool EXACT>
-__device__ __forceinline__ void flush_cols(const uint2 *buf, int &nbuf, const JoinArgs &a, int lane,
-                                           WarpCtl *wc) {
-    __syncwarp();
-    const unsigned col0 = col_base(buf, lane);
-    const int cnt = (int)(((unsigned)nbuf - col0) / (8u * kColPitch));
-    int incl = cnt;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int v = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += v;
-    }
-    const int excl = incl - cnt;
-    const unsigned total = (unsigned)__shfl_sync(kFull, incl, 31);
-    constexpr unsigned long long kPer = GCG ? 1ull : 2ull;  // pairs per buffered hit
-    unsigned long long base = 0;
-    if (lane == 0) {
-        base = atomicAdd(a.emit_ctr, kPer * (unsigned long long)total);
-        wc->wtot += (unsigned long long)total;
-        if (EXACT) {
-            base = wc->wcur;
-            wc->wcur = base + kPer * (unsigned long long)total;
-        } else if (base + kPer * (unsigned long long)total > a.out_cap) {
-            wc->wcur = 1;  // overflow: stop dequeuing
-        }
-    }
-    base = __shfl_sync(kFull, base, 0);
-    const bool fits = base + kPer * (unsigned long long)total <= a.out_cap;
-    uint2 *out2 = reinterpret_cast<uint2 *>(a.out);
-    uint4 *out4 = reinterpret_cast<uint4 *>(a.out) + (base >> 1);  // base is even (mirrored modes)
-    for (unsigned o0 = 0; o0 < total; o0 += 32) {
-        const int o = (int)o0 + lane;
-        int l = 0, el = 0;  // the last column whose exclusive offset is <= o
-#pragma unroll
-        for (int st = 16; st > 0; st >>= 1) {
-            const int e = __shfl_sync(kFull, excl, l + st);
-            if (e <= o) {
-                l += st;
-                el = e;
-            }
-        }
-        if ((unsigned)o < total) {
-            uint2 v;  // {orig q, orig c}; volatile asm: ordered after the column stores
-            asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n"
-                         : "=r"(v.x), "=r"(v.y)
-                         : "r"((unsigned)__cvta_generic_to_shared(buf + (o - el) * kColPitch + l)));
-            if constexpr (GCG) {
-                if (fits || base + (unsigned long long)o < a.out_cap) __stcs(out2 + base + o, v);
-            } else {
-                const unsigned long long slot = base + 2ull * (unsigned long long)o;
-                if (fits || slot + 2 <= a.out_cap)
-                    __stcs(out4 + o, make_uint4(v.x, v.y, v.y, v.x));  // (q,c) and (c,q)
-                else if (slot < a.out_cap)
-                    __stcs(out2 + slot, make_uint2(v.x, v.y));
-            }
-        }
-    }
-    nbuf = (int)col0;
-    __syncwarp();
-}
-
 // Warp-aggregated emission of one evaluation step (all 32 lanes call it): the hits are
 // ranked with __ballot_sync/__popc into the warp's shared buffer.  Before each round the
 // caller makes room for the round's maximum number of hits (flush_if) instead of checking
@@ -431,12 +342,7 @@ __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *
                                      unsigned long long &nhits, unsigned lt, unsigned gbits,
                                      unsigned long long &cur, const JoinArgs &a, int lane) {
     constexpr bool RARE = DIM >= 4;
-    if constexpr (Cols<DIM, MODE>::value) {  // nbuf: shared address of this lane's next column slot
-        if (hit) {
-            asm volatile("st.shared.v2.u32 [%0], {%1, %2};\n" ::"r"(nbuf), "r"(oq), "r"(oc));
-            nbuf += 8 * kColPitch;
-        }
-    } else if constexpr (Mode<MODE>::pairs) {
+    if constexpr (Mode<MODE>::pairs) {
         const unsigned hm = __ballot_sync(kFull, hit);
         if (RARE && hm == 0u) return;  // high dimensions: most steps have no hit in the warp
         if (hit) buf[nbuf + __popc(hm & lt)] = make_uint2(oq, oc);
@@ -453,16 +359,12 @@ __device__ __forceinline__ void emit(bool hit, unsigned oq, unsigned oc, uint2 *
     }
 }
 
-// Make room before a round: `room` = the most hits the round can add to the warp (a multiple
-// of 32; a column gains at most room/32).
+// Make room before a round: `room` = the most hits the round can add to the warp.
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const JoinArgs &a, int lane,
                                          WarpCtl *wc) {
     constexpr int CAP = BufCap<DIM>::value;
-    if constexpr (Cols<DIM, MODE>::value) {
-        const unsigned lim = col_base(buf, lane) + 8u * kColPitch * (unsigned)(kColRows - room / 32);
-        if (__any_sync(kFull, (unsigned)nbuf > lim)) flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
-    } else if constexpr (Mode<MODE>::pairs) {
+    if constexpr (Mode<MODE>::pairs) {
         while (nbuf > CAP - room) nbuf = flush<GCG, Mode<MODE>::exact, Mode<MODE>::blocked>(buf, nbuf, a, lane, wc);
     }
 }
@@ -473,10 +375,7 @@ __device__ __forceinline__ void flush_if(uint2 *buf, int &nbuf, int room, const 
 template <int DIM, int MODE>
 __device__ __forceinline__ bool needs_flush(const uint2 *buf, int nbuf, int room, int lane) {
     constexpr int CAP = BufCap<DIM>::value;
-    if constexpr (Cols<DIM, MODE>::value) {
-        const unsigned lim = col_base(buf, lane) + 8u * kColPitch * (unsigned)(kColRows - room / 32);
-        return __any_sync(kFull, (unsigned)nbuf > lim);
-    } else if constexpr (Mode<MODE>::pairs) {
+    if constexpr (Mode<MODE>::pairs) {
         return nbuf > CAP - room;
     } else {
         return false;
@@ -484,9 +383,7 @@ __device__ __forceinline__ bool needs_flush(const uint2 *buf, int nbuf, int room
 }
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void flush_now(uint2 *buf, int &nbuf, const JoinArgs &a, int lane, WarpCtl *wc) {
-    if constexpr (Cols<DIM, MODE>::value) {
-        flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
-    } else if constexpr (Mode<MODE>::pairs) {
+    if constexpr (Mode<MODE>::pairs) {
         nbuf = flush<GCG, Mode<MODE>::exact, Mode<MODE>::blocked>(buf, nbuf, a, lane, wc);
     }
 }
@@ -495,10 +392,7 @@ __device__ __forceinline__ void flush_now(uint2 *buf, int &nbuf, const JoinArgs 
 template <int DIM, int MODE, bool GCG>
 __device__ __forceinline__ void flush_all(uint2 *buf, int &nbuf, const JoinArgs &a, int lane,
                                           WarpCtl *wc) {
-    if constexpr (Cols<DIM, MODE>::value) {
-        if (__any_sync(kFull, (unsigned)nbuf != col_base(buf, lane)))
-            flush_cols<GCG, Mode<MODE>::exact>(buf, nbuf, a, lane, wc);
-    } else if constexpr (Mode<MODE>::pairs) {
+    if constexpr (Mode<MODE>::pairs) {
         while (nbuf > 0) nbuf = flush<GCG, Mode<MODE>::exact, Mode<MODE>::blocked>(buf, nbuf, a, lane, wc);
     }
 }
@@ -1159,7 +1053,7 @@ __global__ void __launch_bounds__(kJoinThreads, MinBlocks<DIM>::value) join_kern
     const int warp = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     WarpSmem<DIM, MODE> &ws = reinterpret_cast<WarpSmem<DIM, MODE> *>(smem_raw)[warp];
-    int nbuf = Cols<DIM, MODE>::value ? (int)col_base(ws.buf, lane) : 0;  // column modes: see flush_cols
+    int nbuf = 0;  // hits in the warp's buffer (pair modes)
     unsigned long long nhits = 0;
     unsigned ncalcs = 0;  // this lane's distance calculations (instrumented runs; 32 bits per lane)
     // The batch: virtual chunks v_begin, v_begin + v_stride, ... < v_end (contiguous, or the
@@ -1209,7 +1103,7 @@ __global__ void __launch_bounds__(kJoinThreads, MinBlocks<DIM>::value) join_kern
             if (ib >= ws.ctl.vcount) ib = 0xFFFFFFFFu;
             // fused estimator (a9; v_begin 0, stride 1; the sample is whole dequeues): on the
             // first dequeue past the sample, this warp's hits so far all came from sample chunks
-            if (Mode<MODE>::inplace && !Cols<DIM, MODE>::value && !ws.ctl.sclosed && ib >= ws.ctl.sv1) {
+            if (Mode<MODE>::inplace && !ws.ctl.sclosed && ib >= ws.ctl.sv1) {
                 ws.ctl.samp = ws.ctl.wtot + (unsigned long long)nbuf;
                 ws.ctl.sclosed = 1;
             }
