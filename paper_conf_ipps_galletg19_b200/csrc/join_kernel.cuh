@@ -99,6 +99,15 @@ struct GStage {
 #ifndef SJ_FLAT_W
 #define SJ_FLAT_W 64  // flat path for chunks whose longest candidate list is <= this (0: off)
 #endif
+// flat path: independent (query, candidate) pairs per lane and step -- their candidate loads are
+// in flight together (measured: 2-D 4 (C2 K16 join 0.216 -> 0.201 ms), 3-D 2)
+#ifndef SJ_FLAT_U
+#define SJ_FLAT_U 0
+#endif
+template <int DIM>
+struct FlatU {
+    static constexpr int value = SJ_FLAT_U ? SJ_FLAT_U : DIM <= 2 ? 4 : 2;
+};
 // Flat path (flat_chunk): 1-D..3-D, half patterns, the pair / count modes.  runs = the
 // LID-UNICOMP forward runs per cell (pattern_rows()), staged per query.
 template <int DIM, int MODE, bool GCG>
@@ -558,7 +567,7 @@ __device__ __forceinline__ void generic_chunk(const JoinArgs &a, unsigned gmask,
 // Flat path for short candidate lists (the sparse tail of D', whose chunks hold queries of
 // small cells with similar W): the (query, candidate) pairs of all the chunk's generic queries
 // are numbered f = 0 .. T-1 (query by query, each query's list as in generic_chunk: forward runs,
-// then the home half scan) and lane l evaluates pairs l, l+32, ... -- two per step, independent,
+// then the home half scan) and lane l evaluates pairs l, l+32, ... -- FlatU per step, independent,
 // so their candidate loads are in flight together.  The k-lane rounds of generic_chunk instead
 // walk 32/k queries per round with a dependent global load chain each round, which is what the
 // sparse tail's time is made of (it is latency-bound, not issue-bound).  The queries' points,
@@ -611,12 +620,13 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
     if (!__all_sync(kFull, covered)) return false;
     ncalcs += W;
     unsigned long long cur = 0;
-    for (unsigned f0 = 0; f0 < T; f0 += 64) {
-        double qq[2][DIM], cp[2][DIM];
-        unsigned oq[2], oc[2];
-        bool ok[2];
+    constexpr int FU = FlatU<DIM>::value;
+    for (unsigned f0 = 0; f0 < T; f0 += 32 * FU) {
+        double qq[FU][DIM], cp[FU][DIM];
+        unsigned oq[FU], oc[FU];
+        bool ok[FU];
 #pragma unroll
-        for (int u = 0; u < 2; ++u) {
+        for (int u = 0; u < FU; ++u) {
             const unsigned fb = f0 + (unsigned)(u * 32), f = fb + (unsigned)lane;
             ok[u] = f < T;
             // the query of pair f: the r-th non-empty list, r = the non-empty lists starting at
@@ -653,12 +663,12 @@ __device__ __forceinline__ bool flat_chunk(const JoinArgs &a, unsigned gmask, ui
             load_smem_point<DIM>(ws.qry + q * PAD, qq[u]);
             oq[u] = ws.qorig[q];
         }
-        bool hit[2];
+        bool hit[FU];
 #pragma unroll
-        for (int u = 0; u < 2; ++u) hit[u] = ok[u] && sqdist<DIM>(qq[u], cp[u]) <= a.e2;
-        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 64, a, lane, &ws.ctl);
+        for (int u = 0; u < FU; ++u) hit[u] = ok[u] && sqdist<DIM>(qq[u], cp[u]) <= a.e2;
+        flush_if<DIM, MODE, GCG>(ws.buf, nbuf, 32 * FU, a, lane, &ws.ctl);
 #pragma unroll
-        for (int u = 0; u < 2; ++u) emit<DIM, MODE, GCG>(hit[u], oq[u], oc[u], ws.buf, nbuf, nhits, lt, kFull, cur, a, lane);
+        for (int u = 0; u < FU; ++u) emit<DIM, MODE, GCG>(hit[u], oq[u], oc[u], ws.buf, nbuf, nhits, lt, kFull, cur, a, lane);
     }
     return true;
 }
