@@ -639,8 +639,21 @@ __global__ void __launch_bounds__(kThreads) runs_kernel(const unsigned long long
 }
 
 // Empty chunks after the last one (kChunkPad): chunks[C + 1 + t] = the end of the queries.
-__global__ void __launch_bounds__(kThreads) chunk_pad_kernel(uint32_t *chunks, const uint32_t *d_nc, uint32_t end) {
-    chunks[*d_nc + 1u + blockIdx.x * kThreads + threadIdx.x] = end;
+// Also (block 0) the build's tail for the host -- the chunk count into the pinned mailbox
+// (zero-copy, no copy on the stream between the build and the join) -- and the join's counters
+// zeroed (the first join after sj_create launches without a memset of its own).
+__global__ void __launch_bounds__(kThreads) chunk_pad_kernel(uint32_t *chunks, const uint32_t *d_nc, uint32_t end,
+                                                             unsigned long long *tail_host,
+                                                             unsigned long long *zero_ctr, int zero_words) {
+    const uint32_t nc = *d_nc;
+    chunks[nc + 1u + blockIdx.x * kThreads + threadIdx.x] = end;
+    if (blockIdx.x == 0) {
+        if ((int)threadIdx.x < zero_words) zero_ctr[threadIdx.x] = 0ull;
+        if (threadIdx.x == 0 && tail_host) {
+            *reinterpret_cast<volatile unsigned long long *>(tail_host) = nc;
+            __threadfence_system();
+        }
+    }
 }
 
 // a8's queue cells, one fused scan (no count kernel, no separate finalize): load(i) = m of the
@@ -992,7 +1005,8 @@ static int rle(const K *ks, uint64_t n, uint32_t *cellof, unsigned long long *ce
 }
 
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s, cudaEvent_t ev0,
-                cudaEvent_t ev1, float *ms, const BuildPart *part, uint64_t *tail_mail, const BuildSide *side) {
+                cudaEvent_t ev1, float *ms, const BuildPart *part, uint64_t *tail_mail, const BuildSide *side,
+                unsigned long long *zero_ctr, int zero_words) {
     Temps tmp(s);
     // on every exit, the main stream waits for the side stream before the temporaries are freed
     // (stream-ordered, on s) -- also on the error returns
@@ -1449,8 +1463,11 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
     else
         SJ_TRY(scan_fused(M, CellChunkLoad{ix.cellq, qb, big_min}, CellChunkStore{ix.cellq, qb, big_min, ix.chunks}, s,
                           ChunkDone{nq, ix.chunks, d_nc}, &tmp.ws));
-    chunk_pad_kernel<<<kChunkPad / kThreads, kThreads, 0, s>>>(ix.chunks, d_nc,
-                                                                ix.order == SJ_ORDER_INPUT ? (uint32_t)n : (uint32_t)nq);
+    if (tail_mail) tail_mail[0] = tail_mail[1] = 0;
+    chunk_pad_kernel<<<kChunkPad / kThreads, kThreads, 0, s>>>(
+        ix.chunks, d_nc, ix.order == SJ_ORDER_INPUT ? (uint32_t)n : (uint32_t)nq,
+        (tail_mail && zero_copy) ? reinterpret_cast<unsigned long long *>(tail_mail) : nullptr, zero_ctr,
+        zero_ctr ? zero_words : 0);
     note_launch();
     if (side) {
         SJ_CUDA_TRY(cudaStreamWaitEvent(s, side->eq, 0));  // points, ids and D' complete
@@ -1458,10 +1475,10 @@ int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps,
         SJ_CUDA_TRY(cudaEventSynchronize(side->eg));
     }
     if (tail_mail) {
-        // no final round trip: {n_chunks, E} land in the caller's pinned mailbox, read once the
-        // stream has passed ev1 (the join reads n_chunks on the device meanwhile)
-        tail_mail[0] = tail_mail[1] = 0;
-        SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        // no final round trip: {n_chunks, E} land in the caller's pinned mailbox (n_chunks written
+        // by the pad kernel when the mailbox is device-mapped), read once the stream has passed
+        // ev1 (the join reads n_chunks on the device meanwhile)
+        if (!zero_copy) SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail, d_nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         if (bounded && !slots)  // E from the scan of the counts
             SJ_CUDA_TRY(cudaMemcpyAsync(tail_mail + 1, d_E32, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         else

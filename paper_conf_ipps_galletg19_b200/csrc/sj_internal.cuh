@@ -199,7 +199,9 @@ struct BuildSide {
 // Builds the index from device-resident raw points (n x dim AoS).  Returns sj_status.
 int build_index(Index &ix, const double *d_raw, uint64_t n, int dim, double eps, cudaStream_t s,
                 cudaEvent_t ev0, cudaEvent_t ev1, float *ms, const BuildPart *part = nullptr,
-                uint64_t *tail_mail = nullptr, const BuildSide *side = nullptr);
+                uint64_t *tail_mail = nullptr, const BuildSide *side = nullptr,
+                unsigned long long *zero_ctr = nullptr, int zero_words = 0);
+// zero_ctr: zero_words device words the build's last kernel zeroes (the join's counters).
 // tail_mail (pinned host, 2 words): the build ends without a host round trip; {n_chunks, E}
 // arrive there once the stream passes ev1, and ix.n_chunks / ix.n_runs / *ms stay unset
 // until the caller reads them (sj_runtime.cu: ix_ready).  nullptr: synchronous, all set.

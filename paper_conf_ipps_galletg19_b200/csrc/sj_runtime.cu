@@ -208,6 +208,7 @@ struct sj_handle {
     cudaEvent_t ev_in = nullptr;  // the caller's stream, recorded at entry (order_after_caller)
     sj::BuildSide side{};                         // the build's side stream and its events
     int pending = 0;  // 1: the build's tail {n_chunks, E} and its timing not read yet (ix_ready)
+    bool ctr_zeroed = false;  // the build's last kernel zeroed d_ctr (no join has used it since)
     sj::Index ix;
     bool owns_index = true;
     int num_sms = 148;
@@ -839,9 +840,9 @@ int run_in_place_est(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t sch, ui
 // device-sized launch (the kernel reads the chunk count the build left in ix.d_meta and sizes
 // the fused estimator's sample from it), so the GPU goes from the last build kernel straight
 // into the join.  *spairs = the sample's pairs, *total = all pairs emitted.
-int run_in_place_lazy(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *spairs, uint64_t *total) {
+int run_in_place_lazy(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *spairs, uint64_t *total, bool zeroed) {
     cudaStream_t s = h->s_main;
-    SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
+    if (!zeroed) SJ_CUDA_TRY(cudaMemsetAsync(h->d_ctr, 0, kCtrWords * sizeof(unsigned long long), s));
     SJ_CUDA_TRY(cudaEventRecord(h->ev_e, s));
     JoinArgs a = base_args(h);
     a.n_chunks = 0xFFFFFFFFu;      // bounded by the device-side V instead
@@ -981,8 +982,10 @@ int start_join(sj_handle *h, uint32_t *out, uint64_t cap, uint64_t *count) {
                       !getenv("SJ_DEBUG_VRANGE") && !getenv("SJ_SEPARATE_EST") &&
                       !(reinterpret_cast<uintptr_t>(out) & 15u);
     uint64_t lazy_spairs = 0, lazy_total = 0;
+    const bool zeroed = h->ctr_zeroed;  // (only the first join after the build finds them zeroed)
+    h->ctr_zeroed = false;
     if (lazy) {
-        SJ_TRY(run_in_place_lazy(h, out, cap, &lazy_spairs, &lazy_total));
+        SJ_TRY(run_in_place_lazy(h, out, cap, &lazy_spairs, &lazy_total, zeroed));
         debug_mark("join: lazy fast path");
     } else {
         SJ_TRY(ix_ready(h));
@@ -1355,7 +1358,9 @@ static sj_handle *create_impl(const double *points, uint64_t n, int dim, double 
     }();
     if (rc == SJ_OK)
         rc = build_index(h->ix, d_raw, n, dim, eps, s, h->ev_ba, h->ev_bb, &ms, origin ? &part : nullptr,
-                         sync_build ? nullptr : h->mail + 48, h->side.s2 ? &h->side : nullptr);
+                         sync_build ? nullptr : h->mail + 48, h->side.s2 ? &h->side : nullptr, h->d_ctr,
+                         kCtrWords);
+    h->ctr_zeroed = rc == SJ_OK;  // the build's last kernel zeroed the join's counters
     debug_mark("create: build_index");
     dev_free(d_copy, s);
     dev_free(d_ids, s);
