@@ -87,7 +87,9 @@ __global__ void __launch_bounds__(kPrepThreads) compact_prep_kernel(const unsign
     const unsigned long long A = *d_alloc;
     const unsigned long long T = A - G;
     const unsigned long long b0 = T / blk, b1 = (A + blk - 1) / blk;  // source blocks [b0, b1)
-    const int nb = (int)(b1 - b0);  // <= ngap + 1 (A - T = G < ngap * blk)
+    // <= ngap + 1: A - T = G < ngap * blk (a warp opens a block only to write into it); the clamp
+    // only guards the shared arrays -- a violation would leave H != S, and nothing is moved
+    const int nb = (int)min(b1 - b0, (unsigned long long)kMaxGaps + 1ull);
     // holes below T, in warp order; the source blocks' fill (blk unless a warp's last block)
     for (int i = t; i < ngap; i += kPrepThreads) {
         const unsigned long long st = gaps[2 * i], ln = gaps[2 * i + 1];
