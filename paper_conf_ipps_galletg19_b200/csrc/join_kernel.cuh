@@ -50,7 +50,13 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarps = kJoinThreads / 32;
-constexpr int kBufHits = 512;  // hits buffered per warp ({orig q, orig c}, 8 B -> 4 KB)
+// 1-D / 2-D: hits buffered per warp ({orig q, orig c}, 8 B each): 624 fills a warp's 7 KB share of
+// four CTAs per SM (measured against 512: fewer flushes, C5 0.914 -> 0.906 ms, C5 eps 0.2 2.90 ->
+// 2.85 ms; 600 was slower than both)
+#ifndef SJ_BUF2
+#define SJ_BUF2 624
+#endif
+constexpr int kBufHits = SJ_BUF2;
 #ifndef SJ_BUF_HI
 #define SJ_BUF_HI 96
 #endif
@@ -173,6 +179,8 @@ struct WarpSmem {
     unsigned long long qcur[(MODE == kRows || MODE == kDegree) ? 32 : 1];
 };
 static_assert(sizeof(WarpSmem<6, kPairs>) <= 7168, "6-D: four 256-thread CTAs per SM");
+static_assert(sizeof(WarpSmem<2, kPairsB>) <= 7168 && sizeof(WarpSmem<2, kPairs>) <= 7168,
+              "2-D: four 256-thread CTAs per SM");
 
 template <int DIM>
 __device__ __forceinline__ void load_point(const double *__restrict__ p, double (&x)[DIM]) {
