@@ -103,7 +103,8 @@ struct GStage {
     static constexpr int runs = !SJ_GSTAGE ? 0 : DIM == 3 ? 5 : 0;
 };
 #ifndef SJ_FLAT_W
-#define SJ_FLAT_W 64  // flat path for chunks whose longest candidate list is <= this (0: off)
+#define SJ_FLAT_W 128  // flat path for chunks whose longest candidate list is <= this (0: off;
+                       // measured 32 / 64 / 128 / 256: C3 K64 0.679 / 0.676 / 0.669 / 0.670 ms)
 #endif
 // flat path: independent (query, candidate) pairs per lane and step -- their candidate loads are
 // in flight together (measured: 2-D 4 (C2 K16 join 0.216 -> 0.201 ms), 3-D 2)
