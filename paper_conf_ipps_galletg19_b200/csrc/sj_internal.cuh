@@ -20,7 +20,10 @@ constexpr unsigned kChunk = 32;
 // Empty WorkQueue chunks written after the last one: a device-sized join (the host does not know
 // the chunk count yet) may dequeue past it by < grab * world chunks (the runtime checks the bound)
 constexpr unsigned kChunkPad = 4096;
-constexpr unsigned kBigCell = 8;
+#ifndef SJ_BIGCELL
+#define SJ_BIGCELL 8
+#endif
+constexpr unsigned kBigCell = SJ_BIGCELL;
 
 namespace sj {
 
